@@ -1,0 +1,44 @@
+"""CPU oracle for the FMHA forward pass and the GEMM+bias+activation block.
+
+TEST INFRASTRUCTURE ONLY.  Nothing in the product path (the CUDA library under
+``paper_conf_asplos_hagedornfccgg23_b200/csrc`` and its Python binding) may
+import, call, link or execute anything in this package.  The only permitted
+callers are ``tests/``, ``__graft_entry__.smoke()`` and the ``cpu_baseline`` /
+``--impl reference`` legs of ``bench.py``.
+
+The oracle shares no code with the CUDA path: no kernels, headers, helpers,
+constants or pre/post-processing.  Inputs come from ``workloads`` (seeded
+generators that hold none of the method's arithmetic).
+
+Citation key: ``P:Lnnn`` = line nnn of the paper text (Hagedorn et al.,
+"Graphene: An IR for Optimized Tensor Computations on GPUs", ASPLOS '23),
+section/figure named beside it.  ``DESIGN.md R<n>`` = a reading of the paper
+recorded in DESIGN.md §3 where the paper is silent.
+
+Modules
+-------
+fmha   numpy fp64, unfused GEMM -> softmax -> GEMM per (batch, head)   [pinned]
+brute  pure-Python scalar loops with math.fsum, tiny shapes only        [pinned]
+gemm   numpy fp64 act(A @ W^T + b)                                      [pinned]
+
+Every function is pinned by ``tests/test_oracle.py`` against closed forms,
+invariants, a hand-derived golden fixture (``tests/golden/``), brute force and
+torch's fp64 CPU ``scaled_dot_product_attention``.  There is no "parity
+unpinned" function in this package.
+"""
+
+from .fmha import attention_fp64, attention_rows_fp64, softmax_probs_fp64, fmha_flops
+from .brute import attention_brute
+from .gemm import gemm_bias_act_fp64, gelu_erf, gelu_tanh, relu
+
+__all__ = [
+    "attention_fp64",
+    "attention_rows_fp64",
+    "softmax_probs_fp64",
+    "fmha_flops",
+    "attention_brute",
+    "gemm_bias_act_fp64",
+    "gelu_erf",
+    "gelu_tanh",
+    "relu",
+]

@@ -1,0 +1,254 @@
+"""Pins for the CPU oracle (runs without a GPU).
+
+The oracle is pinned to things other than itself (SURVEY.md §8(c) pins P1-P13):
+closed forms, invariants, a hand-derived golden fixture, pure-Python brute force,
+and torch's float64 CPU scaled_dot_product_attention.  Each pin is chosen so a
+plausible slip in oracle/fmha.py (dropped scale, wrong sign in the max shift,
+transposed K, off-by-one causal diagonal, mask on the wrong axis) fails.
+"""
+
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+import torch
+
+from oracle import (attention_brute, attention_fp64, attention_rows_fp64, fmha_flops,
+                    gemm_bias_act_fp64, gelu_erf, gelu_tanh, softmax_probs_fp64)
+from oracle.gemm import ACT_GELU_ERF, ACT_GELU_TANH, ACT_NONE, ACT_RELU
+from workloads import CONFIGS, make_fmha_inputs
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden", "fmha_hand.json")
+
+
+def rnd(shape, seed, sigma=1.0):
+    return np.random.default_rng(seed).standard_normal(shape) * sigma
+
+
+# ---------------------------------------------------------------- golden (hand-derived)
+@pytest.mark.parametrize("case", json.load(open(GOLDEN))["cases"], ids=lambda c: c["name"])
+def test_golden_hand_cases(case):
+    o = attention_fp64(np.array(case["q"]), np.array(case["k"]), np.array(case["v"]),
+                       case["scale"], case["kv_len"], case["causal"])
+    np.testing.assert_allclose(o, np.array(case["expected"]), atol=1e-12, rtol=0)
+    ob = attention_brute(case["q"], case["k"], case["v"], case["scale"], case["kv_len"], case["causal"])
+    np.testing.assert_allclose(np.array(ob), np.array(case["expected"]), atol=1e-12, rtol=0)
+
+
+# ---------------------------------------------------------------- P11 closed form S=2, D=1
+@pytest.mark.parametrize("a,b,v0,v1", [(0.3, -1.2, 2.0, -5.0), (10.0, 9.0, 1.0, 0.0), (-3, 4, 0.5, 0.25)])
+def test_p11_two_keys_closed_form(a, b, v0, v1):
+    q = np.array([[[[1.0]]]])
+    k = np.array([[[[a], [b]]]])
+    v = np.array([[[[v0], [v1]]]])
+    want = (v0 * math.exp(a) + v1 * math.exp(b)) / (math.exp(a) + math.exp(b))
+    assert attention_fp64(q, k, v, 1.0)[0, 0, 0, 0] == pytest.approx(want, abs=1e-14)
+
+
+# ---------------------------------------------------------------- P11 brute force vs numpy
+@pytest.mark.parametrize("seed", range(6))
+def test_p11_brute_force_small(seed):
+    r = np.random.default_rng(100 + seed)
+    b, h = 2, 2
+    sq, skv, d = int(r.integers(1, 9)), int(r.integers(1, 9)), int(r.integers(1, 9))
+    causal = bool(seed % 2)
+    kv_len = None if seed % 3 else [int(r.integers(0, skv + 1)) for _ in range(b)]
+    q, k, v = rnd((b, h, sq, d), seed), rnd((b, h, skv, d), seed + 50), rnd((b, h, skv, d), seed + 99)
+    scale = 1 / math.sqrt(d)
+    o = attention_fp64(q, k, v, scale, kv_len, causal)
+    ob = np.array(attention_brute(q.tolist(), k.tolist(), v.tolist(), scale, kv_len, causal))
+    np.testing.assert_allclose(o, ob, atol=1e-12, rtol=1e-12)
+
+
+# ---------------------------------------------------------------- P12 library special case
+@pytest.mark.parametrize("causal,pad", [(False, False), (True, False), (False, True), (True, True)])
+def test_p12_torch_sdpa_fp64(causal, pad):
+    b, h, sq, skv, d = 3, 2, 37, 53, 16
+    q, k, v = rnd((b, h, sq, d), 1), rnd((b, h, skv, d), 2), rnd((b, h, skv, d), 3)
+    kv_len = [53, 20, 41] if pad else None
+    scale = 0.3
+    o = attention_fp64(q, k, v, scale, kv_len, causal)
+    i = np.arange(sq)[:, None]
+    j = np.arange(skv)[None, :]
+    vis = np.ones((b, 1, sq, skv), dtype=bool)
+    if causal:
+        vis &= (j <= i + (skv - sq))[None, None]
+    if pad:
+        for bb in range(b):
+            vis[bb, :, :, kv_len[bb]:] = False
+    ref = torch.nn.functional.scaled_dot_product_attention(
+        torch.from_numpy(q), torch.from_numpy(k), torch.from_numpy(v),
+        attn_mask=torch.from_numpy(vis), scale=float(np.float32(scale))).numpy()
+    rows = np.broadcast_to(vis.any(-1), (b, h, sq))  # SDPA gives NaN on fully masked rows
+    np.testing.assert_allclose(o[rows], ref[rows], atol=1e-12, rtol=1e-10)
+    assert np.all(o[~rows] == 0.0)
+
+
+# ---------------------------------------------------------------- P1 single key
+def test_p1_single_key_returns_v0():
+    q, k, v = rnd((2, 3, 5, 8), 4, 5.0), rnd((2, 3, 1, 8), 5, 5.0), rnd((2, 3, 1, 8), 6)
+    o = attention_fp64(q, k, v, 0.7)
+    np.testing.assert_array_equal(o, np.broadcast_to(v, o.shape))
+    # kv_len = 1 reduces to the same thing
+    k2, v2 = rnd((2, 3, 9, 8), 7), rnd((2, 3, 9, 8), 8)
+    o2 = attention_fp64(q, k2, v2, 0.7, kv_len=[1, 1])
+    np.testing.assert_allclose(o2, np.broadcast_to(v2[:, :, :1], o2.shape), atol=0, rtol=0)
+
+
+# ---------------------------------------------------------------- P2 constant Q,K with huge scores
+@pytest.mark.parametrize("mag", [1.0, 100.0, 1e4])
+def test_p2_constant_qk_gives_mean_of_visible_v(mag):
+    sq, skv, d = 6, 11, 4
+    q = np.full((1, 1, sq, d), mag)
+    k = np.full((1, 1, skv, d), mag)
+    v = rnd((1, 1, skv, d), 9)
+    o = attention_fp64(q, k, v, 1.0)          # scores = 4*mag^2, up to 4e8: needs max-shift
+    assert np.all(np.isfinite(o))
+    np.testing.assert_allclose(o[0, 0], np.broadcast_to(v[0, 0].mean(0), (sq, d)), atol=1e-12)
+    o = attention_fp64(q, k, v, 1.0, kv_len=[5])
+    np.testing.assert_allclose(o[0, 0], np.broadcast_to(v[0, 0, :5].mean(0), (sq, d)), atol=1e-12)
+    o = attention_fp64(q, k[:, :, :sq], v[:, :, :sq], 1.0, causal=True)
+    for i in range(sq):
+        np.testing.assert_allclose(o[0, 0, i], v[0, 0, :i + 1].mean(0), atol=1e-12)
+
+
+# ---------------------------------------------------------------- P3 uniform V
+def test_p3_uniform_v_identity():
+    q, k = rnd((2, 2, 7, 5), 10, 3.0), rnd((2, 2, 13, 5), 11, 3.0)
+    vrow = rnd((5,), 12)
+    v = np.broadcast_to(vrow, (2, 2, 13, 5)).copy()
+    for kw in ({}, {"causal": True}, {"kv_len": [3, 13]}):
+        o = attention_fp64(q, k, v, 0.4, **kw)
+        np.testing.assert_allclose(o, np.broadcast_to(vrow, o.shape), atol=1e-13)
+
+
+# ---------------------------------------------------------------- P4 scale = 0
+def test_p4_scale_zero_gives_mean():
+    q, k, v = rnd((1, 2, 4, 6), 13, 9.0), rnd((1, 2, 10, 6), 14, 9.0), rnd((1, 2, 10, 6), 15)
+    o = attention_fp64(q, k, v, 0.0)
+    np.testing.assert_allclose(o, np.broadcast_to(v.mean(2, keepdims=True), o.shape), atol=1e-13)
+
+
+# ---------------------------------------------------------------- P5 / P6 permutations
+def test_p5_joint_kv_permutation_invariance():
+    q, k, v = rnd((2, 2, 9, 8), 16), rnd((2, 2, 17, 8), 17), rnd((2, 2, 17, 8), 18)
+    perm = np.random.default_rng(0).permutation(17)
+    o = attention_fp64(q, k, v, 0.35)
+    op = attention_fp64(q, k[:, :, perm], v[:, :, perm], 0.35)
+    np.testing.assert_allclose(o, op, atol=1e-13)
+    # within the valid prefix under key padding
+    perm2 = np.concatenate([np.random.default_rng(1).permutation(10), np.arange(10, 17)])
+    o = attention_fp64(q, k, v, 0.35, kv_len=[10, 10])
+    op = attention_fp64(q, k[:, :, perm2], v[:, :, perm2], 0.35, kv_len=[10, 10])
+    np.testing.assert_allclose(o, op, atol=1e-13)
+    # a K-only permutation must change the result (catches a kernel/oracle ignoring K order)
+    assert not np.allclose(attention_fp64(q, k[:, :, perm], v, 0.35), o)
+
+
+def test_p6_query_permutation_equivariance():
+    q, k, v = rnd((1, 3, 12, 8), 19), rnd((1, 3, 12, 8), 20), rnd((1, 3, 12, 8), 21)
+    perm = np.random.default_rng(2).permutation(12)
+    o = attention_fp64(q, k, v, 0.5)
+    np.testing.assert_allclose(attention_fp64(q[:, :, perm], k, v, 0.5), o[:, :, perm], atol=1e-13)
+
+
+# ---------------------------------------------------------------- P7 masked rows are inert
+def test_p7_garbage_in_masked_kv_rows():
+    q, k, v = rnd((2, 2, 8, 8), 22), rnd((2, 2, 16, 8), 23), rnd((2, 2, 16, 8), 24)
+    kv_len = [5, 16]
+    o = attention_fp64(q, k, v, 0.35, kv_len=kv_len)
+    k2, v2 = k.copy(), v.copy()
+    k2[0, :, 5:] = 6e4
+    v2[0, :, 5:] = -6e4
+    np.testing.assert_array_equal(attention_fp64(q, k2, v2, 0.35, kv_len=kv_len), o)
+    # causal: keys after the diagonal are inert
+    qc, kc, vc = q[:, :, :8], k[:, :, :8].copy(), v[:, :, :8].copy()
+    oc = attention_fp64(qc, kc, vc, 0.35, causal=True)
+    kc[:, :, 7] = 6e4
+    vc[:, :, 7] = 6e4
+    np.testing.assert_array_equal(attention_fp64(qc, kc, vc, 0.35, causal=True)[:, :, :7], oc[:, :, :7])
+
+
+# ---------------------------------------------------------------- P8 convex hull, P9 rows sum to 1
+def test_p8_p9_convexity():
+    q, k, v = rnd((1, 1, 20, 8), 25, 3.0), rnd((1, 1, 30, 8), 26, 3.0), rnd((1, 1, 30, 8), 27)
+    for kw in ({}, {"causal": True}, {"kv_len": [17]}):
+        p = softmax_probs_fp64(q[0, 0], k[0, 0], 0.2, kw.get("kv_len", [None])[0], kw.get("causal", False))
+        assert np.all(p >= 0)
+        np.testing.assert_allclose(p.sum(1), 1.0, atol=1e-12)
+        o = attention_fp64(q, k, v, 0.2, **kw)[0, 0]
+        assert np.all(o <= v[0, 0].max(0) + 1e-12) and np.all(o >= v[0, 0].min(0) - 1e-12)
+
+
+# ---------------------------------------------------------------- P10 row score shift
+def test_p10_row_shift_invariance():
+    q, k, v = rnd((1, 2, 6, 8), 28), rnd((1, 2, 9, 8), 29), rnd((1, 2, 9, 8), 30)
+    outs = []
+    for c in (0.0, 37.0):
+        q2, k2 = q.copy(), k.copy()
+        q2[..., 7] = c
+        k2[..., 7] = 1.0
+        outs.append(attention_fp64(q2, k2, v, 0.5))
+    np.testing.assert_allclose(outs[0], outs[1], atol=1e-12)
+
+
+# ---------------------------------------------------------------- sampled rows == full oracle
+def test_rows_sampler_matches_full():
+    cfg = CONFIGS["bert_base_pad"].with_(batch=3, heads=2, seq_q=40, seq_kv=40)
+    q, k, v, kl = make_fmha_inputs(cfg)
+    full = attention_fp64(q, k, v, cfg.scale, kl)
+    units = [(0, 1, 3), (2, 0, 39), (1, 1, 0)]
+    rows = attention_rows_fp64(q, k, v, cfg.scale, units, kl)
+    for n, (b, h, i) in enumerate(units):
+        np.testing.assert_allclose(rows[n], full[b, h, i], atol=1e-14)
+    fullc = attention_fp64(q, k, v, cfg.scale, causal=True)
+    rowsc = attention_rows_fp64(q, k, v, cfg.scale, units, causal=True)
+    for n, (b, h, i) in enumerate(units):
+        np.testing.assert_allclose(rowsc[n], fullc[b, h, i], atol=1e-14)
+
+
+def test_flop_count():
+    assert fmha_flops(1, 1, 4, 4, 8) == 4 * 8 * 16
+    assert fmha_flops(1, 1, 4, 4, 8, causal=True) == 4 * 8 * 10            # 1+2+3+4
+    assert fmha_flops(2, 3, 4, 6, 8, kv_len=[2, 6]) == 4 * 8 * 3 * (4 * 2 + 4 * 6)
+    assert fmha_flops(1, 1, 3, 2, 1, causal=True) == 4 * (0 + 1 + 2)        # bottom-right
+
+
+# ---------------------------------------------------------------- P13 gemm pins
+def test_p13_gemm_pins():
+    r = np.random.default_rng(31)
+    a = r.uniform(-1, 1, (7, 5))
+    b = r.uniform(-1, 1, 5)
+    eye = np.eye(5)
+    np.testing.assert_allclose(gemm_bias_act_fp64(a, eye, b, ACT_NONE), a + b, atol=1e-15)
+    np.testing.assert_allclose(gemm_bias_act_fp64(a, eye, b, ACT_RELU), np.maximum(a + b, 0), atol=1e-15)
+    np.testing.assert_allclose(gemm_bias_act_fp64(np.zeros((3, 5)), r.normal(size=(5, 5)), b, ACT_GELU_ERF),
+                               np.broadcast_to(gelu_erf(b), (3, 5)), atol=1e-15)
+    x = np.linspace(-6, 6, 101)
+    np.testing.assert_allclose(gelu_erf(x) - gelu_erf(-x), x, atol=1e-14)
+    np.testing.assert_allclose(gelu_tanh(x) - gelu_tanh(-x), x, atol=1e-14)
+    # GELU known values: gelu(1) = Phi(1) = 0.8413447460685429; tanh form within 1e-3 of erf form
+    assert gelu_erf(np.array([1.0]))[0] == pytest.approx(0.8413447460685429, abs=1e-15)
+    assert np.max(np.abs(gelu_tanh(x) - gelu_erf(x))) < 1e-3
+    w = r.normal(size=(6, 5))
+    bias6 = r.normal(size=6)
+    ref = torch.nn.functional.linear(torch.from_numpy(a), torch.from_numpy(w), torch.from_numpy(bias6)).numpy()
+    np.testing.assert_allclose(gemm_bias_act_fp64(a, w, bias6, ACT_NONE), ref, atol=1e-13)
+    np.testing.assert_allclose(gemm_bias_act_fp64(a, w, None, ACT_GELU_TANH),
+                               torch.nn.functional.gelu(torch.from_numpy(a @ w.T), approximate="tanh").numpy(),
+                               atol=1e-14)
+    np.testing.assert_allclose(gemm_bias_act_fp64(a, w, None, ACT_GELU_ERF),
+                               torch.nn.functional.gelu(torch.from_numpy(a @ w.T)).numpy(), atol=1e-14)
+
+
+# ---------------------------------------------------------------- workload generator sanity
+def test_workloads_shard_reproducible():
+    cfg = CONFIGS["bert_base_pad"].with_(batch=4, heads=2, seq_q=16, seq_kv=16)
+    q, k, v, kl = make_fmha_inputs(cfg)
+    q2, k2, v2, kl2 = make_fmha_inputs(cfg.with_(batch=2), batch_offset=2)
+    assert torch.equal(q[2:], q2) and torch.equal(v[2:], v2)
+    assert list(kl[2:]) == list(kl2)
+    assert kl[0] == 16 and all(16 >= x >= 16 for x in kl[:1])
+    assert q.dtype == torch.float16

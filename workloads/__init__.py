@@ -1,0 +1,146 @@
+"""Seeded synthetic workloads shared by the tests, the bench and smoke().
+
+This module holds NONE of the method's arithmetic: it only defines the shapes of
+BASELINE.json's configs and draws seeded random inputs, rounded (RNE) to the I/O
+dtype.  Both the CUDA path and the oracle consume what it produces; neither is
+imported here.
+
+Recipe:
+  * seed 20230325 (the paper's conference date); every (b, h) slice of every
+    tensor is drawn from its own ``SeedSequence([seed, cfg_id, tensor_id, b, h])``
+    so a shard (a contiguous range of b) reproduces the global tensor exactly;
+  * Q, K ~ N(0, 1) (scaled scores ~ N(0, 1) at scale = 1/sqrt(D)); V ~ U(-1, 1),
+    so |O| <= 1; the stress variant draws Q, K ~ N(0, 3^2);
+  * drawn in float32, then rounded to fp16 / bf16 with round-to-nearest-even;
+  * key padding (BERT-base config): kv_len[b] ~ U{32..S}, with kv_len[0] = S so
+    at least one batch is unpadded;
+  * MLP: A ~ U(-1, 1), W ~ N(0, 1/K), b ~ U(-1, 1).
+"""
+
+from __future__ import annotations
+
+from dataclasses import dataclass, replace
+
+import numpy as np
+import torch
+
+SEED = 20230325
+
+MASK_NONE, MASK_KEY_PADDING, MASK_CAUSAL = 0, 1, 2
+
+
+@dataclass(frozen=True)
+class FmhaConfig:
+    name: str
+    cfg_id: int
+    batch: int
+    heads: int
+    seq_q: int
+    seq_kv: int
+    head_dim: int
+    dtype: str          # "fp16" | "bf16"
+    mask: int = MASK_NONE
+    qk_sigma: float = 1.0
+
+    @property
+    def units(self) -> int:
+        return self.batch * self.heads
+
+    @property
+    def scale(self) -> float:
+        return float(np.float32(1.0 / np.sqrt(self.head_dim)))
+
+    @property
+    def torch_dtype(self):
+        return torch.float16 if self.dtype == "fp16" else torch.bfloat16
+
+    def with_(self, **kw) -> "FmhaConfig":
+        return replace(self, **kw)
+
+
+# BASELINE.json "configs" (BJ:L7-L11)
+CONFIGS = {
+    "tiny": FmhaConfig("tiny", 1, 1, 1, 64, 64, 64, "fp16"),
+    "bert_base_pad": FmhaConfig("bert_base_pad", 2, 32, 12, 128, 128, 64, "fp16", MASK_KEY_PADDING),
+    "bert_large_384": FmhaConfig("bert_large_384", 3, 32, 16, 384, 384, 64, "fp16"),
+    "bert_large_512": FmhaConfig("bert_large_512", 4, 32, 16, 512, 512, 64, "fp16"),
+    "gpt_causal": FmhaConfig("gpt_causal", 5, 8, 32, 2048, 2048, 128, "bf16", MASK_CAUSAL),
+}
+
+
+@dataclass(frozen=True)
+class MlpConfig:
+    name: str
+    cfg_id: int
+    tokens: int
+    d_model: int
+    d_ff: int
+    dtype: str = "fp16"
+
+
+MLP_CONFIG = MlpConfig("mlp", 6, 16384, 1024, 4096)
+
+
+def _round(x32: np.ndarray, tdtype) -> torch.Tensor:
+    # torch's float32 -> fp16/bf16 conversion is round-to-nearest-even
+    return torch.from_numpy(np.ascontiguousarray(x32, dtype=np.float32)).to(tdtype)
+
+
+def _rng(cfg_id: int, tensor_id: int, b: int, h: int, seed: int = SEED):
+    return np.random.default_rng(np.random.SeedSequence([seed, cfg_id, tensor_id, b, h]))
+
+
+def kv_lengths(cfg: FmhaConfig, batch_offset: int = 0, seed: int = SEED) -> np.ndarray | None:
+    """Per-batch valid key count for key-padding configs (right padding)."""
+    if cfg.mask != MASK_KEY_PADDING:
+        return None
+    out = np.empty(cfg.batch, dtype=np.int32)
+    for b in range(cfg.batch):
+        gb = b + batch_offset
+        if gb == 0:
+            out[b] = cfg.seq_kv
+        else:
+            lo = min(32, cfg.seq_kv)
+            out[b] = _rng(cfg.cfg_id, 9, gb, 0, seed).integers(lo, cfg.seq_kv + 1)
+    return out
+
+
+def make_fmha_inputs(cfg: FmhaConfig, batch_offset: int = 0, seed: int = SEED):
+    """Returns (q, k, v, kv_len) as CPU torch tensors [B,H,S,D] in cfg's dtype
+    (kv_len: int32 numpy array or None).  Global batch index = b + batch_offset."""
+    b_, h_, sq, skv, d = cfg.batch, cfg.heads, cfg.seq_q, cfg.seq_kv, cfg.head_dim
+    q = np.empty((b_, h_, sq, d), dtype=np.float32)
+    k = np.empty((b_, h_, skv, d), dtype=np.float32)
+    v = np.empty((b_, h_, skv, d), dtype=np.float32)
+    for b in range(b_):
+        gb = b + batch_offset
+        for h in range(h_):
+            q[b, h] = _rng(cfg.cfg_id, 0, gb, h, seed).standard_normal((sq, d), dtype=np.float32) * cfg.qk_sigma
+            k[b, h] = _rng(cfg.cfg_id, 1, gb, h, seed).standard_normal((skv, d), dtype=np.float32) * cfg.qk_sigma
+            v[b, h] = _rng(cfg.cfg_id, 2, gb, h, seed).uniform(-1.0, 1.0, (skv, d)).astype(np.float32)
+    td = cfg.torch_dtype
+    return _round(q, td), _round(k, td), _round(v, td), kv_lengths(cfg, batch_offset, seed)
+
+
+def make_mlp_inputs(cfg: MlpConfig = MLP_CONFIG, tokens: int | None = None, seed: int = SEED):
+    """Returns (x [T,d_model], w1 [d_ff,d_model], b1 [d_ff], w2 [d_model,d_ff], b2 [d_model])
+    as fp16 CPU tensors."""
+    t = cfg.tokens if tokens is None else tokens
+    r = lambda tid: _rng(cfg.cfg_id, tid, 0, 0, seed)
+    x = r(0).uniform(-1, 1, (t, cfg.d_model)).astype(np.float32)
+    w1 = (r(1).standard_normal((cfg.d_ff, cfg.d_model), dtype=np.float32) / np.sqrt(cfg.d_model)).astype(np.float32)
+    b1 = r(2).uniform(-1, 1, cfg.d_ff).astype(np.float32)
+    w2 = (r(3).standard_normal((cfg.d_model, cfg.d_ff), dtype=np.float32) / np.sqrt(cfg.d_ff)).astype(np.float32)
+    b2 = r(4).uniform(-1, 1, cfg.d_model).astype(np.float32)
+    td = torch.float16
+    return tuple(_round(a, td) for a in (x, w1, b1, w2, b2))
+
+
+def make_gemm_inputs(m: int, n: int, k: int, seed: int = SEED, cfg_id: int = 7):
+    """Generic GEMM+bias test inputs: A ~ U(-1,1) [M,K], W ~ N(0,1/K) [N,K], b ~ U(-1,1) [N]."""
+    r = lambda tid: _rng(cfg_id, tid, m, n * 100003 + k, seed)
+    a = r(0).uniform(-1, 1, (m, k)).astype(np.float32)
+    w = (r(1).standard_normal((n, k), dtype=np.float32) / np.sqrt(max(k, 1))).astype(np.float32)
+    b = r(2).uniform(-1, 1, n).astype(np.float32)
+    td = torch.float16
+    return _round(a, td), _round(w, td), _round(b, td)
