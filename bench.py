@@ -1,0 +1,338 @@
+#!/usr/bin/env python
+"""Benchmark: FMHA forward TFLOP/s at BERT-large shapes (BASELINE.json metric) on N GPUs.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--workload NAME]
+
+A step is one pass of the whole hot path (one fmha_fwd launch through the C ABI) over one batch
+of the workload (default bert_large_512: B=32, H=16, S=512, D=64, fp16).  N > 1 runs under
+torchrun, one process per GPU; every rank processes its own batch (weak scaling, no collective
+on the data path); value = all ranks' algorithmic flops / max-over-ranks device time.
+
+Rank 0 prints ONE JSON line.  See DESIGN.md §6 for every field.
+"""
+
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+from workloads import CONFIGS, MASK_CAUSAL, MASK_KEY_PADDING, make_fmha_inputs  # noqa: E402
+
+METRIC = "FMHA fwd TFLOP/s & % of B200 fp16 tensor peak at BERT-large shapes, 1/2/4/8 GPU"
+SPEC_TFLOPS = 2250.0
+L2_BYTES = 126 * 1024 * 1024
+
+
+def alg_flops(cfg, kv_len) -> float:
+    """4*D per visible (query, key) pair — SURVEY §8(d); masked pairs are not counted."""
+    b, h, sq, skv, d = cfg.batch, cfg.heads, cfg.seq_q, cfg.seq_kv, cfg.head_dim
+    if cfg.mask == MASK_CAUSAL:
+        off = skv - sq
+        i = np.arange(sq)
+        pairs = int(np.clip(np.minimum(skv, i + off + 1), 0, None).sum()) * b * h
+    elif cfg.mask == MASK_KEY_PADDING:
+        pairs = int(sum(sq * min(int(x), skv) for x in kv_len)) * h
+    else:
+        pairs = b * h * sq * skv
+    return 4.0 * d * pairs
+
+
+def alg_bytes(cfg) -> float:
+    e = 2
+    return float(e * cfg.batch * cfg.heads * cfg.head_dim * (2 * cfg.seq_q + 2 * cfg.seq_kv))
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d["bf16_tflops"], d.get("bf16_tflops_sustained"), d["hbm_gbs"], "measured"
+    return 1590.0, 1400.0, 6650.0, "fallback"
+
+
+class ClockSampler:
+    """Samples SM clock and throttle reasons through NVML while the timed region runs."""
+
+    REASONS = {
+        "gpu_idle": 0x1, "applications_clocks_setting": 0x2, "sw_power_cap": 0x4, "hw_slowdown": 0x8,
+        "sync_boost": 0x10, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
+        "hw_power_brake_slowdown": 0x80, "display_clock_setting": 0x100,
+    }
+
+    def __init__(self, index: int):
+        self.samples, self.reasons, self.ok = [], set(), False
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            self.max_mhz = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksThrottleReasons(self.h)
+                for k, bit in self.REASONS.items():
+                    if r & bit and k != "gpu_idle":
+                        self.reasons.add(k)
+            except Exception:
+                pass
+            time.sleep(0.002)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def cpu_oracle_sample(cfg, q, k, v, kv_len, budget_s: float):
+    """Times the CPU oracle (as it stands) on whole (b,h) units of this workload until ~budget_s."""
+    from oracle import attention_fp64
+    try:
+        from threadpoolctl import threadpool_info
+        cores = max([t.get("num_threads", 1) for t in threadpool_info()] or [1])
+    except Exception:
+        cores = os.cpu_count()
+    done_flops, units, t0 = 0.0, 0, time.perf_counter()
+    causal = cfg.mask == MASK_CAUSAL
+    while True:
+        b, h = divmod(units % cfg.units, cfg.heads)
+        kl = None if kv_len is None else [int(kv_len[b])]
+        attention_fp64(q[b:b + 1, h:h + 1], k[b:b + 1, h:h + 1], v[b:b + 1, h:h + 1], cfg.scale, kl, causal)
+        done_flops += alg_flops(cfg.with_(batch=1, heads=1), kl)
+        units += 1
+        el = time.perf_counter() - t0
+        if el >= budget_s or units >= cfg.units:
+            break
+    return {"value": done_flops / el / 1e12, "unit": "TFLOP/s", "cores": int(cores), "kind": "oracle",
+            "sample": f"{units} of {cfg.units} (b,h) units of {cfg.name}, numpy fp64, {el:.1f} s"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--workload", default="bert_large_512", choices=sorted(CONFIGS))
+    ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of CPU oracle timing")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    cfg = CONFIGS[args.workload]
+
+    if args.impl == "reference":
+        return run_reference(args, cfg, world, rank)
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+
+    import paper_conf_asplos_hagedornfccgg23_b200 as fm
+
+    q, k, v, kv_len = make_fmha_inputs(cfg, batch_offset=rank * cfg.batch)  # weak scaling: own batch
+    set_bytes = alg_bytes(cfg)
+    n_sets = max(1, int(np.ceil(3 * L2_BYTES / set_bytes)))  # rotate > 3x L2 of inputs+outputs
+    qd, kd, vd = q.to(dev), k.to(dev), v.to(dev)
+    sets = [(qd, kd, vd, torch.empty_like(qd))] + [
+        (qd.clone(), kd.clone(), vd.clone(), torch.empty_like(qd)) for _ in range(n_sets - 1)]
+    kl_dev = None if kv_len is None else torch.from_numpy(kv_len).to(dev)
+    causal = cfg.mask == MASK_CAUSAL
+    stream = torch.cuda.current_stream(dev)
+
+    def step(i):
+        s = sets[i % n_sets]
+        fm.fmha_fwd(s[0], s[1], s[2], kv_len=kl_dev, causal=causal, scale=cfg.scale, out=s[3])
+
+    for i in range(args.warmup):
+        step(i)
+    torch.cuda.synchronize()
+    # The K timed steps are captured once into a CUDA graph (K kernel launches, rotating input sets)
+    # so host-side launch overhead cannot starve a ~tens-of-microseconds kernel.  One untimed replay
+    # uploads the graph before the timed replay.
+    graph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(graph):
+        for i in range(args.steps):
+            step(i)
+    graph.replay()
+    torch.cuda.synchronize()
+
+    sampler = ClockSampler(local)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with sampler:
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+        ev0.record(stream)
+        graph.replay()
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        if dist:
+            dist.barrier()
+    ms = ev0.elapsed_time(ev1)
+    if dist:
+        t = torch.tensor([ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    flops_rank = alg_flops(cfg, kv_len)
+    ms_step = ms / args.steps
+    value = flops_rank * world / (ms_step * 1e-3) / 1e12
+
+    # ---- end to end through the C ABI with pinned HOST buffers (copies inside the timed region)
+    e2e = None
+    if not args.no_e2e:
+        pq, pk, pv = q.pin_memory(), k.pin_memory(), v.pin_memory()
+        po = torch.empty_like(pq).pin_memory()
+        ws = torch.empty(fm.workspace_bytes(cfg.batch, cfg.heads, cfg.seq_q, cfg.seq_kv, cfg.head_dim),
+                         dtype=torch.uint8, device=dev)
+        klh = None if kv_len is None else torch.from_numpy(kv_len).pin_memory()
+        e2e_steps = max(3, min(args.steps, 20))
+        for _ in range(2):
+            fm.fmha_fwd_from_host(pq, pk, pv, po, ws, kv_len=klh, causal=causal, scale=cfg.scale, stream=stream)
+        torch.cuda.synchronize()
+        if dist:
+            dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(e2e_steps):
+            fm.fmha_fwd_from_host(pq, pk, pv, po, ws, kv_len=klh, causal=causal, scale=cfg.scale, stream=stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ems = e0.elapsed_time(e1)
+        if dist:
+            t = torch.tensor([ems], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ems = float(t.item())
+        in_bytes = (pq.numel() + pk.numel() + pv.numel()) * pq.element_size() + (0 if klh is None else klh.numel() * 4)
+        e2e = {"value": flops_rank * world / (ems / e2e_steps * 1e-3) / 1e12, "unit": "TFLOP/s",
+               "h2d_bytes_per_step": int(in_bytes), "d2h_bytes_per_step": int(po.numel() * po.element_size()),
+               "ms_per_step": ems / e2e_steps}
+
+    # ---- check this rank's last output against sampled oracle rows (cheap sanity, not timed)
+    from oracle import attention_rows_fp64
+    units = [(0, 0, 0), (cfg.batch - 1, cfg.heads - 1, cfg.seq_q - 1), (cfg.batch // 2, 1, cfg.seq_q // 3)]
+    ref = attention_rows_fp64(q, k, v, cfg.scale, units, kv_len, causal)
+    o_last = sets[(args.steps - 1) % n_sets][3]
+    got = np.stack([o_last[b, h, i].double().cpu().numpy() for b, h, i in units])
+    check_err = float(np.abs(got - ref).max())
+
+    peak_burst, peak_sust, hbm, peak_src = measured_peaks()
+    if dist:
+        dist.barrier()
+    if rank == 0:
+        cpu = None
+        if world == 1 and not args.no_cpu_baseline:
+            cpu = cpu_oracle_sample(cfg, q, k, v, kv_len, args.cpu_budget)
+        traffic = None
+        tp = os.path.join(ROOT, "profiles", "traffic.json")
+        if os.path.exists(tp):
+            traffic = json.load(open(tp)).get(cfg.name)
+        achieved = flops_rank / (ms_step * 1e-3) / 1e12  # per-GPU kernel throughput (1 launch / step)
+        line = {
+            "metric": METRIC, "value": round(value, 2), "unit": "TFLOP/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 5),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "f16" if cfg.dtype == "fp16" else "bf16", "data": "synthetic",
+            "config": {"workload": cfg.name, "batch_per_gpu": cfg.batch, "heads": cfg.heads, "seq_q": cfg.seq_q,
+                       "seq_kv": cfg.seq_kv, "head_dim": cfg.head_dim,
+                       "mask": ["none", "key_padding", "causal"][cfg.mask], "parallelism": f"dp{world} (b x h shards)",
+                       "l2": f"rotating {n_sets} input/output sets ({n_sets * set_bytes / 1e6:.0f} MB > 126 MB L2)"},
+            "pct_of_spec_2250": round(100 * achieved / SPEC_TFLOPS, 2),
+            "pct_of_measured_peak": round(100 * achieved / peak_burst, 2),
+            "achieved_gbs": round(alg_bytes(cfg) / (ms_step * 1e-3) / 1e9, 1),
+            "clocks": sampler.summary(),
+            "e2e": e2e,
+            "gpu_launches": args.steps,
+            "roofline": {"bound": "tensor", "achieved": round(achieved, 2), "peak": peak_burst, "unit": "TFLOP/s",
+                         "frac": round(achieved / peak_burst, 4), "traffic": traffic,
+                         "peak_source": f"{peak_src} bf16 dense burst (fp16 = bf16 rate)",
+                         "kernel": "fmha_fwd_kernel"},
+            "cpu_baseline": cpu,
+            "check_max_abs_err": check_err,
+        }
+        print(json.dumps(line), flush=True)
+    if dist:
+        dist.destroy_process_group()
+
+
+def run_reference(args, cfg, world, rank):
+    """Reference arm for this tier = the CPU oracle, as it stands, on the host cores (rank 0 only)."""
+    if rank != 0:
+        return
+    q, k, v, kv_len = make_fmha_inputs(cfg)
+    from oracle import attention_fp64
+    causal = cfg.mask == MASK_CAUSAL
+    # each step: a bounded sample of the workload (a fixed number of whole (b,h) units)
+    per_unit = None
+    t0 = time.perf_counter()
+    attention_fp64(q[:1, :1], k[:1, :1], v[:1, :1], cfg.scale, None if kv_len is None else kv_len[:1], causal)
+    per_unit = time.perf_counter() - t0
+    per_step_s = min(2.0, 90.0 / max(1, args.steps + min(args.warmup, 3)))  # whole run ~<= 1.5 min
+    n_units = int(max(1, min(cfg.units, per_step_s / max(per_unit, 1e-6))))
+    sub = cfg.with_(batch=max(1, n_units // cfg.heads) if n_units >= cfg.heads else 1,
+                    heads=cfg.heads if n_units >= cfg.heads else n_units)
+    qs, ks, vs = q[:sub.batch, :sub.heads], k[:sub.batch, :sub.heads], v[:sub.batch, :sub.heads]
+    kls = None if kv_len is None else kv_len[:sub.batch]
+    for _ in range(args.warmup if args.warmup <= 3 else 3):
+        attention_fp64(qs, ks, vs, cfg.scale, kls, causal)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        attention_fp64(qs, ks, vs, cfg.scale, kls, causal)
+    el = time.perf_counter() - t0
+    val = alg_flops(sub, kls) * args.steps / el / 1e12
+    try:
+        from threadpoolctl import threadpool_info
+        cores = max([t.get("num_threads", 1) for t in threadpool_info()] or [1])
+    except Exception:
+        cores = os.cpu_count()
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "TFLOP/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": el / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "f64", "data": "synthetic",
+            "config": {"workload": cfg.name, "batch_per_gpu": cfg.batch, "heads": cfg.heads, "seq_q": cfg.seq_q,
+                       "seq_kv": cfg.seq_kv, "head_dim": cfg.head_dim,
+                       "mask": ["none", "key_padding", "causal"][cfg.mask]},
+            "cpu_baseline": {"value": val, "unit": "TFLOP/s", "cores": int(cores), "kind": "oracle",
+                             "sample": f"{sub.batch * sub.heads} of {cfg.units} (b,h) units of {cfg.name} per step"},
+            "e2e": {"value": val, "unit": "TFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,114 @@
+/* fmha.h — C ABI of libb200fmha: B200-native (sm_100a) fused multi-head attention forward and
+ * GEMM + bias + activation.
+ *
+ * Operation (paper §6 "Fused Multi-Head Attention": "two back-to-back GEMMs with a
+ * softmax computation in between"; shapes of MLPerf BERT inference, L489):
+ *
+ *     O[b,h,i,:] = sum_j softmax_j( scale * <Q[b,h,i,:], K[b,h,j,:]> + mask[b,i,j] ) * V[b,h,j,:]
+ *
+ * for every batch b < batch, head h < heads, query row i < seq_q, key j < seq_kv.
+ * Precision ("FP16 tensors using FP32 Tensor Core accumulation"): inputs and output
+ * fp16 (fmha_fwd) or bf16 (fmha_fwd_bf16); both GEMMs accumulate in fp32 on the tensor cores;
+ * the softmax runs in fp32; P is rounded to the I/O type before the second GEMM; O is rounded
+ * once, round-to-nearest-even.
+ *
+ * Layout: Q, O are [batch, heads, seq_q, head_dim] and K, V are [batch, heads, seq_kv, head_dim],
+ * dense row-major (head_dim contiguous), no padding between rows.
+ *
+ * Masks (the paper's FMHA has none; BASELINE.json configs add them; R3-R6):
+ *   FMHA_MASK_NONE         every key visible.
+ *   FMHA_MASK_KEY_PADDING  key j visible iff j < kv_len[b] (right padding, shared by all heads).
+ *                          kv_len is a DEVICE int32 array [batch]; values are clamped to [0, seq_kv].
+ *   FMHA_MASK_CAUSAL       key j visible iff j <= i + (seq_kv - seq_q)  (bottom-right aligned).
+ * A query row with no visible key produces O = 0 (never NaN).
+ *
+ * Ownership and errors: every tensor pointer is caller-owned; the library never allocates device
+ * memory, never synchronises the stream and retains no pointer past the call (kv_len must stay
+ * valid until the kernel completes, stream-ordered).  `mask` is read on the host during the call.
+ * Validation failures return a non-zero fmha_status_t before anything is launched; launch failures
+ * return FMHA_ERR_CUDA.  Device faults surface at the caller's next synchronisation.  The library
+ * is stateless and thread-safe (cached: the driver entry point for tensor-map encoding, per-device
+ * kernel attributes).  There is no CPU fallback: without an sm_100 device every entry point that
+ * launches returns FMHA_ERR_NO_DEVICE.
+ */
+#ifndef B200FMHA_FMHA_H
+#define B200FMHA_FMHA_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define FMHA_API __attribute__((visibility("default")))
+#else
+#define FMHA_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st* fmha_stream_t; /* == cudaStream_t; NULL = legacy default stream */
+
+typedef enum {
+  FMHA_OK = 0,
+  FMHA_ERR_INVALID_ARG = 1, /* null pointer, negative size, non-finite scale, ...            */
+  FMHA_ERR_UNSUPPORTED = 2, /* head_dim not in {64,128}, negative scale, unknown mask / act   */
+  FMHA_ERR_MISALIGNED = 3,  /* a tensor pointer is not 16-byte aligned (TMA requirement)       */
+  FMHA_ERR_CUDA = 4,        /* a CUDA runtime/driver call failed; see fmha_last_cuda_error()   */
+  FMHA_ERR_NO_DEVICE = 5    /* no sm_100 device is current                                    */
+} fmha_status_t;
+
+typedef enum { FMHA_MASK_NONE = 0, FMHA_MASK_KEY_PADDING = 1, FMHA_MASK_CAUSAL = 2 } fmha_mask_kind_t;
+
+typedef struct {
+  int32_t kind;          /* fmha_mask_kind_t                                          */
+  const int32_t* kv_len; /* DEVICE pointer, [batch]; required for KEY_PADDING, else ignored */
+} fmha_mask_t;
+
+/* FMHA forward, fp16 in / fp16 out.
+ *   Q, K, V, O : DEVICE pointers, 16-byte aligned, layouts above.
+ *   mask       : HOST pointer or NULL (= FMHA_MASK_NONE).
+ *   batch, heads, seq_q, seq_kv >= 0 (seq_kv >= 1 unless batch*heads*seq_q == 0);
+ *   head_dim   : 64 or 128.
+ *   scale      : finite, >= 0; usually 1/sqrt(head_dim).
+ *   stream     : CUDA stream the kernel is enqueued on.
+ * batch*heads*seq_q == 0 returns FMHA_OK without launching. */
+FMHA_API int fmha_fwd(const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask, int batch,
+             int heads, int seq_q, int seq_kv, int head_dim, float scale, fmha_stream_t stream);
+
+/* Identical contract with bf16 tensors. */
+FMHA_API int fmha_fwd_bf16(const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask, int batch,
+                  int heads, int seq_q, int seq_kv, int head_dim, float scale, fmha_stream_t stream);
+
+/* End-to-end variant: Q/K/V/O and kv_len are HOST buffers (pinned memory for asynchronous copies).
+ * Copies Q, K, V (and kv_len) host->device into `workspace`, runs the same kernel, copies O
+ * device->host, all enqueued on `stream` (no synchronisation: the caller syncs before reading O).
+ * dtype: 0 = fp16, 1 = bf16.  `workspace` is a DEVICE buffer of at least
+ * fmha_workspace_bytes(batch, heads, seq_q, seq_kv, head_dim) bytes, 256-byte aligned.
+ * For this entry point mask->kv_len is a HOST pointer. */
+FMHA_API size_t fmha_workspace_bytes(int batch, int heads, int seq_q, int seq_kv, int head_dim);
+FMHA_API int fmha_fwd_from_host(int dtype, const void* hQ, const void* hK, const void* hV, void* hO,
+                       const fmha_mask_t* mask, void* workspace, size_t workspace_bytes, int batch, int heads,
+                       int seq_q, int seq_kv, int head_dim, float scale, fmha_stream_t stream);
+
+/* GEMM + bias + activation, the MLP building block:
+ *     C[m,n] = act( sum_k A[m,k] * W[n,k] + bias[n] )
+ * A [M,K], W [N,K] (nn.Linear layout), bias [N] (or NULL), C [M,N]: fp16, row-major, DEVICE,
+ * 16-byte aligned; fp32 accumulation, bias and activation in fp32, one RNE rounding to fp16.
+ * Requires K % 8 == 0 and N % 8 == 0 (16-byte row pitch for TMA).
+ * act: 0 none, 1 ReLU, 2 GELU (erf), 3 GELU (tanh). */
+typedef enum { ACT_NONE = 0, ACT_RELU = 1, ACT_GELU_ERF = 2, ACT_GELU_TANH = 3 } fmha_act_t;
+FMHA_API int gemm_bias_act(const void* A, const void* W, const void* bias, void* C, int M, int N, int K, int act,
+                  fmha_stream_t stream);
+
+/* Human-readable text for a status code (static storage). */
+FMHA_API const char* fmha_status_string(int status);
+/* Text of the last CUDA error seen by this thread inside the library ("" if none). */
+FMHA_API const char* fmha_last_cuda_error(void);
+/* Library version string. */
+FMHA_API const char* fmha_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* B200FMHA_FMHA_H */

@@ -1,0 +1,125 @@
+"""B200-native (sm_100a) fused multi-head attention forward and GEMM+bias+activation.
+
+Python surface over the C ABI of ``lib/libb200fmha.so`` (include/fmha.h).  PyTorch provides
+device memory and streams only; every step of the computation runs in the hand-written CUDA
+kernels behind the ABI.  There is no CPU or library fallback: without the built library or an
+sm_100 device these functions raise.
+
+    fmha_fwd(q, k, v, kv_len=None, causal=False, scale=None, out=None) -> O
+    fmha_fwd_from_host(q, k, v, ..., workspace) -> O  (host tensors; copies inside the call)
+    gemm_bias_act(a, w, bias=None, act="none", out=None) -> C
+"""
+
+from __future__ import annotations
+
+import ctypes
+import math
+
+import torch
+
+from . import _lib
+from ._lib import FmhaError, FmhaMask
+
+__all__ = ["fmha_fwd", "fmha_fwd_from_host", "gemm_bias_act", "workspace_bytes", "FmhaError",
+           "MASK_NONE", "MASK_KEY_PADDING", "MASK_CAUSAL", "ACTS", "version"]
+
+MASK_NONE, MASK_KEY_PADDING, MASK_CAUSAL = 0, 1, 2
+ACTS = {"none": 0, "relu": 1, "gelu": 2, "gelu_erf": 2, "gelu_tanh": 3}
+
+
+def version() -> str:
+    return _lib.load().fmha_version().decode()
+
+
+def _stream_ptr(dev: torch.device) -> int:
+    return torch.cuda.current_stream(dev).cuda_stream
+
+
+def _mask(kv_len, causal: bool):
+    if kv_len is not None and causal:
+        raise ValueError("key padding and causal masks are mutually exclusive in this ABI")
+    if kv_len is not None:
+        return FmhaMask(MASK_KEY_PADDING, kv_len.data_ptr())
+    if causal:
+        return FmhaMask(MASK_CAUSAL, None)
+    return FmhaMask(MASK_NONE, None)
+
+
+def fmha_fwd(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, kv_len: torch.Tensor | None = None,
+             causal: bool = False, scale: float | None = None, out: torch.Tensor | None = None) -> torch.Tensor:
+    """O = softmax(scale * Q K^T + mask) V.  q: [B,H,Sq,D], k/v: [B,H,Skv,D] contiguous CUDA
+    fp16/bf16 tensors; kv_len: CUDA int32 [B] (key padding) or None; causal: bottom-right mask.
+    Calls ``fmha_fwd`` / ``fmha_fwd_bf16`` of the C ABI on the current stream."""
+    lib = _lib.load()
+    if q.dtype not in (torch.float16, torch.bfloat16) or k.dtype != q.dtype or v.dtype != q.dtype:
+        raise TypeError("q, k, v must share dtype fp16 or bf16")
+    if not (q.is_cuda and k.is_cuda and v.is_cuda):
+        raise TypeError("q, k, v must be CUDA tensors (no CPU fallback)")
+    if not (q.is_contiguous() and k.is_contiguous() and v.is_contiguous()):
+        raise ValueError("q, k, v must be contiguous [B,H,S,D]")
+    b, h, sq, d = q.shape
+    skv = k.shape[2]
+    if k.shape != (b, h, skv, d) or v.shape != k.shape:
+        raise ValueError(f"shape mismatch q{tuple(q.shape)} k{tuple(k.shape)} v{tuple(v.shape)}")
+    if kv_len is not None:
+        if kv_len.dtype != torch.int32 or not kv_len.is_cuda or kv_len.numel() != b:
+            raise ValueError("kv_len must be a CUDA int32 tensor of length batch")
+        kv_len = kv_len.contiguous()
+    if out is None:
+        out = torch.empty_like(q)
+    scale = 1.0 / math.sqrt(d) if scale is None else float(scale)
+    m = _mask(kv_len, causal)
+    fn = lib.fmha_fwd if q.dtype == torch.float16 else lib.fmha_fwd_bf16
+    st = fn(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), ctypes.byref(m), b, h, sq, skv, d,
+            scale, _stream_ptr(q.device))
+    _lib.check(st, "fmha_fwd")
+    return out
+
+
+def workspace_bytes(b: int, h: int, sq: int, skv: int, d: int) -> int:
+    return int(_lib.load().fmha_workspace_bytes(b, h, sq, skv, d))
+
+
+def fmha_fwd_from_host(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, out: torch.Tensor,
+                       workspace: torch.Tensor, kv_len: torch.Tensor | None = None, causal: bool = False,
+                       scale: float | None = None, stream: torch.cuda.Stream | None = None) -> torch.Tensor:
+    """End-to-end call with HOST (pinned) q/k/v/out and a device workspace: H2D copies, kernel and
+    D2H copy are all enqueued on ``stream`` by ``fmha_fwd_from_host`` of the C ABI (async; the
+    caller synchronises before reading ``out``)."""
+    lib = _lib.load()
+    b, h, sq, d = q.shape
+    skv = k.shape[2]
+    dt = {torch.float16: 0, torch.bfloat16: 1}[q.dtype]
+    m = FmhaMask(MASK_NONE, None)
+    if kv_len is not None:
+        m = FmhaMask(MASK_KEY_PADDING, kv_len.data_ptr())  # HOST int32 for this entry point
+    elif causal:
+        m = FmhaMask(MASK_CAUSAL, None)
+    scale = 1.0 / math.sqrt(d) if scale is None else float(scale)
+    s = stream if stream is not None else torch.cuda.current_stream(workspace.device)
+    st = lib.fmha_fwd_from_host(dt, q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), ctypes.byref(m),
+                                workspace.data_ptr(), workspace.numel() * workspace.element_size(), b, h, sq, skv,
+                                d, scale, s.cuda_stream)
+    _lib.check(st, "fmha_fwd_from_host")
+    return out
+
+
+def gemm_bias_act(a: torch.Tensor, w: torch.Tensor, bias: torch.Tensor | None = None, act: str = "none",
+                  out: torch.Tensor | None = None) -> torch.Tensor:
+    """C = act(A W^T + bias): a [M,K], w [N,K], bias [N] fp16 CUDA tensors -> [M,N] fp16."""
+    lib = _lib.load()
+    if a.dtype != torch.float16 or w.dtype != torch.float16 or (bias is not None and bias.dtype != torch.float16):
+        raise TypeError("gemm_bias_act takes fp16 tensors")
+    if not (a.is_cuda and w.is_cuda):
+        raise TypeError("CUDA tensors required (no CPU fallback)")
+    a, w = a.contiguous(), w.contiguous()
+    m_, k_ = a.shape
+    n_ = w.shape[0]
+    if w.shape[1] != k_:
+        raise ValueError("K mismatch")
+    if out is None:
+        out = torch.empty((m_, n_), dtype=torch.float16, device=a.device)
+    st = lib.gemm_bias_act(a.data_ptr(), w.data_ptr(), None if bias is None else bias.contiguous().data_ptr(),
+                           out.data_ptr(), m_, n_, k_, ACTS[act], _stream_ptr(a.device))
+    _lib.check(st, "gemm_bias_act")
+    return out

@@ -1,0 +1,266 @@
+// api.cu — the C ABI declared in include/fmha.h: argument validation, TMA tensor-map encoding,
+// kernel selection and launch.  No allocation, no synchronisation, no CPU fallback.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+
+#include "../../include/fmha.h"
+#include "fmha_kernel.cuh"
+#include "gemm_kernel.cuh"
+
+namespace {
+
+thread_local char g_last_cuda_error[256] = "";
+
+int cuda_fail(cudaError_t e, const char* where) {
+  snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "%s: %s", where, cudaGetErrorString(e));
+  return FMHA_ERR_CUDA;
+}
+
+using EncodeTiledFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn get_encode_fn() {
+  static EncodeTiledFn fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* ptr = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPointByVersion("cuTensorMapEncodeTiled", &ptr, 12000, cudaEnableDefault, &q) ==
+            cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncodeTiledFn>(ptr);
+  });
+  return fn;
+}
+
+// Checks that the current device is an sm_100 part.  Cached per device ordinal.
+int check_device(int* sm_count) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return FMHA_ERR_NO_DEVICE;
+  }
+  static int cached_major[64], cached_sms[64];
+  static bool cached[64];
+  if (dev < 64 && cached[dev]) {
+    if (sm_count) *sm_count = cached_sms[dev];
+    return cached_major[dev] == 10 ? FMHA_OK : FMHA_ERR_NO_DEVICE;
+  }
+  int major = 0, minor = 0, sms = 0;
+  if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev) != cudaSuccess ||
+      cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev) != cudaSuccess ||
+      cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) {
+    cudaGetLastError();
+    return FMHA_ERR_NO_DEVICE;
+  }
+  if (dev < 64) {
+    cached_major[dev] = (major == 10 && minor == 0) ? 10 : -1;
+    cached_sms[dev] = sms;
+    cached[dev] = true;
+  }
+  if (sm_count) *sm_count = sms;
+  return (major == 10 && minor == 0) ? FMHA_OK : FMHA_ERR_NO_DEVICE;
+}
+
+// 3-D tile map over a [units, rows, cols] row-major tensor of 16-bit elements.
+// Box = {64 cols (128 B, the SWIZZLE_128B span), box_rows, 1}.  OOB elements read as zero.
+int make_map_3d(CUtensorMap* m, const void* base, bool bf16, uint64_t cols, uint64_t rows, uint64_t units,
+                uint32_t box_rows) {
+  EncodeTiledFn enc = get_encode_fn();
+  if (!enc) {
+    snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "cuTensorMapEncodeTiled entry point unavailable");
+    return FMHA_ERR_CUDA;
+  }
+  cuuint64_t dims[3] = {cols, rows, units};
+  cuuint64_t strides[2] = {cols * 2, cols * rows * 2};
+  cuuint32_t box[3] = {64, box_rows, 1};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = enc(m, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 3,
+                   const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) {
+    snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "cuTensorMapEncodeTiled failed (%d)", int(r));
+    return FMHA_ERR_CUDA;
+  }
+  return FMHA_OK;
+}
+
+bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+template <int D, bool BF16>
+int launch_fmha(const b200::FmhaParams& prm, cudaStream_t stream) {
+  using C = b200::FmhaCfg<D>;
+  auto kern = b200::fmha_fwd_kernel<D, BF16>;
+  static bool attr_done[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 64 || !attr_done[dev]) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_ALLOC);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(fmha)");
+    if (dev < 64) attr_done[dev] = true;
+  }
+  dim3 grid = (prm.mask_kind == b200::MASK_CAUSAL) ? dim3(prm.num_units, prm.num_q_tiles, 1)
+                                                   : dim3(prm.num_q_tiles, prm.num_units, 1);
+  kern<<<grid, C::THREADS, C::SMEM_ALLOC, stream>>>(prm);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(e, "fmha_fwd_kernel launch");
+  return FMHA_OK;
+}
+
+int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask,
+                int batch, int heads, int seq_q, int seq_kv, int head_dim, float scale, cudaStream_t stream) {
+  g_last_cuda_error[0] = 0;
+  if (batch < 0 || heads < 0 || seq_q < 0 || seq_kv < 0) return FMHA_ERR_INVALID_ARG;
+  if (!std::isfinite(scale)) return FMHA_ERR_INVALID_ARG;
+  if (head_dim != 64 && head_dim != 128) return FMHA_ERR_UNSUPPORTED;
+  if (scale < 0.f) return FMHA_ERR_UNSUPPORTED;
+  const int kind = mask ? mask->kind : FMHA_MASK_NONE;
+  if (kind != FMHA_MASK_NONE && kind != FMHA_MASK_KEY_PADDING && kind != FMHA_MASK_CAUSAL)
+    return FMHA_ERR_UNSUPPORTED;
+  const long long units = static_cast<long long>(batch) * heads;
+  if (units == 0 || seq_q == 0) return FMHA_OK;
+  if (seq_kv == 0) return FMHA_ERR_INVALID_ARG;
+  if (!Q || !K || !V || !O) return FMHA_ERR_INVALID_ARG;
+  if (kind == FMHA_MASK_KEY_PADDING && !mask->kv_len) return FMHA_ERR_INVALID_ARG;
+  if (!aligned16(Q) || !aligned16(K) || !aligned16(V) || !aligned16(O)) return FMHA_ERR_MISALIGNED;
+  if (units > 2147483647LL || static_cast<long long>(seq_q) * head_dim * units * 2 > (1LL << 40))
+    return FMHA_ERR_INVALID_ARG;
+  int st = check_device(nullptr);
+  if (st != FMHA_OK) return st;
+
+  b200::FmhaParams prm;
+  memset(&prm, 0, sizeof(prm));
+  if ((st = make_map_3d(&prm.tmQ, Q, bf16, head_dim, seq_q, units, 128)) != FMHA_OK) return st;
+  if ((st = make_map_3d(&prm.tmK, K, bf16, head_dim, seq_kv, units, 128)) != FMHA_OK) return st;
+  if ((st = make_map_3d(&prm.tmV, V, bf16, head_dim, seq_kv, units, 128)) != FMHA_OK) return st;
+  if ((st = make_map_3d(&prm.tmO, O, bf16, head_dim, seq_q, units, 128)) != FMHA_OK) return st;
+  prm.kv_len = (kind == FMHA_MASK_KEY_PADDING) ? mask->kv_len : nullptr;
+  prm.seq_q = seq_q;
+  prm.seq_kv = seq_kv;
+  prm.heads = heads;
+  prm.num_q_tiles = (seq_q + 127) / 128;
+  prm.num_units = static_cast<int>(units);
+  prm.mask_kind = kind;
+  prm.scale_log2 = scale * 1.4426950408889634f;
+  if (prm.num_q_tiles > 65535 && kind == FMHA_MASK_CAUSAL) return FMHA_ERR_UNSUPPORTED;
+  if (units > 65535 && kind != FMHA_MASK_CAUSAL) return FMHA_ERR_UNSUPPORTED;
+
+  if (head_dim == 64) return bf16 ? launch_fmha<64, true>(prm, stream) : launch_fmha<64, false>(prm, stream);
+  return bf16 ? launch_fmha<128, true>(prm, stream) : launch_fmha<128, false>(prm, stream);
+}
+
+size_t round_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+}  // namespace
+
+namespace b200 {
+int make_map_2d_rows(CUtensorMap* m, const void* base, uint64_t cols, uint64_t rows, uint32_t box_rows, char* err,
+                     size_t errlen) {
+  int st = make_map_3d(m, base, false, cols, rows, 1, box_rows);
+  if (st != FMHA_OK && err && errlen) snprintf(err, errlen, "%s", g_last_cuda_error);
+  return st;
+}
+}  // namespace b200
+
+extern "C" {
+
+int fmha_fwd(const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask, int batch, int heads,
+             int seq_q, int seq_kv, int head_dim, float scale, fmha_stream_t stream) {
+  return fmha_common(false, Q, K, V, O, mask, batch, heads, seq_q, seq_kv, head_dim, scale,
+                     reinterpret_cast<cudaStream_t>(stream));
+}
+
+int fmha_fwd_bf16(const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask, int batch,
+                  int heads, int seq_q, int seq_kv, int head_dim, float scale, fmha_stream_t stream) {
+  return fmha_common(true, Q, K, V, O, mask, batch, heads, seq_q, seq_kv, head_dim, scale,
+                     reinterpret_cast<cudaStream_t>(stream));
+}
+
+size_t fmha_workspace_bytes(int batch, int heads, int seq_q, int seq_kv, int head_dim) {
+  if (batch < 0 || heads < 0 || seq_q < 0 || seq_kv < 0 || head_dim < 0) return 0;
+  const size_t u = static_cast<size_t>(batch) * heads;
+  const size_t q = round_up(u * seq_q * head_dim * 2, 256);
+  const size_t kv = round_up(u * seq_kv * head_dim * 2, 256);
+  return 2 * q + 2 * kv + round_up(static_cast<size_t>(batch) * 4, 256);
+}
+
+int fmha_fwd_from_host(int dtype, const void* hQ, const void* hK, const void* hV, void* hO, const fmha_mask_t* mask,
+                       void* workspace, size_t workspace_bytes, int batch, int heads, int seq_q, int seq_kv,
+                       int head_dim, float scale, fmha_stream_t stream_) {
+  g_last_cuda_error[0] = 0;
+  cudaStream_t stream = reinterpret_cast<cudaStream_t>(stream_);
+  if (dtype != 0 && dtype != 1) return FMHA_ERR_UNSUPPORTED;
+  if (batch < 0 || heads < 0 || seq_q < 0 || seq_kv < 0) return FMHA_ERR_INVALID_ARG;
+  const size_t u = static_cast<size_t>(batch) * heads;
+  if (u == 0 || seq_q == 0) return FMHA_OK;
+  if (!hQ || !hK || !hV || !hO || !workspace) return FMHA_ERR_INVALID_ARG;
+  if (workspace_bytes < fmha_workspace_bytes(batch, heads, seq_q, seq_kv, head_dim)) return FMHA_ERR_INVALID_ARG;
+  if ((reinterpret_cast<uintptr_t>(workspace) & 255u) != 0) return FMHA_ERR_MISALIGNED;
+  const size_t qb = u * seq_q * head_dim * 2, kvb = u * seq_kv * head_dim * 2;
+  uint8_t* w = static_cast<uint8_t*>(workspace);
+  uint8_t* dQ = w;
+  uint8_t* dO = dQ + round_up(qb, 256);
+  uint8_t* dK = dO + round_up(qb, 256);
+  uint8_t* dV = dK + round_up(kvb, 256);
+  int32_t* dL = reinterpret_cast<int32_t*>(dV + round_up(kvb, 256));
+  fmha_mask_t dmask = {FMHA_MASK_NONE, nullptr};
+  if (mask) {
+    dmask.kind = mask->kind;
+    if (mask->kind == FMHA_MASK_KEY_PADDING) {
+      if (!mask->kv_len) return FMHA_ERR_INVALID_ARG;
+      cudaError_t e = cudaMemcpyAsync(dL, mask->kv_len, sizeof(int32_t) * batch, cudaMemcpyHostToDevice, stream);
+      if (e != cudaSuccess) return cuda_fail(e, "H2D kv_len");
+      dmask.kv_len = dL;
+    }
+  }
+  cudaError_t e;
+  if ((e = cudaMemcpyAsync(dQ, hQ, qb, cudaMemcpyHostToDevice, stream)) != cudaSuccess) return cuda_fail(e, "H2D Q");
+  if ((e = cudaMemcpyAsync(dK, hK, kvb, cudaMemcpyHostToDevice, stream)) != cudaSuccess) return cuda_fail(e, "H2D K");
+  if ((e = cudaMemcpyAsync(dV, hV, kvb, cudaMemcpyHostToDevice, stream)) != cudaSuccess) return cuda_fail(e, "H2D V");
+  int st = fmha_common(dtype == 1, dQ, dK, dV, dO, &dmask, batch, heads, seq_q, seq_kv, head_dim, scale, stream);
+  if (st != FMHA_OK) return st;
+  if ((e = cudaMemcpyAsync(hO, dO, qb, cudaMemcpyDeviceToHost, stream)) != cudaSuccess) return cuda_fail(e, "D2H O");
+  return FMHA_OK;
+}
+
+int gemm_bias_act(const void* A, const void* W, const void* bias, void* Cm, int M, int N, int K, int act,
+                  fmha_stream_t stream) {
+  g_last_cuda_error[0] = 0;
+  if (M < 0 || N < 0 || K < 0) return FMHA_ERR_INVALID_ARG;
+  if (act < ACT_NONE || act > ACT_GELU_TANH) return FMHA_ERR_UNSUPPORTED;
+  if (M == 0 || N == 0) return FMHA_OK;
+  if (!A || !W || !Cm || K == 0) return FMHA_ERR_INVALID_ARG;
+  if ((K % 8) != 0 || (N % 8) != 0) return FMHA_ERR_UNSUPPORTED;
+  if (!aligned16(A) || !aligned16(W) || !aligned16(Cm) || (bias && !aligned16(bias))) return FMHA_ERR_MISALIGNED;
+  int sms = 0;
+  int st = check_device(&sms);
+  if (st != FMHA_OK) return st;
+  return b200::launch_gemm_bias_act(A, W, bias, Cm, M, N, K, act, sms, reinterpret_cast<cudaStream_t>(stream),
+                                    g_last_cuda_error, sizeof(g_last_cuda_error));
+}
+
+const char* fmha_status_string(int status) {
+  switch (status) {
+    case FMHA_OK: return "FMHA_OK";
+    case FMHA_ERR_INVALID_ARG: return "FMHA_ERR_INVALID_ARG: invalid argument";
+    case FMHA_ERR_UNSUPPORTED: return "FMHA_ERR_UNSUPPORTED: unsupported configuration";
+    case FMHA_ERR_MISALIGNED: return "FMHA_ERR_MISALIGNED: pointer not 16-byte aligned";
+    case FMHA_ERR_CUDA: return "FMHA_ERR_CUDA: CUDA error (see fmha_last_cuda_error)";
+    case FMHA_ERR_NO_DEVICE: return "FMHA_ERR_NO_DEVICE: no sm_100 device is current";
+    default: return "unknown status";
+  }
+}
+
+const char* fmha_last_cuda_error(void) { return g_last_cuda_error; }
+
+const char* fmha_version(void) { return "b200fmha 0.1 (sm_100a)"; }
+
+}  // extern "C"
