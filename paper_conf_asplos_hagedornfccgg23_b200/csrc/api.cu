@@ -6,6 +6,7 @@
 #include <cmath>
 #include <cstdio>
 #include <cstring>
+#include <algorithm>
 #include <mutex>
 
 #include "../../include/fmha.h"
@@ -96,9 +97,9 @@ int make_map_3d(CUtensorMap* m, const void* base, bool bf16, uint64_t cols, uint
 bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
 template <int D, bool BF16>
-int launch_fmha(const b200::FmhaParams& prm, cudaStream_t stream) {
+int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) {
   using C = b200::FmhaCfg<D>;
-  auto kern = b200::fmha_fwd_kernel<D, BF16>;
+  auto kern = b200::fmha_fwd_sm100<D, BF16>;
   static bool attr_done[64];
   int dev = 0;
   cudaGetDevice(&dev);
@@ -107,8 +108,8 @@ int launch_fmha(const b200::FmhaParams& prm, cudaStream_t stream) {
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(fmha)");
     if (dev < 64) attr_done[dev] = true;
   }
-  dim3 grid = (prm.mask_kind == b200::MASK_CAUSAL) ? dim3(prm.num_units, prm.num_q_tiles, 1)
-                                                   : dim3(prm.num_q_tiles, prm.num_units, 1);
+  // persistent: one CTA per SM (or fewer when there is less work)
+  dim3 grid(static_cast<unsigned>(std::min(prm.num_items, sm_count)), 1, 1);
   kern<<<grid, C::THREADS, C::SMEM_ALLOC, stream>>>(prm);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "fmha_fwd_kernel launch");
@@ -133,7 +134,8 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   if (!aligned16(Q) || !aligned16(K) || !aligned16(V) || !aligned16(O)) return FMHA_ERR_MISALIGNED;
   if (units > 2147483647LL || static_cast<long long>(seq_q) * head_dim * units * 2 > (1LL << 40))
     return FMHA_ERR_INVALID_ARG;
-  int st = check_device(nullptr);
+  int sm_count = 0;
+  int st = check_device(&sm_count);
   if (st != FMHA_OK) return st;
 
   b200::FmhaParams prm;
@@ -149,12 +151,17 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   prm.num_q_tiles = (seq_q + 127) / 128;
   prm.num_units = static_cast<int>(units);
   prm.mask_kind = kind;
-  prm.scale_log2 = scale * 1.4426950408889634f;
-  if (prm.num_q_tiles > 65535 && kind == FMHA_MASK_CAUSAL) return FMHA_ERR_UNSUPPORTED;
-  if (units > 65535 && kind != FMHA_MASK_CAUSAL) return FMHA_ERR_UNSUPPORTED;
+  // scale = 0 is legal (every visible key gets weight 1); keep c strictly positive so masked
+  // scores (-inf) still map to exp2(-inf) = 0 instead of -inf * 0 = NaN.  1e-30 perturbs visible
+  // scores by < 1e-25 in the exponent.
+  prm.scale_log2 = std::max(scale * 1.4426950408889634f, 1e-30f);
+  const long long items = units * ((prm.num_q_tiles + 1) / 2);
+  if (items > 2147483647LL) return FMHA_ERR_UNSUPPORTED;
+  prm.num_items = static_cast<int>(items);
 
-  if (head_dim == 64) return bf16 ? launch_fmha<64, true>(prm, stream) : launch_fmha<64, false>(prm, stream);
-  return bf16 ? launch_fmha<128, true>(prm, stream) : launch_fmha<128, false>(prm, stream);
+  if (head_dim == 64)
+    return bf16 ? launch_fmha<64, true>(prm, sm_count, stream) : launch_fmha<64, false>(prm, sm_count, stream);
+  return bf16 ? launch_fmha<128, true>(prm, sm_count, stream) : launch_fmha<128, false>(prm, sm_count, stream);
 }
 
 size_t round_up(size_t x, size_t a) { return (x + a - 1) / a * a; }

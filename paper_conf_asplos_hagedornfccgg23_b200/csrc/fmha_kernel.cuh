@@ -1,28 +1,30 @@
-// fmha_kernel.cuh — FMHA forward for sm_100a.
+// fmha_kernel.cuh — FMHA forward for sm_100a (persistent, warp-specialised, two Q tiles ping-pong).
 //
-// The operation is the paper's fused multi-head attention (§6): two back-to-back
-// GEMMs with a softmax between, per (batch, head).  This kernel is the B200-native design:
+// The operation is the paper's fused multi-head attention (§6 "Fused Multi-Head
+// Attention"): two back-to-back GEMMs with a softmax between them, per (batch, head).  The paper's
+// kernel was written for Ampere (ldmatrix + mma.sync, specialised to BERT shapes, L489); this is
+// the B200-native redesign:
 //
-//   unit of work     one 128-row query tile of one (b, h)                        [SURVEY §8(a) a1]
-//   warp roles       warp 0: TMA producer      (Q once, then K_j / V_j through a smem ring) [a2, a3]
-//                    warp 1: MMA issuer        (one thread issues tcgen05.mma)              [a4, a8]
-//                    warps 2-5: softmax group  (thread = query row; online softmax,
-//                                               O correction, epilogue)                     [a5-a7, a9]
-//   S = Q K^T        tcgen05.mma SS, M=128 N=128 K=D, fp32 accumulator in TMEM cols [0,128)
-//   P                exp2 of the scaled, max-shifted scores, rounded to fp16/bf16 and written
-//                    back into TMEM over S (cols [0,64)), so it never touches shared memory
-//   O += P V         tcgen05.mma TS (A = P from TMEM, B = V from smem, MN-major), fp32 in TMEM
-//                    cols [128, 128+D)
-//   epilogue         O / l, RNE to fp16/bf16, 128-bit swizzled st.shared into the (dead) Q
-//                    buffer, one TMA store per 64-column box (rows >= seq_q are clipped)
+//   work item     two consecutive 128-row query tiles (t = 0, 1) of one (b, h) sharing every
+//                 K/V tile load; persistent CTAs (one per SM) walk a static list of items   [a1]
+//   warps 0-3     softmax group for tile 0    (thread = query row; TMEM lane = row)        [a5, a6]
+//   warps 4-7     softmax group for tile 1
+//   warps 8-11    correction group: rescales O_t in TMEM when a row max moved by more than
+//                 2^8 (lazy), then the epilogue O_t / l -> fp16/bf16 -> smem -> TMA store  [a7, a9]
+//   warp 12       MMA issuer (one thread): S_t = Q_t K_j^T (SS), O_t += P_t V_j (TS)     [a4, a8]
+//   warp 13       TMA producer: Q_t per item, K_j / V_j through an NS-slot smem ring       [a2, a3]
+//   warps 14-15   idle (keep warpgroup 3 whole for setmaxnreg)
 //
-// Because tcgen05.ld hands each thread one full TMEM lane (= one query row), the row max and row
-// sum are thread-local: no warp-shuffle reduction is needed.
+//   TMEM (512 columns x 128 lanes, fp32):  S_0 [0,128)  S_1 [128,256)  O_0 [256,256+D)  O_1 [..+D)
+//   P_t (16-bit, two per column) overwrites the first 64 columns of S_t once S_t is in registers.
 //
-// Ordering facts the pipeline relies on:
-//   * tcgen05.mma ops issued by one thread execute in issue order, so QK_{j+1} may be issued into
-//     the S columns right after PV_j (which reads P_j from the same columns).
-//   * tcgen05.commit arrives once every earlier tcgen05 op of the issuing thread has completed.
+// Ordering facts relied on:
+//   * tcgen05.mma ops of one thread execute in issue order: QK_{t,j+1} may overwrite S_t right
+//     after PV_{t,j} (which reads P_t from the same columns) has been issued.
+//   * tcgen05.commit arrives once all earlier tcgen05 ops of the issuing thread have completed.
+//
+// Row statistics are thread-local because tcgen05.ld 32x32b gives each thread one whole row
+// (SURVEY D6): no warp-shuffle reductions.
 #pragma once
 #include "sm100.cuh"
 
@@ -41,84 +43,122 @@ struct FmhaParams {
   int heads;
   int num_q_tiles;
   int num_units;  // B*H
+  int num_items;  // num_units * ceil(num_q_tiles / 2)
   int mask_kind;
   float scale_log2;  // scale * log2(e)
 };
 
 template <int D>
 struct FmhaCfg {
-  static constexpr int BM = 128;                  // query rows per tile (UMMA M)
-  static constexpr int BN = 128;                  // keys per KV tile (UMMA N of QK^T, K of PV)
-  static constexpr int CHUNK = 128 * 64 * 2;      // one SW128 TMA box: 128 rows x 64 halves
-  static constexpr int TILE = BM * D * 2;         // bytes of a Q / K / V / O tile
-  static constexpr int NSLOT = (D == 64) ? 4 : 2; // K,V ring slots (K_j and V_j alternate)
-  static constexpr int OFF_Q = 0;
-  static constexpr int OFF_KV = TILE;
-  static constexpr int OFF_BAR = OFF_KV + NSLOT * TILE;
-  static constexpr int NUM_BARS = 4 + 2 * NSLOT;
+  static constexpr int BM = 128;                 // query rows per tile (UMMA M)
+  static constexpr int BN = 128;                 // keys per KV tile
+  static constexpr int CHUNK = 128 * 64 * 2;     // one SW128 TMA box: 128 rows x 64 16-bit elements
+  static constexpr int TILE = BM * D * 2;        // bytes of one Q / K / V / O tile
+  static constexpr int NS = (D == 64) ? 8 : 3;   // K/V ring slots (K_j, V_j alternate)
+  static constexpr int OFF_Q = 0;                // Q_0, Q_1
+  static constexpr int OFF_RING = 2 * TILE;
+  static constexpr int NSTG = (D == 64) ? 2 : 1;        // O staging buffers (D=128 shares one)
+  static constexpr int OFF_STG = OFF_RING + NS * TILE;
+  static constexpr int OFF_ALPHA = OFF_STG + NSTG * TILE;  // float alpha[2][128]
+  static constexpr int OFF_LSUM = OFF_ALPHA + 2 * 128 * 4;
+  static constexpr int OFF_BAR = OFF_LSUM + 2 * 128 * 4;
+  // barriers: 2x {q_full, q_empty, s_full, p_full, o_ready, pv_done, st_full, st_empty, l_full}
+  //           + NS x {kv_full, kv_empty}
+  static constexpr int NUM_BARS = 18 + 2 * NS;
   static constexpr int OFF_TMEMPTR = OFF_BAR + NUM_BARS * 8;
   static constexpr int SMEM_BYTES = OFF_TMEMPTR + 16;
   static constexpr int SMEM_ALLOC = SMEM_BYTES + 1024;  // slack for manual 1024-B alignment
-  static constexpr int TMEM_COLS = 256;
-  static constexpr int TMEM_S = 0;    // S (fp32, 128 cols); P (packed 16-bit, cols 0..63) aliases it
-  static constexpr int TMEM_O = 128;  // O accumulator (fp32, D cols)
-  static constexpr int THREADS = 192;
+  static constexpr int TMEM_COLS = 512;
+  static constexpr int THREADS = 512;
+  static_assert(SMEM_ALLOC <= 232448, "shared memory budget");
 };
 
+// One work item = q-tiles {2*pair, 2*pair+1} of unit bh.  Every role decodes items identically.
+struct WorkItem {
+  int bh;
+  int q0;         // first query row of tile 0
+  int kv_valid;   // keys >= kv_valid are masked for every row (key padding)
+  int n[2];       // KV tiles visited by tile t (0 = tile absent or fully masked)
+  bool has[2];    // tile t exists (rows < seq_q)
+};
+
+__device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
+  WorkItem w;
+  const int pairs = (p.num_q_tiles + 1) >> 1;
+  int pr;
+  if (p.mask_kind == MASK_CAUSAL) {  // longest-first: the last query tiles see the most keys
+    pr = pairs - 1 - idx / p.num_units;
+    w.bh = idx % p.num_units;
+  } else {  // both pairs of a (b,h) back to back so K/V are re-read from L2
+    w.bh = idx / pairs;
+    pr = idx % pairs;
+  }
+  w.q0 = pr * 256;
+  w.kv_valid = p.seq_kv;
+  if (p.mask_kind == MASK_KEY_PADDING) w.kv_valid = min(max(__ldg(p.kv_len + w.bh / p.heads), 0), p.seq_kv);
+  const int off = p.seq_kv - p.seq_q;
+#pragma unroll
+  for (int t = 0; t < 2; ++t) {
+    const int qt = 2 * pr + t;
+    w.has[t] = qt < p.num_q_tiles;
+    int kv_end = w.kv_valid;
+    if (p.mask_kind == MASK_CAUSAL) kv_end = min(kv_end, max(0, qt * 128 + 128 + off));
+    w.n[t] = w.has[t] ? (kv_end + 127) / 128 : 0;
+  }
+  return w;
+}
+
 template <int D, bool BF16>
-__global__ void __launch_bounds__(192, 2) fmha_fwd_kernel(const __grid_constant__ FmhaParams p) {
+__global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
   using C = FmhaCfg<D>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const uint32_t sbase = smem_u32(smem);
-  const uint32_t sQ = sbase + C::OFF_Q;
-  const uint32_t sKV = sbase + C::OFF_KV;
   const uint32_t bar = sbase + C::OFF_BAR;
-  const uint32_t BAR_Q = bar, BAR_S = bar + 8, BAR_P = bar + 16, BAR_O = bar + 24;
-  auto BAR_FULL = [&](int s) { return bar + 32 + 8 * s; };
-  auto BAR_EMPTY = [&](int s) { return bar + 32 + 8 * C::NSLOT + 8 * s; };
+  // barrier addresses (t = tile 0/1, s = ring slot)
+  auto Q_FULL = [&](int t) { return bar + 8 * (0 + t); };
+  auto Q_EMPTY = [&](int t) { return bar + 8 * (2 + t); };
+  auto S_FULL = [&](int t) { return bar + 8 * (4 + t); };
+  auto P_FULL = [&](int t) { return bar + 8 * (6 + t); };
+  auto O_READY = [&](int t) { return bar + 8 * (8 + t); };
+  auto PV_DONE = [&](int t) { return bar + 8 * (10 + t); };
+  auto ST_FULL = [&](int t) { return bar + 8 * (12 + t); };
+  auto ST_EMPTY = [&](int t) { return bar + 8 * (14 + t); };
+  auto L_FULL = [&](int t) { return bar + 8 * (16 + t); };
+  auto KV_FULL = [&](int s) { return bar + 8 * (18 + s); };
+  auto KV_EMPTY = [&](int s) { return bar + 8 * (18 + C::NS + s); };
+  float* s_alpha = reinterpret_cast<float*>(smem + C::OFF_ALPHA);
+  float* s_lsum = reinterpret_cast<float*>(smem + C::OFF_LSUM);
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(smem + C::OFF_TMEMPTR);
 
   const int warp = warp_id();
   const int lane = lane_id();
 
-  // ---- work unit.  Causal: longest (last) q-tiles first, across all heads.
-  int qtile, bh;
-  if (p.mask_kind == MASK_CAUSAL) {
-    bh = blockIdx.x;
-    qtile = p.num_q_tiles - 1 - static_cast<int>(blockIdx.y);
-  } else {
-    qtile = blockIdx.x;
-    bh = blockIdx.y;
-  }
-  const int b = bh / p.heads;
-  const int q0 = qtile * C::BM;
-  int kv_valid = p.seq_kv;
-  if (p.mask_kind == MASK_KEY_PADDING) kv_valid = min(max(__ldg(p.kv_len + b), 0), p.seq_kv);
-  const int causal_off = p.seq_kv - p.seq_q;
-  int kv_end = kv_valid;  // keys [kv_end, seq_kv) are invisible to every row of this tile
-  if (p.mask_kind == MASK_CAUSAL) kv_end = min(kv_end, max(0, q0 + C::BM + causal_off));
-  const int n_tiles = (kv_end + C::BN - 1) / C::BN;  // fully masked KV tiles are skipped (a5)
-
-  // ---- one-time setup
   if (threadIdx.x == 0) {
-    mbar_init(BAR_Q, 1);
-    mbar_init(BAR_S, 1);
-    mbar_init(BAR_P, 128);
-    mbar_init(BAR_O, 1);
-    for (int s = 0; s < C::NSLOT; ++s) {
-      mbar_init(BAR_FULL(s), 1);
-      mbar_init(BAR_EMPTY(s), 1);
+    for (int t = 0; t < 2; ++t) {
+      mbar_init(Q_FULL(t), 1);
+      mbar_init(Q_EMPTY(t), 1);
+      mbar_init(S_FULL(t), 1);
+      mbar_init(P_FULL(t), 128);
+      mbar_init(O_READY(t), 128);
+      mbar_init(PV_DONE(t), 1);
+      mbar_init(ST_FULL(t), 128);
+      mbar_init(ST_EMPTY(t), 128);
+      mbar_init(L_FULL(t), 128);
+    }
+    for (int s = 0; s < C::NS; ++s) {
+      mbar_init(KV_FULL(s), 1);
+      mbar_init(KV_EMPTY(s), 1);
     }
     fence_mbar_init();
   }
-  if (warp == 0 && lane == 0) {
+  if (warp == 13 && lane == 0) {
     tma_prefetch_desc(&p.tmQ);
     tma_prefetch_desc(&p.tmK);
     tma_prefetch_desc(&p.tmV);
     tma_prefetch_desc(&p.tmO);
   }
-  if (warp == 1) {
+  if (warp == 12) {
     tmem_alloc(smem_u32(tmem_holder), C::TMEM_COLS);
     tmem_relinquish();
   }
@@ -126,206 +166,303 @@ __global__ void __launch_bounds__(192, 2) fmha_fwd_kernel(const __grid_constant_
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_holder;
+  const int first = blockIdx.x, stride = gridDim.x;
 
-  if (warp == 0) {
-    // ================================================================ TMA producer (a2, a3)
-    if (lane == 0 && n_tiles > 0) {
-      const uint64_t keep = policy_evict_last();   // K/V are re-read by the other q-tiles of (b,h)
-      const uint64_t once = policy_evict_first();  // Q is read exactly once
-      mbar_arrive_expect_tx(BAR_Q, C::TILE);
+  if (warp >= 12) {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
+    if (warp == 13 && lane == 0) {
+      // ============================================================ TMA producer (a2, a3)
+      const uint64_t keep = policy_evict_last();   // K/V: re-read by the other q-tile pairs
+      const uint64_t once = policy_evict_first();  // Q: read once
+      uint32_t kv = 0, qc[2] = {0, 0};
+      for (int idx = first; idx < p.num_items; idx += stride) {
+        const WorkItem w = decode_item(p, idx);
+        const int N = max(w.n[0], w.n[1]);
 #pragma unroll
-      for (int c = 0; c < D / 64; ++c) tma_load_3d_hint(sQ + c * C::CHUNK, &p.tmQ, BAR_Q, c * 64, q0, bh, once);
-      for (int j = 0; j < n_tiles; ++j) {
-#pragma unroll
-        for (int w = 0; w < 2; ++w) {  // w = 0: K_j, w = 1: V_j
-          const int t = 2 * j + w;
-          const int slot = t % C::NSLOT;
-          const uint32_t ph = (t / C::NSLOT) & 1;
-          mbar_wait(BAR_EMPTY(slot), ph ^ 1);
-          mbar_arrive_expect_tx(BAR_FULL(slot), C::TILE);
-          const CUtensorMap* m = w ? &p.tmV : &p.tmK;
+        for (int t = 0; t < 2; ++t) {
+          if (w.n[t] == 0) continue;
+          mbar_wait(Q_EMPTY(t), (qc[t] & 1) ^ 1);
+          mbar_arrive_expect_tx(Q_FULL(t), C::TILE);
 #pragma unroll
           for (int c = 0; c < D / 64; ++c)
-            tma_load_3d_hint(sKV + slot * C::TILE + c * C::CHUNK, m, BAR_FULL(slot), c * 64, j * C::BN, bh, keep);
+            tma_load_3d_hint(sbase + C::OFF_Q + t * C::TILE + c * C::CHUNK, &p.tmQ, Q_FULL(t), c * 64,
+                             w.q0 + 128 * t, w.bh, once);
+          ++qc[t];
+        }
+        for (int j = 0; j < N; ++j) {
+#pragma unroll
+          for (int m = 0; m < 2; ++m, ++kv) {  // m = 0: K_j, m = 1: V_j
+            const int s = kv % C::NS;
+            mbar_wait(KV_EMPTY(s), ((kv / C::NS) & 1) ^ 1);
+            mbar_arrive_expect_tx(KV_FULL(s), C::TILE);
+            const CUtensorMap* map = m ? &p.tmV : &p.tmK;
+#pragma unroll
+            for (int c = 0; c < D / 64; ++c)
+              tma_load_3d_hint(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64, j * 128,
+                               w.bh, keep);
+          }
         }
       }
-    }
-  } else if (warp == 1) {
-    // ================================================================ MMA issuer (a4, a8)
-    if (lane == 0 && n_tiles > 0) {
-      constexpr uint32_t IDESC_QK = idesc_f16(BF16, 128, 128, false, false);  // Q, K both K-major
-      constexpr uint32_t IDESC_PV = idesc_f16(BF16, 128, D, false, true);     // P K-major, V MN-major
-      const uint32_t tS = tmem + C::TMEM_S;
-      const uint32_t tO = tmem + C::TMEM_O;
-      mbar_wait(BAR_Q, 0);
-      tc_fence_after();
-      auto issue_qk = [&](int j) {
-        const int t = 2 * j;
-        const int slot = t % C::NSLOT;
-        mbar_wait(BAR_FULL(slot), (t / C::NSLOT) & 1);
+    } else if (warp == 12 && lane == 0) {
+      // ============================================================ MMA issuer (a4, a8)
+      constexpr uint32_t IDESC_QK = idesc_f16(BF16, 128, 128, false, false);  // Q, K: K-major
+      constexpr uint32_t IDESC_PV = idesc_f16(BF16, 128, D, false, true);     // P: K-major (TMEM), V: MN-major
+      uint32_t kv = 0, qc[2] = {0, 0}, pc[2] = {0, 0}, oc[2] = {0, 0};
+      auto ring_wait = [&](uint32_t k) {
+        const int s = k % C::NS;
+        mbar_wait(KV_FULL(s), (k / C::NS) & 1);
         tc_fence_after();
-        const uint32_t sK = sKV + slot * C::TILE;
+        return sbase + C::OFF_RING + s * C::TILE;
+      };
+      auto qk = [&](int t, uint32_t sK) {
+        const uint32_t sQ = sbase + C::OFF_Q + t * C::TILE;
 #pragma unroll
         for (int kk = 0; kk < D / 16; ++kk) {
           const uint32_t off = (kk / 4) * C::CHUNK + (kk % 4) * 32;
-          umma_ss(tS, sdesc_sw128(sQ + off, 16, 1024), sdesc_sw128(sK + off, 16, 1024), IDESC_QK, kk > 0);
+          umma_ss(tmem + 128 * t, sdesc_sw128(sQ + off, 16, 1024), sdesc_sw128(sK + off, 16, 1024), IDESC_QK,
+                  kk > 0);
         }
-        umma_commit(BAR_EMPTY(slot));  // K_j slot free once this QK completes
-        umma_commit(BAR_S);            // S_j ready for the softmax group
+        umma_commit(S_FULL(t));
       };
-      issue_qk(0);
-      for (int j = 0; j < n_tiles; ++j) {
-        mbar_wait(BAR_P, j & 1);  // P_j written into TMEM, O rescaled
-        tc_fence_after();
-        const int t = 2 * j + 1;
-        const int slot = t % C::NSLOT;
-        mbar_wait(BAR_FULL(slot), (t / C::NSLOT) & 1);
-        tc_fence_after();
-        const uint32_t sV = sKV + slot * C::TILE;
+      for (int idx = first; idx < p.num_items; idx += stride) {
+        const WorkItem w = decode_item(p, idx);
+        const int N = max(w.n[0], w.n[1]);
+        if (N == 0) continue;
 #pragma unroll
-        for (int kk = 0; kk < C::BN / 16; ++kk)
-          umma_ts(tO, tS + kk * 8, sdesc_sw128(sV + kk * 2048, C::CHUNK, 1024), IDESC_PV, (j > 0 || kk > 0));
-        umma_commit(BAR_EMPTY(slot));  // V_j slot free
-        umma_commit(BAR_O);            // O holds sum_{<=j} P V
-        if (j + 1 < n_tiles) issue_qk(j + 1);
+        for (int t = 0; t < 2; ++t)
+          if (w.n[t] > 0) {
+            mbar_wait(Q_FULL(t), qc[t] & 1);
+            ++qc[t];
+          }
+        tc_fence_after();
+        uint32_t kslot = kv++;
+        uint32_t sK = ring_wait(kslot);
+#pragma unroll
+        for (int t = 0; t < 2; ++t)
+          if (w.n[t] > 0) qk(t, sK);
+        umma_commit(KV_EMPTY(kslot % C::NS));
+        for (int j = 0; j < N; ++j) {
+          const uint32_t vslot = kv++;
+          const uint32_t sV = ring_wait(vslot);
+          bool k_taken = false;
+#pragma unroll
+          for (int t = 0; t < 2; ++t) {
+            if (j >= w.n[t]) continue;
+            mbar_wait(P_FULL(t), pc[t] & 1);
+            ++pc[t];
+            mbar_wait(O_READY(t), oc[t] & 1);
+            ++oc[t];
+            tc_fence_after();
+            const uint32_t tO = tmem + 256 + t * D;
+            const uint32_t tP = tmem + 128 * t;
+#pragma unroll
+            for (int kk = 0; kk < 8; ++kk)
+              umma_ts(tO, tP + kk * 8, sdesc_sw128(sV + kk * 2048, C::CHUNK, 1024), IDESC_PV, (j > 0 || kk > 0));
+            umma_commit(PV_DONE(t));
+            if (j + 1 < w.n[t]) {
+              if (!k_taken) {
+                kslot = kv++;
+                sK = ring_wait(kslot);
+                k_taken = true;
+              }
+              qk(t, sK);
+            }
+          }
+          umma_commit(KV_EMPTY(vslot % C::NS));
+          if (k_taken) umma_commit(KV_EMPTY(kslot % C::NS));
+          if (j + 1 < N && !k_taken) {
+            // neither tile needs K_{j+1} (cannot happen: N = max n_t), keep the ring in step anyway
+            kslot = kv++;
+            ring_wait(kslot);
+            umma_commit(KV_EMPTY(kslot % C::NS));
+          }
+        }
+#pragma unroll
+        for (int t = 0; t < 2; ++t)
+          if (w.n[t] > 0) umma_commit(Q_EMPTY(t));
       }
     }
+  } else if (warp < 8) {
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 176;");
+    // ============================================================== softmax group t (a5, a6)
+    const int t = warp >> 2;
+    const int quad = warp & 3;
+    const int row = quad * 32 + lane;
+    const uint32_t tS = tmem + (static_cast<uint32_t>(quad * 32) << 16) + 128 * t;
+    const float c = p.scale_log2;
+    const int off = p.seq_kv - p.seq_q;
+    uint32_t sc = 0, stc = 0;
+    for (int idx = first; idx < p.num_items; idx += stride) {
+      const WorkItem w = decode_item(p, idx);
+      if (!w.has[t]) continue;
+      const int n = w.n[t];
+      const int qi = w.q0 + 128 * t + row;
+      int lim = w.kv_valid;  // keys j < lim are visible to this row
+      if (p.mask_kind == MASK_CAUSAL) lim = min(lim, qi + off + 1);
+      float m_ref = -INFINITY;  // max used as the exp2 reference (lags the true max by < 2^8)
+      float l = 0.f;
+      for (int j = 0; j < n; ++j) {
+        mbar_wait(S_FULL(t), sc & 1);
+        ++sc;
+        tc_fence_after();
+        uint32_t s[128];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) tmem_ld_32x32b_x32(tS + 32 * q, *reinterpret_cast<uint32_t(*)[32]>(&s[32 * q]));
+        tmem_wait_ld();
+        reg_fence(s);
+        const int rem = lim - j * 128;
+        const bool masked = rem < 128;
+        if (masked) {
+#pragma unroll
+          for (int k = 0; k < 128; ++k)
+            if (k >= rem) s[k] = __float_as_uint(-INFINITY);
+        }
+        float mx0 = m_ref, mx1 = -INFINITY;
+#pragma unroll
+        for (int k = 0; k < 128; k += 4) {
+          mx0 = fmax3(mx0, __uint_as_float(s[k]), __uint_as_float(s[k + 1]));
+          mx1 = fmax3(mx1, __uint_as_float(s[k + 2]), __uint_as_float(s[k + 3]));
+        }
+        const float m_new = fmaxf(mx0, mx1);
+        // Lazy rescale: keep the old reference while the max grows by < 8 in the log2 domain (the
+        // p's then stay <= 2^8, exact in fp32 and fp16/bf16 range); l and O share the reference.
+        float alpha = 1.f;
+        if (m_new > m_ref && (m_ref == -INFINITY || (m_new - m_ref) * c > 8.f)) {
+          alpha = (m_ref == -INFINITY) ? 0.f : ex2((m_ref - m_new) * c);
+          m_ref = m_new;
+        }
+        // hand alpha to the correction group (it rescales O_t before PV_{t,j})
+        mbar_wait(ST_EMPTY(t), (stc & 1) ^ 1);
+        s_alpha[t * 128 + row] = (j == 0) ? 1.f : alpha;
+        mbar_arrive(ST_FULL(t));
+        ++stc;
+
+        const float mc = (m_ref == -INFINITY) ? 0.f : m_ref * c;
+        float2 acc0 = make_float2(0.f, 0.f), acc1 = make_float2(0.f, 0.f);
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          uint32_t pk[32];
+#pragma unroll
+          for (int u = 0; u < 32; u += 2) {
+            const int k = 64 * h + 2 * u;
+            float2 x0 = ffma2(make_float2(__uint_as_float(s[k]), __uint_as_float(s[k + 1])), c, -mc);
+            float2 x1 = ffma2(make_float2(__uint_as_float(s[k + 2]), __uint_as_float(s[k + 3])), c, -mc);
+            x0.x = ex2(x0.x);
+            x0.y = ex2(x0.y);
+            x1.x = ex2(x1.x);
+            x1.y = ex2(x1.y);
+            acc0 = fadd2(acc0, x0);
+            acc1 = fadd2(acc1, x1);
+            pk[u] = pack2<BF16>(x0.x, x0.y);
+            pk[u + 1] = pack2<BF16>(x1.x, x1.y);
+          }
+          tmem_st_32x32b_x32(tS + 32 * h, pk);
+        }
+        tmem_wait_st();
+        tc_fence_before();
+        mbar_arrive(P_FULL(t));
+        l = l * alpha + ((acc0.x + acc0.y) + (acc1.x + acc1.y));
+      }
+      s_lsum[t * 128 + row] = l;
+      mbar_arrive(L_FULL(t));
+    }
   } else {
-    // ================================================================ softmax group (a5, a6, a7, a9)
-    const int quad = warp & 3;  // TMEM lane quadrant this warp may access
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 96;");
+    // ================================================================ correction group (a7, a9)
+    const int quad = warp & 3;
     const int row = quad * 32 + lane;
     const uint32_t lane_off = static_cast<uint32_t>(quad * 32) << 16;
-    const uint32_t tS = tmem + lane_off + C::TMEM_S;
-    const uint32_t tO = tmem + lane_off + C::TMEM_O;
-    const int qi = q0 + row;
-    int lim = kv_valid;  // keys j < lim are visible to this row
-    if (p.mask_kind == MASK_CAUSAL) lim = min(lim, qi + causal_off + 1);
-    const float c = p.scale_log2;
-    float m = -INFINITY;  // running max of raw scores
-    float l = 0.f;        // running sum of exp2(c*(s - m))
-
-    for (int j = 0; j < n_tiles; ++j) {
-      mbar_wait(BAR_S, j & 1);
-      tc_fence_after();
-      uint32_t s[128];
+    uint32_t stc[2] = {0, 0}, pvc[2] = {0, 0}, lc[2] = {0, 0};
+    for (int idx = first; idx < p.num_items; idx += stride) {
+      const WorkItem w = decode_item(p, idx);
+      const int N = max(w.n[0], w.n[1]);
+      for (int j = 0; j < N; ++j) {
 #pragma unroll
-      for (int q = 0; q < 4; ++q) tmem_ld_32x32b_x32(tS + 32 * q, *reinterpret_cast<uint32_t(*)[32]>(&s[32 * q]));
-      tmem_wait_ld();
-      reg_fence(s);
-
-      const int rem = lim - j * C::BN;  // visible keys of this row in this tile
-      const bool masked = rem < C::BN;  // boundary tile for this row (a5)
-      float mt0 = -INFINITY, mt1 = -INFINITY, mt2 = -INFINITY, mt3 = -INFINITY;
-      if (masked) {
+        for (int t = 0; t < 2; ++t) {
+          if (j >= w.n[t]) continue;
+          mbar_wait(ST_FULL(t), stc[t] & 1);
+          const float alpha = s_alpha[t * 128 + row];
+          mbar_arrive(ST_EMPTY(t));
+          ++stc[t];
+          if (j > 0) {
+            mbar_wait(PV_DONE(t), pvc[t] & 1);  // PV_{t,j-1} has landed in O_t
+            ++pvc[t];
+            if (__any_sync(0xffffffffu, alpha != 1.f)) {
+              tc_fence_after();
+              const uint32_t tO = tmem + lane_off + 256 + t * D;
 #pragma unroll
-        for (int k = 0; k < 128; k += 4) {
-          mt0 = fmaxf(mt0, k + 0 < rem ? __uint_as_float(s[k + 0]) : -INFINITY);
-          mt1 = fmaxf(mt1, k + 1 < rem ? __uint_as_float(s[k + 1]) : -INFINITY);
-          mt2 = fmaxf(mt2, k + 2 < rem ? __uint_as_float(s[k + 2]) : -INFINITY);
-          mt3 = fmaxf(mt3, k + 3 < rem ? __uint_as_float(s[k + 3]) : -INFINITY);
-        }
-      } else {
+              for (int q = 0; q < D / 32; ++q) {
+                uint32_t o[32];
+                tmem_ld_32x32b_x32(tO + 32 * q, o);
+                tmem_wait_ld();
+                reg_fence(o);
 #pragma unroll
-        for (int k = 0; k < 128; k += 4) {
-          mt0 = fmaxf(mt0, __uint_as_float(s[k + 0]));
-          mt1 = fmaxf(mt1, __uint_as_float(s[k + 1]));
-          mt2 = fmaxf(mt2, __uint_as_float(s[k + 2]));
-          mt3 = fmaxf(mt3, __uint_as_float(s[k + 3]));
+                for (int k = 0; k < 32; ++k) o[k] = __float_as_uint(__uint_as_float(o[k]) * alpha);
+                tmem_st_32x32b_x32(tO + 32 * q, o);
+              }
+              tmem_wait_st();
+            }
+          }
+          tc_fence_before();
+          mbar_arrive(O_READY(t));
         }
       }
-      const float m_new = fmaxf(m, fmaxf(fmaxf(mt0, mt1), fmaxf(mt2, mt3)));
-
-      if (j > 0) {
-        // O correction (a7): O <- alpha * O once PV_{j-1} has landed.
-        mbar_wait(BAR_O, (j - 1) & 1);
-        tc_fence_after();
-        const float alpha = (m_new > m) ? ((m == -INFINITY) ? 0.f : ex2((m - m_new) * c)) : 1.f;
-        if (__any_sync(0xffffffffu, alpha != 1.f)) {
+      // ------------------------------------------------------------ epilogue per tile (a9)
+#pragma unroll 1
+      for (int t = 0; t < 2; ++t) {
+        if (!w.has[t]) continue;
+        mbar_wait(L_FULL(t), lc[t] & 1);
+        ++lc[t];
+        const float l = s_lsum[t * 128 + row];
+        if (w.n[t] > 0) {
+          mbar_wait(PV_DONE(t), pvc[t] & 1);  // last PV of this tile
+          ++pvc[t];
+          tc_fence_after();
+        }
+        const float inv_l = (l > 0.f) ? 1.f / l : 0.f;  // fully masked row -> 0 (R4)
+        const uint32_t stg = sbase + C::OFF_STG + (t % C::NSTG) * C::TILE;
+        if (row == 0) tma_store_wait_read0();  // previous store out of this staging buffer done
+        named_bar_sync(1, 128);
+        const uint32_t tO = tmem + lane_off + 256 + t * D;
 #pragma unroll
-          for (int q = 0; q < D / 32; ++q) {
-            uint32_t o[32];
+        for (int q = 0; q < D / 32; ++q) {
+          uint32_t o[32];
+          if (w.n[t] > 0) {
             tmem_ld_32x32b_x32(tO + 32 * q, o);
             tmem_wait_ld();
             reg_fence(o);
+          } else {
 #pragma unroll
-            for (int k = 0; k < 32; ++k) o[k] = __float_as_uint(__uint_as_float(o[k]) * alpha);
-            tmem_st_32x32b_x32(tO + 32 * q, o);
+            for (int k = 0; k < 32; ++k) o[k] = 0u;
+          }
+          const int col0 = 32 * q;
+          const uint32_t box = stg + (col0 / 64) * C::CHUNK + row * 128;
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const int unit = ((col0 % 64) / 8) + u;
+            st_shared_v4(box + ((unit ^ (row & 7)) << 4),
+                         pack2<BF16>(__uint_as_float(o[8 * u + 0]) * inv_l, __uint_as_float(o[8 * u + 1]) * inv_l),
+                         pack2<BF16>(__uint_as_float(o[8 * u + 2]) * inv_l, __uint_as_float(o[8 * u + 3]) * inv_l),
+                         pack2<BF16>(__uint_as_float(o[8 * u + 4]) * inv_l, __uint_as_float(o[8 * u + 5]) * inv_l),
+                         pack2<BF16>(__uint_as_float(o[8 * u + 6]) * inv_l, __uint_as_float(o[8 * u + 7]) * inv_l));
           }
         }
-        l *= alpha;
-      }
-      m = m_new;
-      const float mc = (m == -INFINITY) ? 0.f : m * c;
-
-      // P = exp2(c*s - c*m) (a6), rounded to the I/O type and stored over S in TMEM.
-      float l0 = 0.f, l1 = 0.f;
+        fence_proxy_async_smem();
+        named_bar_sync(1, 128);
+        if (row == 0) {
 #pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        uint32_t pk[32];
-#pragma unroll
-        for (int t = 0; t < 32; ++t) {
-          const int k = 64 * h + 2 * t;
-          float e0 = ex2(fmaf(__uint_as_float(s[k]), c, -mc));
-          float e1 = ex2(fmaf(__uint_as_float(s[k + 1]), c, -mc));
-          if (masked) {
-            e0 = (k < rem) ? e0 : 0.f;
-            e1 = (k + 1 < rem) ? e1 : 0.f;
-          }
-          l0 += e0;
-          l1 += e1;
-          pk[t] = pack2<BF16>(e0, e1);
+          for (int c2 = 0; c2 < D / 64; ++c2)
+            tma_store_3d(&p.tmO, stg + c2 * C::CHUNK, c2 * 64, w.q0 + 128 * t, w.bh);
+          tma_store_commit();
         }
-        tmem_st_32x32b_x32(tS + 32 * h, pk);
-      }
-      l += l0 + l1;
-      tmem_wait_st();
-      tc_fence_before();
-      mbar_arrive(BAR_P);
-    }
-
-    // ---------------------------------------------------------------- epilogue (a9)
-    if (n_tiles > 0) {
-      mbar_wait(BAR_O, (n_tiles - 1) & 1);
-      tc_fence_after();
-    }
-    const float inv_l = (l > 0.f) ? 1.f / l : 0.f;  // fully masked row -> O = 0 (R4)
-#pragma unroll
-    for (int q = 0; q < D / 32; ++q) {
-      uint32_t o[32];
-      if (n_tiles > 0) {
-        tmem_ld_32x32b_x32(tO + 32 * q, o);
-        tmem_wait_ld();
-        reg_fence(o);
-      } else {
-#pragma unroll
-        for (int k = 0; k < 32; ++k) o[k] = 0u;
-      }
-      const int col0 = 32 * q;
-      const uint32_t box = sQ + (col0 / 64) * C::CHUNK + row * 128;
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const int unit = ((col0 % 64) / 8) + u;  // 16-byte unit within the 128-byte row
-        const uint32_t addr = box + ((unit ^ (row & 7)) << 4);  // SWIZZLE_128B placement
-        st_shared_v4(addr,
-                     pack2<BF16>(__uint_as_float(o[8 * u + 0]) * inv_l, __uint_as_float(o[8 * u + 1]) * inv_l),
-                     pack2<BF16>(__uint_as_float(o[8 * u + 2]) * inv_l, __uint_as_float(o[8 * u + 3]) * inv_l),
-                     pack2<BF16>(__uint_as_float(o[8 * u + 4]) * inv_l, __uint_as_float(o[8 * u + 5]) * inv_l),
-                     pack2<BF16>(__uint_as_float(o[8 * u + 6]) * inv_l, __uint_as_float(o[8 * u + 7]) * inv_l));
       }
     }
-    fence_proxy_async_smem();
-    named_bar_sync(1, 128);
-    if (row == 0) {
-#pragma unroll
-      for (int c2 = 0; c2 < D / 64; ++c2) tma_store_3d(&p.tmO, sQ + c2 * C::CHUNK, c2 * 64, q0, bh);
-      tma_store_commit();
-      tma_store_wait_read0();
-    }
+    if (row == 0) tma_store_wait0();
   }
 
   tc_fence_before();
   __syncthreads();
-  if (warp == 1) {
+  if (warp == 12) {
     tc_fence_after();
     tmem_dealloc(tmem, C::TMEM_COLS);
   }
