@@ -239,7 +239,10 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         uint32_t sK = ring_wait(kslot);
 #pragma unroll
         for (int t = 0; t < 2; ++t)
-          if (w.n[t] > 0) qk(t, sK);
+          if (w.n[t] > 0) {
+            qk(t, sK);
+            if (w.n[t] == 1) umma_commit(Q_EMPTY(t));
+          }
         umma_commit(KV_EMPTY(kslot % C::NS));
         for (int j = 0; j < N; ++j) {
           const uint32_t vslot = kv++;
@@ -266,6 +269,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
                 k_taken = true;
               }
               qk(t, sK);
+              if (j + 2 == w.n[t]) umma_commit(Q_EMPTY(t));  // last QK of tile t: Q_t slot reusable
             }
           }
           umma_commit(KV_EMPTY(vslot % C::NS));
@@ -277,31 +281,38 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             umma_commit(KV_EMPTY(kslot % C::NS));
           }
         }
-#pragma unroll
-        for (int t = 0; t < 2; ++t)
-          if (w.n[t] > 0) umma_commit(Q_EMPTY(t));
       }
     }
   } else if (warp < 8) {
     asm volatile("setmaxnreg.inc.sync.aligned.u32 176;");
     // ============================================================== softmax group t (a5, a6)
+    // The two groups take turns for the exp2 phase (named barriers 2 + t): while one group
+    // exponentiates, the other loads/reduces its next S and the tensor core runs the first
+    // group's PV and next QK, so MUFU and tensor pipes overlap instead of running in lockstep.
     const int t = warp >> 2;
     const int quad = warp & 3;
     const int row = quad * 32 + lane;
     const uint32_t tS = tmem + (static_cast<uint32_t>(quad * 32) << 16) + 128 * t;
     const float c = p.scale_log2;
     const int off = p.seq_kv - p.seq_q;
+    const uint32_t my_turn = 2 + t, other_turn = 3 - t;
+    if (t == 1) named_bar_arrive(2, 256);  // tile 0 goes first
     uint32_t sc = 0, stc = 0;
     for (int idx = first; idx < p.num_items; idx += stride) {
       const WorkItem w = decode_item(p, idx);
-      if (!w.has[t]) continue;
+      const int N = max(w.n[0], w.n[1]);
       const int n = w.n[t];
       const int qi = w.q0 + 128 * t + row;
       int lim = w.kv_valid;  // keys j < lim are visible to this row
       if (p.mask_kind == MASK_CAUSAL) lim = min(lim, qi + off + 1);
       float m_ref = -INFINITY;  // max used as the exp2 reference (lags the true max by < 2^8)
       float l = 0.f;
-      for (int j = 0; j < n; ++j) {
+      for (int j = 0; j < N; ++j) {
+        if (j >= n) {  // this tile has no KV tile j: keep the turn order
+          named_bar_sync(my_turn, 256);
+          named_bar_arrive(other_turn, 256);
+          continue;
+        }
         mbar_wait(S_FULL(t), sc & 1);
         ++sc;
         tc_fence_after();
@@ -311,8 +322,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         tmem_wait_ld();
         reg_fence(s);
         const int rem = lim - j * 128;
-        const bool masked = rem < 128;
-        if (masked) {
+        if (rem < 128) {  // boundary tile for this row (a5)
 #pragma unroll
           for (int k = 0; k < 128; ++k)
             if (k >= rem) s[k] = __float_as_uint(-INFINITY);
@@ -325,7 +335,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         }
         const float m_new = fmaxf(mx0, mx1);
         // Lazy rescale: keep the old reference while the max grows by < 8 in the log2 domain (the
-        // p's then stay <= 2^8, exact in fp32 and fp16/bf16 range); l and O share the reference.
+        // p's then stay <= 2^8, exact in fp32 and in fp16/bf16 range); l and O share the reference.
         float alpha = 1.f;
         if (m_new > m_ref && (m_ref == -INFINITY || (m_new - m_ref) * c > 8.f)) {
           alpha = (m_ref == -INFINITY) ? 0.f : ex2((m_ref - m_new) * c);
@@ -339,6 +349,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
 
         const float mc = (m_ref == -INFINITY) ? 0.f : m_ref * c;
         float2 acc0 = make_float2(0.f, 0.f), acc1 = make_float2(0.f, 0.f);
+        named_bar_sync(my_turn, 256);
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           uint32_t pk[32];
@@ -358,14 +369,18 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           }
           tmem_st_32x32b_x32(tS + 32 * h, pk);
         }
+        named_bar_arrive(other_turn, 256);
         tmem_wait_st();
         tc_fence_before();
         mbar_arrive(P_FULL(t));
         l = l * alpha + ((acc0.x + acc0.y) + (acc1.x + acc1.y));
       }
-      s_lsum[t * 128 + row] = l;
-      mbar_arrive(L_FULL(t));
+      if (w.has[t]) {
+        s_lsum[t * 128 + row] = l;
+        mbar_arrive(L_FULL(t));
+      }
     }
+    if (t == 0) named_bar_sync(2, 256);  // consume tile 1's last hand-over
   } else {
     asm volatile("setmaxnreg.dec.sync.aligned.u32 96;");
     // ================================================================ correction group (a7, a9)
