@@ -268,6 +268,22 @@ const char* fmha_status_string(int status) {
 
 const char* fmha_last_cuda_error(void) { return g_last_cuda_error; }
 
+#if FMHA_TRACE
+// Debug-build only (not part of include/fmha.h): point the timeline recorder at a device buffer
+// of 65536 uint64 records and reset its counter; fmha_trace_count() returns the record count.
+FMHA_API int fmha_trace_set(void* dev_buf) {
+  unsigned int zero = 0;
+  if (cudaMemcpyToSymbol(b200::g_fmha_trace, &dev_buf, sizeof(void*)) != cudaSuccess) return FMHA_ERR_CUDA;
+  if (cudaMemcpyToSymbol(b200::g_fmha_trace_n, &zero, sizeof(zero)) != cudaSuccess) return FMHA_ERR_CUDA;
+  return FMHA_OK;
+}
+FMHA_API unsigned int fmha_trace_count(void) {
+  unsigned int n = 0;
+  cudaMemcpyFromSymbol(&n, b200::g_fmha_trace_n, sizeof(n));
+  return n;
+}
+#endif
+
 const char* fmha_version(void) { return "b200fmha 0.1 (sm_100a)"; }
 
 }  // extern "C"

@@ -28,7 +28,39 @@
 #pragma once
 #include "sm100.cuh"
 
+// Debug timeline (build with -DFMHA_TRACE=1, see Makefile target `trace`): lane 0 of each warp of
+// CTA 0 appends (clock64, warp, event, aux) records to a global buffer.  Compiled out otherwise.
+#ifndef FMHA_TRACE
+#define FMHA_TRACE 0
+#endif
+
 namespace b200 {
+
+#if FMHA_TRACE
+__device__ unsigned long long* g_fmha_trace = nullptr;
+__device__ unsigned int g_fmha_trace_n = 0;
+// per-warp slices of 4096 records, plain stores (no atomics on the timed path)
+#define TRACE_EV(ev, aux)                                                                                \
+  do {                                                                                                   \
+    if (blockIdx.x == 0 && (threadIdx.x & 31) == 0 && trace_buf && trace_i < 4096u) {                    \
+      trace_buf[(threadIdx.x >> 5) * 4096u + trace_i++] =                                                \
+          (static_cast<unsigned long long>(clock64()) << 24) |                                           \
+          (static_cast<unsigned long long>(threadIdx.x >> 5) << 18) |                                    \
+          (static_cast<unsigned long long>(ev) << 12) | (static_cast<unsigned>(aux) & 0xFFFu);           \
+    }                                                                                                    \
+  } while (0)
+#define TRACE_DECL                                    \
+  unsigned long long* trace_buf = g_fmha_trace;      \
+  unsigned int trace_i = 0;
+#else
+#define TRACE_EV(ev, aux) \
+  do {                    \
+  } while (0)
+#define TRACE_DECL
+#endif
+// event ids
+enum : int { EV_S_WAIT = 1, EV_S_READY, EV_MAX_DONE, EV_TURN, EV_EXP_DONE, EV_MMA_P, EV_MMA_O, EV_MMA_PV,
+             EV_MMA_QK, EV_COR_ST, EV_COR_PV, EV_COR_ORDY, EV_EPI, EV_TMA_KV, EV_ITEM };
 
 enum : int { MASK_NONE = 0, MASK_KEY_PADDING = 1, MASK_CAUSAL = 2 };
 
@@ -54,9 +86,10 @@ struct FmhaCfg {
   static constexpr int BN = 128;                 // keys per KV tile
   static constexpr int CHUNK = 128 * 64 * 2;     // one SW128 TMA box: 128 rows x 64 16-bit elements
   static constexpr int TILE = BM * D * 2;        // bytes of one Q / K / V / O tile
-  static constexpr int NS = (D == 64) ? 8 : 3;   // K/V ring slots (K_j, V_j alternate)
-  static constexpr int OFF_Q = 0;                // Q_0, Q_1
-  static constexpr int OFF_RING = 2 * TILE;
+  static constexpr int NS = (D == 64) ? 6 : 3;   // K/V ring slots (K_j, V_j alternate)
+  static constexpr int QS = (D == 64) ? 2 : 1;   // Q stages per tile: the next item's Q loads early
+  static constexpr int OFF_Q = 0;                // Q[stage][tile]
+  static constexpr int OFF_RING = 2 * QS * TILE;
   static constexpr int NSTG = (D == 64) ? 2 : 1;        // O staging buffers (D=128 shares one)
   static constexpr int OFF_STG = OFF_RING + NS * TILE;
   static constexpr int OFF_ALPHA = OFF_STG + NSTG * TILE;  // float alpha[2][128]
@@ -64,12 +97,22 @@ struct FmhaCfg {
   static constexpr int OFF_BAR = OFF_LSUM + 2 * 128 * 4;
   // barriers: 2x {q_full, q_empty, s_full, p_full, o_ready, pv_done, st_full, st_empty, l_full}
   //           + NS x {kv_full, kv_empty}
-  static constexpr int NUM_BARS = 18 + 2 * NS;
+  static constexpr int NUM_BARS = 28 + 2 * NS;
   static constexpr int OFF_TMEMPTR = OFF_BAR + NUM_BARS * 8;
   static constexpr int SMEM_BYTES = OFF_TMEMPTR + 16;
-  static constexpr int SMEM_ALLOC = SMEM_BYTES + 1024;  // slack for manual 1024-B alignment
+  static constexpr int SMEM_ALLOC = SMEM_BYTES;
   static constexpr int TMEM_COLS = 512;
   static constexpr int THREADS = 512;
+  // D = 64: S_0, S_1, O_0, O_1 use 384 columns, so P_t gets its own 64 columns at 384 + 64 t and
+  // QK_{t,j+1} can be issued as soon as S_{t,j} is in registers (S_FREE), overlapping the softmax.
+  // D = 128: TMEM is full; P_t overwrites S_t and QK_{t,j+1} must follow PV_{t,j}.
+  static constexpr bool SEP_P = (D == 64);
+  static constexpr int TMEM_P = 384;
+  // exp-phase turn-taking between the two softmax groups (named barriers 2, 3).  With HALF_TURN
+  // the turn passes after half of the exp loop, so the groups overlap by half a phase: one warp's
+  // TMEM load + row max runs under the other's exponentials, and MUFU still sees two warps.
+  static constexpr bool TURNS = true;
+  static constexpr bool HALF_TURN = SEP_P;
   static_assert(SMEM_ALLOC <= 232448, "shared memory budget");
 };
 
@@ -111,13 +154,15 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
 template <int D, bool BF16>
 __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
   using C = FmhaCfg<D>;
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // Dynamic shared memory starts at the (1024-byte aligned) base of the CTA's shared window; the
+  // SWIZZLE_128B tiles need that alignment.  Using the base directly keeps every smem address a
+  // compile-time-uniform value, so UMMA descriptors live in uniform registers.
+  extern __shared__ __align__(1024) uint8_t smem[];
   const uint32_t sbase = smem_u32(smem);
   const uint32_t bar = sbase + C::OFF_BAR;
   // barrier addresses (t = tile 0/1, s = ring slot)
-  auto Q_FULL = [&](int t) { return bar + 8 * (0 + t); };
-  auto Q_EMPTY = [&](int t) { return bar + 8 * (2 + t); };
+  auto Q_FULL = [&](int t, int q) { return bar + 8 * (20 + C::NS * 2 + 2 * q + t); };  // q = Q stage
+  auto Q_EMPTY = [&](int t, int q) { return bar + 8 * (24 + C::NS * 2 + 2 * q + t); };
   auto S_FULL = [&](int t) { return bar + 8 * (4 + t); };
   auto P_FULL = [&](int t) { return bar + 8 * (6 + t); };
   auto O_READY = [&](int t) { return bar + 8 * (8 + t); };
@@ -125,19 +170,24 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
   auto ST_FULL = [&](int t) { return bar + 8 * (12 + t); };
   auto ST_EMPTY = [&](int t) { return bar + 8 * (14 + t); };
   auto L_FULL = [&](int t) { return bar + 8 * (16 + t); };
-  auto KV_FULL = [&](int s) { return bar + 8 * (18 + s); };
-  auto KV_EMPTY = [&](int s) { return bar + 8 * (18 + C::NS + s); };
+  auto S_FREE = [&](int t) { return bar + 8 * (18 + t); };
+  auto KV_FULL = [&](int s) { return bar + 8 * (20 + s); };
+  auto KV_EMPTY = [&](int s) { return bar + 8 * (20 + C::NS + s); };
   float* s_alpha = reinterpret_cast<float*>(smem + C::OFF_ALPHA);
   float* s_lsum = reinterpret_cast<float*>(smem + C::OFF_LSUM);
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(smem + C::OFF_TMEMPTR);
 
   const int warp = warp_id();
   const int lane = lane_id();
+  TRACE_DECL
 
   if (threadIdx.x == 0) {
+    if (sbase & 1023u) __trap();  // the layout below assumes a 1024-byte aligned window
     for (int t = 0; t < 2; ++t) {
-      mbar_init(Q_FULL(t), 1);
-      mbar_init(Q_EMPTY(t), 1);
+      for (int q = 0; q < 2; ++q) {
+        mbar_init(Q_FULL(t, q), 1);
+        mbar_init(Q_EMPTY(t, q), 1);
+      }
       mbar_init(S_FULL(t), 1);
       mbar_init(P_FULL(t), 128);
       mbar_init(O_READY(t), 128);
@@ -145,10 +195,11 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       mbar_init(ST_FULL(t), 128);
       mbar_init(ST_EMPTY(t), 128);
       mbar_init(L_FULL(t), 128);
+      mbar_init(S_FREE(t), 128);
     }
     for (int s = 0; s < C::NS; ++s) {
       mbar_init(KV_FULL(s), 1);
-      mbar_init(KV_EMPTY(s), 1);
+      mbar_init(KV_EMPTY(s), 2);  // released by both MMA warps
     }
     fence_mbar_init();
   }
@@ -170,7 +221,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
 
   if (warp >= 12) {
     asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
-    if (warp == 13 && lane == 0) {
+    if (warp == 13) {
       // ============================================================ TMA producer (a2, a3)
       const uint64_t keep = policy_evict_last();   // K/V: re-read by the other q-tile pairs
       const uint64_t once = policy_evict_first();  // Q: read once
@@ -181,104 +232,115 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
 #pragma unroll
         for (int t = 0; t < 2; ++t) {
           if (w.n[t] == 0) continue;
-          mbar_wait(Q_EMPTY(t), (qc[t] & 1) ^ 1);
-          mbar_arrive_expect_tx(Q_FULL(t), C::TILE);
+          const int qs = qc[t] % C::QS;
+          mbar_wait(Q_EMPTY(t, qs), ((qc[t] / C::QS) & 1) ^ 1);
+          mbar_arrive_expect_tx_elect(Q_FULL(t, qs), C::TILE);
 #pragma unroll
           for (int c = 0; c < D / 64; ++c)
-            tma_load_3d_hint(sbase + C::OFF_Q + t * C::TILE + c * C::CHUNK, &p.tmQ, Q_FULL(t), c * 64,
-                             w.q0 + 128 * t, w.bh, once);
+            tma_load_3d_hint_elect(sbase + C::OFF_Q + (2 * qs + t) * C::TILE + c * C::CHUNK, &p.tmQ, Q_FULL(t, qs),
+                                   c * 64, w.q0 + 128 * t, w.bh, once);
           ++qc[t];
+          TRACE_EV(EV_ITEM, 3 + t);
         }
         for (int j = 0; j < N; ++j) {
 #pragma unroll
           for (int m = 0; m < 2; ++m, ++kv) {  // m = 0: K_j, m = 1: V_j
             const int s = kv % C::NS;
             mbar_wait(KV_EMPTY(s), ((kv / C::NS) & 1) ^ 1);
-            mbar_arrive_expect_tx(KV_FULL(s), C::TILE);
+            TRACE_EV(EV_TMA_KV, m * 64 + j);
+            mbar_arrive_expect_tx_elect(KV_FULL(s), C::TILE);
             const CUtensorMap* map = m ? &p.tmV : &p.tmK;
 #pragma unroll
             for (int c = 0; c < D / 64; ++c)
-              tma_load_3d_hint(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64, j * 128,
+              tma_load_3d_hint_elect(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64, j * 128,
                                w.bh, keep);
           }
         }
       }
-    } else if (warp == 12 && lane == 0) {
-      // ============================================================ MMA issuer (a4, a8)
+    } else if (warp == 12 || warp == 14) {
+      // ============================================================ MMA issuers (a4, a8)
+      // Warp 12 issues tile 0's MMAs, warp 14 tile 1's: each tile's chain (QK -> softmax -> PV)
+      // then depends only on its own softmax group.  Both warps release every K/V slot (count 2).
+      const int t = (warp == 12) ? 0 : 1;
       constexpr uint32_t IDESC_QK = idesc_f16(BF16, 128, 128, false, false);  // Q, K: K-major
       constexpr uint32_t IDESC_PV = idesc_f16(BF16, 128, D, false, true);     // P: K-major (TMEM), V: MN-major
-      uint32_t kv = 0, qc[2] = {0, 0}, pc[2] = {0, 0}, oc[2] = {0, 0};
+      // descriptors differ only in the start-address field: build one base and add (offset >> 4)
+      const uint64_t desc0 = sdesc_sw128(sbase, 16, 1024);          // K-major Q / K tiles
+      const uint64_t vdesc0 = sdesc_sw128(sbase, C::CHUNK, 1024);   // MN-major V tiles
+      const uint32_t tS = tmem + 128 * t;
+      const uint32_t tO = tmem + 256 + t * D;
+      const uint32_t tP = tmem + (C::SEP_P ? C::TMEM_P + 64 * t : 128 * t);
+      uint32_t kv = 0, qc = 0, pc = 0, oc = 0, qkc = 0;
       auto ring_wait = [&](uint32_t k) {
-        const int s = k % C::NS;
-        mbar_wait(KV_FULL(s), (k / C::NS) & 1);
+        mbar_wait(KV_FULL(k % C::NS), (k / C::NS) & 1);
         tc_fence_after();
-        return sbase + C::OFF_RING + s * C::TILE;
-      };
-      auto qk = [&](int t, uint32_t sK) {
-        const uint32_t sQ = sbase + C::OFF_Q + t * C::TILE;
-#pragma unroll
-        for (int kk = 0; kk < D / 16; ++kk) {
-          const uint32_t off = (kk / 4) * C::CHUNK + (kk % 4) * 32;
-          umma_ss(tmem + 128 * t, sdesc_sw128(sQ + off, 16, 1024), sdesc_sw128(sK + off, 16, 1024), IDESC_QK,
-                  kk > 0);
-        }
-        umma_commit(S_FULL(t));
+        return sbase + C::OFF_RING + (k % C::NS) * C::TILE;
       };
       for (int idx = first; idx < p.num_items; idx += stride) {
         const WorkItem w = decode_item(p, idx);
         const int N = max(w.n[0], w.n[1]);
         if (N == 0) continue;
+        const int n = w.n[t];
+        int qs = 0;
+        if (n > 0) {
+          qs = qc % C::QS;
+          mbar_wait(Q_FULL(t, qs), (qc / C::QS) & 1);
+          ++qc;
+          tc_fence_after();
+        }
+        const uint32_t qoff = C::OFF_Q + (2 * qs + t) * C::TILE;
+        const uint32_t base = kv;  // ring index of K_0 of this item; K_j = base + 2j, V_j = base + 2j + 1
+        kv += 2 * N;
+        // S_t <- Q_t K_j^T (with separate P buffers: once softmax t has read the previous S_t)
+        auto issue_qk = [&](int j) {
+          const uint32_t kidx = base + 2 * j;
+          const uint32_t sK = ring_wait(kidx);
+          if (j < n) {
+            if (C::SEP_P && qkc > 0) {
+              mbar_wait(S_FREE(t), (qkc - 1) & 1);
+              tc_fence_after();
+            }
+            ++qkc;
+            const uint32_t koff = sK - sbase;
 #pragma unroll
-        for (int t = 0; t < 2; ++t)
-          if (w.n[t] > 0) {
-            mbar_wait(Q_FULL(t), qc[t] & 1);
-            ++qc[t];
+            for (int kk = 0; kk < D / 16; ++kk) {
+              const uint32_t off = (kk / 4) * C::CHUNK + (kk % 4) * 32;
+              umma_ss_elect(tS, desc0 + ((qoff + off) >> 4), desc0 + ((koff + off) >> 4), IDESC_QK, kk > 0);
+            }
+            umma_commit_elect(S_FULL(t));
+            TRACE_EV(EV_MMA_QK, t * 64 + j);
+            if (j + 1 == n) umma_commit_elect(Q_EMPTY(t, qs));  // last QK of this tile: Q slot reusable
           }
-        tc_fence_after();
-        uint32_t kslot = kv++;
-        uint32_t sK = ring_wait(kslot);
-#pragma unroll
-        for (int t = 0; t < 2; ++t)
-          if (w.n[t] > 0) {
-            qk(t, sK);
-            if (w.n[t] == 1) umma_commit(Q_EMPTY(t));
-          }
-        umma_commit(KV_EMPTY(kslot % C::NS));
-        for (int j = 0; j < N; ++j) {
-          const uint32_t vslot = kv++;
-          const uint32_t sV = ring_wait(vslot);
-          bool k_taken = false;
-#pragma unroll
-          for (int t = 0; t < 2; ++t) {
-            if (j >= w.n[t]) continue;
-            mbar_wait(P_FULL(t), pc[t] & 1);
-            ++pc[t];
-            mbar_wait(O_READY(t), oc[t] & 1);
-            ++oc[t];
+          umma_commit_elect(KV_EMPTY(kidx % C::NS));
+        };
+        // O_t (+)= P_t V_j once softmax t wrote P_t and the correction group rescaled O_t
+        auto issue_pv = [&](int j) {
+          const uint32_t vidx = base + 2 * j + 1;
+          const uint32_t sV = ring_wait(vidx);
+          if (j < n) {
+            mbar_wait(P_FULL(t), pc & 1);
+            ++pc;
+            TRACE_EV(EV_MMA_P, t * 64 + j);
+            mbar_wait(O_READY(t), oc & 1);
+            ++oc;
+            TRACE_EV(EV_MMA_O, t * 64 + j);
             tc_fence_after();
-            const uint32_t tO = tmem + 256 + t * D;
-            const uint32_t tP = tmem + 128 * t;
 #pragma unroll
             for (int kk = 0; kk < 8; ++kk)
-              umma_ts(tO, tP + kk * 8, sdesc_sw128(sV + kk * 2048, C::CHUNK, 1024), IDESC_PV, (j > 0 || kk > 0));
-            umma_commit(PV_DONE(t));
-            if (j + 1 < w.n[t]) {
-              if (!k_taken) {
-                kslot = kv++;
-                sK = ring_wait(kslot);
-                k_taken = true;
-              }
-              qk(t, sK);
-              if (j + 2 == w.n[t]) umma_commit(Q_EMPTY(t));  // last QK of tile t: Q_t slot reusable
-            }
+              umma_ts_elect(tO, tP + kk * 8, vdesc0 + ((sV - sbase + kk * 2048) >> 4), IDESC_PV, (j > 0 || kk > 0));
+            umma_commit_elect(PV_DONE(t));
+            TRACE_EV(EV_MMA_PV, t * 64 + j);
           }
-          umma_commit(KV_EMPTY(vslot % C::NS));
-          if (k_taken) umma_commit(KV_EMPTY(kslot % C::NS));
-          if (j + 1 < N && !k_taken) {
-            // neither tile needs K_{j+1} (cannot happen: N = max n_t), keep the ring in step anyway
-            kslot = kv++;
-            ring_wait(kslot);
-            umma_commit(KV_EMPTY(kslot % C::NS));
+          umma_commit_elect(KV_EMPTY(vidx % C::NS));
+        };
+        issue_qk(0);
+        for (int j = 0; j < N; ++j) {
+          if (C::SEP_P) {  // next scores first: they only need S_t free, not P_t
+            if (j + 1 < N) issue_qk(j + 1);
+            issue_pv(j);
+          } else {  // P_t overwrites S_t: QK_{t,j+1} must follow PV_{t,j} (in-order tensor pipe)
+            issue_pv(j);
+            if (j + 1 < N) issue_qk(j + 1);
           }
         }
       }
@@ -296,8 +358,9 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     const float c = p.scale_log2;
     const int off = p.seq_kv - p.seq_q;
     const uint32_t my_turn = 2 + t, other_turn = 3 - t;
-    if (t == 1) named_bar_arrive(2, 256);  // tile 0 goes first
-    uint32_t sc = 0, stc = 0;
+    if (C::TURNS && t == 1) named_bar_arrive(2, 256);  // tile 0 goes first
+    const uint32_t tP = tmem + (static_cast<uint32_t>(quad * 32) << 16) + (C::SEP_P ? C::TMEM_P + 64 * t : 128 * t);
+    uint32_t sc = 0, stc = 0, gstep = 0;
     for (int idx = first; idx < p.num_items; idx += stride) {
       const WorkItem w = decode_item(p, idx);
       const int N = max(w.n[0], w.n[1]);
@@ -309,18 +372,26 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       float l = 0.f;
       for (int j = 0; j < N; ++j) {
         if (j >= n) {  // this tile has no KV tile j: keep the turn order
-          named_bar_sync(my_turn, 256);
-          named_bar_arrive(other_turn, 256);
+          if (C::TURNS) {
+            named_bar_sync(my_turn, 256);
+            named_bar_arrive(other_turn, 256);
+          }
           continue;
         }
+        TRACE_EV(EV_S_WAIT, j);
         mbar_wait(S_FULL(t), sc & 1);
         ++sc;
+        TRACE_EV(EV_S_READY, j);
         tc_fence_after();
         uint32_t s[128];
 #pragma unroll
         for (int q = 0; q < 4; ++q) tmem_ld_32x32b_x32(tS + 32 * q, *reinterpret_cast<uint32_t(*)[32]>(&s[32 * q]));
         tmem_wait_ld();
         reg_fence(s);
+        if (C::SEP_P) {  // S_t is in registers: the tensor core may overwrite it with S_{t,j+1}
+          tc_fence_before();
+          mbar_arrive(S_FREE(t));
+        }
         const int rem = lim - j * 128;
         if (rem < 128) {  // boundary tile for this row (a5)
 #pragma unroll
@@ -349,7 +420,14 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
 
         const float mc = (m_ref == -INFINITY) ? 0.f : m_ref * c;
         float2 acc0 = make_float2(0.f, 0.f), acc1 = make_float2(0.f, 0.f);
-        named_bar_sync(my_turn, 256);
+        TRACE_EV(EV_MAX_DONE, j);
+        if (C::TURNS) named_bar_sync(my_turn, 256);
+        TRACE_EV(EV_TURN, j);
+        if (C::SEP_P && gstep > 0) {  // P_t buffer still read by PV_{t,j-1}?
+          mbar_wait(PV_DONE(t), (gstep - 1) & 1);
+          tc_fence_after();
+        }
+        ++gstep;
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           uint32_t pk[32];
@@ -367,9 +445,11 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             pk[u] = pack2<BF16>(x0.x, x0.y);
             pk[u + 1] = pack2<BF16>(x1.x, x1.y);
           }
-          tmem_st_32x32b_x32(tS + 32 * h, pk);
+          tmem_st_32x32b_x32(tP + 32 * h, pk);
+          if (C::TURNS && C::HALF_TURN && h == 0) named_bar_arrive(other_turn, 256);
         }
-        named_bar_arrive(other_turn, 256);
+        if (C::TURNS && !C::HALF_TURN) named_bar_arrive(other_turn, 256);
+        TRACE_EV(EV_EXP_DONE, j);
         tmem_wait_st();
         tc_fence_before();
         mbar_arrive(P_FULL(t));
@@ -380,7 +460,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         mbar_arrive(L_FULL(t));
       }
     }
-    if (t == 0) named_bar_sync(2, 256);  // consume tile 1's last hand-over
+    if (C::TURNS && t == 0) named_bar_sync(2, 256);  // consume tile 1's last hand-over
   } else {
     asm volatile("setmaxnreg.dec.sync.aligned.u32 96;");
     // ================================================================ correction group (a7, a9)
@@ -396,6 +476,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         for (int t = 0; t < 2; ++t) {
           if (j >= w.n[t]) continue;
           mbar_wait(ST_FULL(t), stc[t] & 1);
+          TRACE_EV(EV_COR_ST, t * 64 + j);
           const float alpha = s_alpha[t * 128 + row];
           mbar_arrive(ST_EMPTY(t));
           ++stc[t];
@@ -420,6 +501,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           }
           tc_fence_before();
           mbar_arrive(O_READY(t));
+          TRACE_EV(EV_COR_ORDY, t * 64 + j);
         }
       }
       // ------------------------------------------------------------ epilogue per tile (a9)
