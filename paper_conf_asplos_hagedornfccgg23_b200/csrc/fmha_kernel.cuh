@@ -1,4 +1,4 @@
-// fmha_kernel.cuh — FMHA forward for sm_100a (persistent, warp-specialised, two Q tiles ping-pong).
+// fmha_kernel.cuh — FMHA forward for sm_100a (persistent, warp-specialised, two Q tiles per CTA).
 //
 // The operation is the paper's fused multi-head attention (§6 "Fused Multi-Head
 // Attention"): two back-to-back GEMMs with a softmax between them, per (batch, head).  The paper's
@@ -6,30 +6,35 @@
 // the B200-native redesign:
 //
 //   work item     two consecutive 128-row query tiles (t = 0, 1) of one (b, h) sharing every
-//                 K/V tile load; persistent CTAs (one per SM) walk a static list of items   [a1]
-//   warps 0-3     softmax group for tile 0    (thread = query row; TMEM lane = row)        [a5, a6]
-//   warps 4-7     softmax group for tile 1
-//   warps 8-11    correction group: rescales O_t in TMEM when a row max moved by more than
-//                 2^8 (lazy), then the epilogue O_t / l -> fp16/bf16 -> smem -> TMA store  [a7, a9]
-//   warp 12       MMA issuer (one thread): S_t = Q_t K_j^T (SS), O_t += P_t V_j (TS)     [a4, a8]
-//   warp 13       TMA producer: Q_t per item, K_j / V_j through an NS-slot smem ring       [a2, a3]
-//   warps 14-15   idle (keep warpgroup 3 whole for setmaxnreg)
+//                 K/V tile load; persistent CTAs (one per SM) walk a static item list        [a1]
+//   warps 0-15    softmax: warp (t, h, q) = 8t + 4h + q handles rows 32q..32q+31 of tile t and
+//                 key columns 64h..64h+63 of every 128-key S tile (two warps per row, so each
+//                 SMSP runs four softmax warps and MUFU.EX2 never idles on one warp's latency;
+//                 the two halves exchange their partial row max through smem)              [a5, a6]
+//   warps 16-19   correction: rescale O_t in TMEM when a row max grew by more than 2^8
+//                 (lazy), then the epilogue O_t / l -> fp16/bf16 -> smem -> TMA store      [a7, a9]
+//   warps 20, 21  MMA issuers for tile 0 / tile 1 (one elected lane each):
+//                 S_t = Q_t K_j^T (SS), O_t += P_t V_j (TS)                                [a4, a8]
+//   warp 22       TMA producer: Q_t per item (double-buffered at D=64), K_j / V_j ring     [a2, a3]
 //
 //   TMEM (512 columns x 128 lanes, fp32):  S_0 [0,128)  S_1 [128,256)  O_0 [256,256+D)  O_1 [..+D)
-//   P_t (16-bit, two per column) overwrites the first 64 columns of S_t once S_t is in registers.
+//   D = 64 : P_t (16-bit, two per column) has its own columns [384 + 64t, 448 + 64t), so
+//            QK_{t,j+1} starts as soon as S_{t,j} is in registers (S_FREE).
+//   D = 128: TMEM is full; P_t overwrites the first 64 columns of S_t and QK_{t,j+1} follows
+//            PV_{t,j} (tcgen05.mma ops of one thread execute in issue order).
 //
 // Ordering facts relied on:
-//   * tcgen05.mma ops of one thread execute in issue order: QK_{t,j+1} may overwrite S_t right
-//     after PV_{t,j} (which reads P_t from the same columns) has been issued.
+//   * tcgen05.mma ops of one thread execute in issue order;
 //   * tcgen05.commit arrives once all earlier tcgen05 ops of the issuing thread have completed.
 //
-// Row statistics are thread-local because tcgen05.ld 32x32b gives each thread one whole row
-// (SURVEY D6): no warp-shuffle reductions.
+// Because tcgen05.ld 32x32b gives each thread whole TMEM lanes (= query rows), row statistics are
+// thread-local: no warp-shuffle reductions.  The two column halves of a row meet
+// through one 4-byte smem slot per row and a 64-thread named barrier.
 #pragma once
 #include "sm100.cuh"
 
 // Debug timeline (build with -DFMHA_TRACE=1, see Makefile target `trace`): lane 0 of each warp of
-// CTA 0 appends (clock64, warp, event, aux) records to a global buffer.  Compiled out otherwise.
+// CTA 0 appends (clock64, warp, event, aux) records to its slice of a global buffer.
 #ifndef FMHA_TRACE
 #define FMHA_TRACE 0
 #endif
@@ -39,18 +44,17 @@ namespace b200 {
 #if FMHA_TRACE
 __device__ unsigned long long* g_fmha_trace = nullptr;
 __device__ unsigned int g_fmha_trace_n = 0;
-// per-warp slices of 4096 records, plain stores (no atomics on the timed path)
 #define TRACE_EV(ev, aux)                                                                                \
   do {                                                                                                   \
-    if (blockIdx.x == 0 && (threadIdx.x & 31) == 0 && trace_buf && trace_i < 4096u) {                    \
-      trace_buf[(threadIdx.x >> 5) * 4096u + trace_i++] =                                                \
+    if (blockIdx.x == 0 && (threadIdx.x & 31) == 0 && trace_buf && trace_i < 2048u) {                    \
+      trace_buf[(threadIdx.x >> 5) * 2048u + trace_i++] =                                                \
           (static_cast<unsigned long long>(clock64()) << 24) |                                           \
           (static_cast<unsigned long long>(threadIdx.x >> 5) << 18) |                                    \
           (static_cast<unsigned long long>(ev) << 12) | (static_cast<unsigned>(aux) & 0xFFFu);           \
     }                                                                                                    \
   } while (0)
-#define TRACE_DECL                                    \
-  unsigned long long* trace_buf = g_fmha_trace;      \
+#define TRACE_DECL                               \
+  unsigned long long* trace_buf = g_fmha_trace; \
   unsigned int trace_i = 0;
 #else
 #define TRACE_EV(ev, aux) \
@@ -58,8 +62,7 @@ __device__ unsigned int g_fmha_trace_n = 0;
   } while (0)
 #define TRACE_DECL
 #endif
-// event ids
-enum : int { EV_S_WAIT = 1, EV_S_READY, EV_MAX_DONE, EV_TURN, EV_EXP_DONE, EV_MMA_P, EV_MMA_O, EV_MMA_PV,
+enum : int { EV_S_WAIT = 1, EV_S_READY, EV_MAX_DONE, EV_XCHG, EV_EXP_DONE, EV_MMA_P, EV_MMA_O, EV_MMA_PV,
              EV_MMA_QK, EV_COR_ST, EV_COR_PV, EV_COR_ORDY, EV_EPI, EV_TMA_KV, EV_ITEM };
 
 enum : int { MASK_NONE = 0, MASK_KEY_PADDING = 1, MASK_CAUSAL = 2 };
@@ -82,47 +85,47 @@ struct FmhaParams {
 
 template <int D>
 struct FmhaCfg {
-  static constexpr int BM = 128;                 // query rows per tile (UMMA M)
-  static constexpr int BN = 128;                 // keys per KV tile
-  static constexpr int CHUNK = 128 * 64 * 2;     // one SW128 TMA box: 128 rows x 64 16-bit elements
-  static constexpr int TILE = BM * D * 2;        // bytes of one Q / K / V / O tile
-  static constexpr int NS = (D == 64) ? 6 : 3;   // K/V ring slots (K_j, V_j alternate)
-  static constexpr int QS = (D == 64) ? 2 : 1;   // Q stages per tile: the next item's Q loads early
-  static constexpr int OFF_Q = 0;                // Q[stage][tile]
+  static constexpr int BM = 128;                // query rows per tile (UMMA M)
+  static constexpr int BN = 128;                // keys per KV tile
+  static constexpr int CHUNK = 128 * 64 * 2;    // one SW128 TMA box: 128 rows x 64 16-bit elements
+  static constexpr int TILE = BM * D * 2;       // bytes of one Q / K / V / O tile
+  static constexpr int NS = (D == 64) ? 6 : 3;  // K/V ring slots (K_j, V_j alternate)
+  static constexpr int QS = (D == 64) ? 2 : 1;  // Q stages per tile: the next item's Q loads early
+  static constexpr int NSTG = (D == 64) ? 2 : 1;  // O staging buffers (D=128: both tiles share one)
+  static constexpr int OFF_Q = 0;               // Q[stage][tile]
   static constexpr int OFF_RING = 2 * QS * TILE;
-  static constexpr int NSTG = (D == 64) ? 2 : 1;        // O staging buffers (D=128 shares one)
   static constexpr int OFF_STG = OFF_RING + NS * TILE;
-  static constexpr int OFF_ALPHA = OFF_STG + NSTG * TILE;  // float alpha[2][128]
-  static constexpr int OFF_LSUM = OFF_ALPHA + 2 * 128 * 4;
-  static constexpr int OFF_BAR = OFF_LSUM + 2 * 128 * 4;
-  // barriers: 2x {q_full, q_empty, s_full, p_full, o_ready, pv_done, st_full, st_empty, l_full}
-  //           + NS x {kv_full, kv_empty}
-  static constexpr int NUM_BARS = 28 + 2 * NS;
+  static constexpr int OFF_ALPHA = OFF_STG + NSTG * TILE;  // float alpha[2 tiles][128 rows]
+  static constexpr int OFF_LSUM = OFF_ALPHA + 2 * 128 * 4;  // float l[2 tiles][2 halves][128]
+  static constexpr int OFF_PMAX = OFF_LSUM + 4 * 128 * 4;   // float pmax[2 parity][2][2][128]
+  static constexpr int OFF_BAR = OFF_PMAX + 8 * 128 * 4;
+  // barrier slots
+  enum : int {
+    B_S_FULL = 0, B_P_FULL = 2, B_O_READY = 4, B_PV_DONE = 6, B_ST_FULL = 8, B_ST_EMPTY = 10, B_L_FULL = 12,
+    B_S_FREE = 14, B_Q_FULL = 16, B_Q_EMPTY = 20, B_KV = 24
+  };
+  static constexpr int NUM_BARS = B_KV + 2 * NS;
   static constexpr int OFF_TMEMPTR = OFF_BAR + NUM_BARS * 8;
-  static constexpr int SMEM_BYTES = OFF_TMEMPTR + 16;
-  static constexpr int SMEM_ALLOC = SMEM_BYTES;
+  static constexpr int SMEM_ALLOC = OFF_TMEMPTR + 16;
   static constexpr int TMEM_COLS = 512;
-  static constexpr int THREADS = 512;
-  // D = 64: S_0, S_1, O_0, O_1 use 384 columns, so P_t gets its own 64 columns at 384 + 64 t and
-  // QK_{t,j+1} can be issued as soon as S_{t,j} is in registers (S_FREE), overlapping the softmax.
-  // D = 128: TMEM is full; P_t overwrites S_t and QK_{t,j+1} must follow PV_{t,j}.
+  static constexpr int THREADS = 768;
   static constexpr bool SEP_P = (D == 64);
   static constexpr int TMEM_P = 384;
-  // exp-phase turn-taking between the two softmax groups (named barriers 2, 3).  With HALF_TURN
-  // the turn passes after half of the exp loop, so the groups overlap by half a phase: one warp's
-  // TMEM load + row max runs under the other's exponentials, and MUFU still sees two warps.
-  static constexpr bool TURNS = true;
-  static constexpr bool HALF_TURN = SEP_P;
+  // registers after setmaxnreg.  setmaxnreg.inc only draws on the CTA's launch allocation
+  // (80 x 768 = 61440), so 16 x 32 x 96 + 4 x 32 x 56 + 4 x 32 x 40 = 61440 must not be exceeded.
+  static constexpr int REG_SOFTMAX = 96, REG_CORR = 56, REG_MISC = 40;
+  static_assert(16 * 32 * REG_SOFTMAX + 4 * 32 * REG_CORR + 4 * 32 * REG_MISC <= 80 * THREADS, "register pool");
   static_assert(SMEM_ALLOC <= 232448, "shared memory budget");
 };
 
 // One work item = q-tiles {2*pair, 2*pair+1} of unit bh.  Every role decodes items identically.
 struct WorkItem {
   int bh;
-  int q0;         // first query row of tile 0
-  int kv_valid;   // keys >= kv_valid are masked for every row (key padding)
-  int n[2];       // KV tiles visited by tile t (0 = tile absent or fully masked)
-  bool has[2];    // tile t exists (rows < seq_q)
+  int q0;        // first query row of tile 0
+  int kv_valid;  // keys >= kv_valid are masked for every row (key padding)
+  int n0, n1;    // KV tiles visited by tile 0 / 1 (0 = tile absent or fully masked)
+  bool has1;     // tile 1 exists (tile 0 always does)
+  __device__ __forceinline__ int n(int t) const { return t ? n1 : n0; }
 };
 
 __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
@@ -140,41 +143,33 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
   w.kv_valid = p.seq_kv;
   if (p.mask_kind == MASK_KEY_PADDING) w.kv_valid = min(max(__ldg(p.kv_len + w.bh / p.heads), 0), p.seq_kv);
   const int off = p.seq_kv - p.seq_q;
-#pragma unroll
-  for (int t = 0; t < 2; ++t) {
-    const int qt = 2 * pr + t;
-    w.has[t] = qt < p.num_q_tiles;
-    int kv_end = w.kv_valid;
-    if (p.mask_kind == MASK_CAUSAL) kv_end = min(kv_end, max(0, qt * 128 + 128 + off));
-    w.n[t] = w.has[t] ? (kv_end + 127) / 128 : 0;
+  int kv_end0 = w.kv_valid, kv_end1 = w.kv_valid;
+  if (p.mask_kind == MASK_CAUSAL) {
+    kv_end0 = min(kv_end0, max(0, w.q0 + 128 + off));
+    kv_end1 = min(kv_end1, max(0, w.q0 + 256 + off));
   }
+  w.has1 = 2 * pr + 1 < p.num_q_tiles;
+  w.n0 = (kv_end0 + 127) / 128;
+  w.n1 = w.has1 ? (kv_end1 + 127) / 128 : 0;
   return w;
 }
 
 template <int D, bool BF16>
-__global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
+__global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
   using C = FmhaCfg<D>;
   // Dynamic shared memory starts at the (1024-byte aligned) base of the CTA's shared window; the
-  // SWIZZLE_128B tiles need that alignment.  Using the base directly keeps every smem address a
-  // compile-time-uniform value, so UMMA descriptors live in uniform registers.
+  // SWIZZLE_128B tiles need that alignment.  Using the base directly keeps smem addresses uniform.
   extern __shared__ __align__(1024) uint8_t smem[];
   const uint32_t sbase = smem_u32(smem);
   const uint32_t bar = sbase + C::OFF_BAR;
-  // barrier addresses (t = tile 0/1, s = ring slot)
-  auto Q_FULL = [&](int t, int q) { return bar + 8 * (20 + C::NS * 2 + 2 * q + t); };  // q = Q stage
-  auto Q_EMPTY = [&](int t, int q) { return bar + 8 * (24 + C::NS * 2 + 2 * q + t); };
-  auto S_FULL = [&](int t) { return bar + 8 * (4 + t); };
-  auto P_FULL = [&](int t) { return bar + 8 * (6 + t); };
-  auto O_READY = [&](int t) { return bar + 8 * (8 + t); };
-  auto PV_DONE = [&](int t) { return bar + 8 * (10 + t); };
-  auto ST_FULL = [&](int t) { return bar + 8 * (12 + t); };
-  auto ST_EMPTY = [&](int t) { return bar + 8 * (14 + t); };
-  auto L_FULL = [&](int t) { return bar + 8 * (16 + t); };
-  auto S_FREE = [&](int t) { return bar + 8 * (18 + t); };
-  auto KV_FULL = [&](int s) { return bar + 8 * (20 + s); };
-  auto KV_EMPTY = [&](int s) { return bar + 8 * (20 + C::NS + s); };
+  auto BAR = [&](int slot) { return bar + 8 * slot; };
+  auto Q_FULL = [&](int t, int q) { return BAR(C::B_Q_FULL + 2 * q + t); };
+  auto Q_EMPTY = [&](int t, int q) { return BAR(C::B_Q_EMPTY + 2 * q + t); };
+  auto KV_FULL = [&](int s) { return BAR(C::B_KV + s); };
+  auto KV_EMPTY = [&](int s) { return BAR(C::B_KV + C::NS + s); };
   float* s_alpha = reinterpret_cast<float*>(smem + C::OFF_ALPHA);
   float* s_lsum = reinterpret_cast<float*>(smem + C::OFF_LSUM);
+  float* s_pmax = reinterpret_cast<float*>(smem + C::OFF_PMAX);
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(smem + C::OFF_TMEMPTR);
 
   const int warp = warp_id();
@@ -184,18 +179,18 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
   if (threadIdx.x == 0) {
     if (sbase & 1023u) __trap();  // the layout below assumes a 1024-byte aligned window
     for (int t = 0; t < 2; ++t) {
+      mbar_init(BAR(C::B_S_FULL + t), 1);
+      mbar_init(BAR(C::B_P_FULL + t), 256);   // both column halves of all 128 rows
+      mbar_init(BAR(C::B_O_READY + t), 128);  // correction threads
+      mbar_init(BAR(C::B_PV_DONE + t), 1);
+      mbar_init(BAR(C::B_ST_FULL + t), 128);  // half-0 softmax threads
+      mbar_init(BAR(C::B_ST_EMPTY + t), 128);
+      mbar_init(BAR(C::B_L_FULL + t), 256);
+      mbar_init(BAR(C::B_S_FREE + t), 256);
       for (int q = 0; q < 2; ++q) {
         mbar_init(Q_FULL(t, q), 1);
         mbar_init(Q_EMPTY(t, q), 1);
       }
-      mbar_init(S_FULL(t), 1);
-      mbar_init(P_FULL(t), 128);
-      mbar_init(O_READY(t), 128);
-      mbar_init(PV_DONE(t), 1);
-      mbar_init(ST_FULL(t), 128);
-      mbar_init(ST_EMPTY(t), 128);
-      mbar_init(L_FULL(t), 128);
-      mbar_init(S_FREE(t), 128);
     }
     for (int s = 0; s < C::NS; ++s) {
       mbar_init(KV_FULL(s), 1);
@@ -203,13 +198,13 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     }
     fence_mbar_init();
   }
-  if (warp == 13 && lane == 0) {
+  if (warp == 22 && lane == 0) {
     tma_prefetch_desc(&p.tmQ);
     tma_prefetch_desc(&p.tmK);
     tma_prefetch_desc(&p.tmV);
     tma_prefetch_desc(&p.tmO);
   }
-  if (warp == 12) {
+  if (warp == 20) {
     tmem_alloc(smem_u32(tmem_holder), C::TMEM_COLS);
     tmem_relinquish();
   }
@@ -219,28 +214,29 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
   const uint32_t tmem = *tmem_holder;
   const int first = blockIdx.x, stride = gridDim.x;
 
-  if (warp >= 12) {
-    asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
-    if (warp == 13) {
+  if (warp >= 20) {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(C::REG_MISC));
+    if (warp == 22) {
       // ============================================================ TMA producer (a2, a3)
       const uint64_t keep = policy_evict_last();   // K/V: re-read by the other q-tile pairs
       const uint64_t once = policy_evict_first();  // Q: read once
-      uint32_t kv = 0, qc[2] = {0, 0};
+      uint32_t kv = 0, qc0 = 0, qc1 = 0;
       for (int idx = first; idx < p.num_items; idx += stride) {
         const WorkItem w = decode_item(p, idx);
-        const int N = max(w.n[0], w.n[1]);
+        const int N = max(w.n0, w.n1);
 #pragma unroll
         for (int t = 0; t < 2; ++t) {
-          if (w.n[t] == 0) continue;
-          const int qs = qc[t] % C::QS;
-          mbar_wait(Q_EMPTY(t, qs), ((qc[t] / C::QS) & 1) ^ 1);
+          if (w.n(t) == 0) continue;
+          uint32_t& qc = t ? qc1 : qc0;
+          const int qs = qc % C::QS;
+          mbar_wait(Q_EMPTY(t, qs), ((qc / C::QS) & 1) ^ 1);
           mbar_arrive_expect_tx_elect(Q_FULL(t, qs), C::TILE);
 #pragma unroll
           for (int c = 0; c < D / 64; ++c)
             tma_load_3d_hint_elect(sbase + C::OFF_Q + (2 * qs + t) * C::TILE + c * C::CHUNK, &p.tmQ, Q_FULL(t, qs),
                                    c * 64, w.q0 + 128 * t, w.bh, once);
-          ++qc[t];
-          TRACE_EV(EV_ITEM, 3 + t);
+          ++qc;
+          TRACE_EV(EV_ITEM, 4 + t);
         }
         for (int j = 0; j < N; ++j) {
 #pragma unroll
@@ -252,159 +248,209 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             const CUtensorMap* map = m ? &p.tmV : &p.tmK;
 #pragma unroll
             for (int c = 0; c < D / 64; ++c)
-              tma_load_3d_hint_elect(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64, j * 128,
-                               w.bh, keep);
+              tma_load_3d_hint_elect(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64,
+                                     j * 128, w.bh, keep);
           }
         }
       }
-    } else if (warp == 12 || warp == 14) {
+    } else if (warp == 20 || warp == 21) {
       // ============================================================ MMA issuers (a4, a8)
-      // Warp 12 issues tile 0's MMAs, warp 14 tile 1's: each tile's chain (QK -> softmax -> PV)
-      // then depends only on its own softmax group.  Both warps release every K/V slot (count 2).
-      const int t = (warp == 12) ? 0 : 1;
+      // Warp 20 issues tile 0's MMAs, warp 21 tile 1's, so each tile's chain (QK -> softmax ->
+      // PV) depends only on its own softmax warps.  Both warps release every K/V slot (count 2).
+      const int t = warp - 20;
       constexpr uint32_t IDESC_QK = idesc_f16(BF16, 128, 128, false, false);  // Q, K: K-major
       constexpr uint32_t IDESC_PV = idesc_f16(BF16, 128, D, false, true);     // P: K-major (TMEM), V: MN-major
-      // descriptors differ only in the start-address field: build one base and add (offset >> 4)
-      const uint64_t desc0 = sdesc_sw128(sbase, 16, 1024);          // K-major Q / K tiles
-      const uint64_t vdesc0 = sdesc_sw128(sbase, C::CHUNK, 1024);   // MN-major V tiles
+      // descriptors differ only in the start-address field: one base, plus (offset >> 4)
+      const uint64_t desc0 = sdesc_sw128(sbase, 16, 1024);         // K-major Q / K tiles
+      const uint64_t vdesc0 = sdesc_sw128(sbase, C::CHUNK, 1024);  // MN-major V tiles
       const uint32_t tS = tmem + 128 * t;
       const uint32_t tO = tmem + 256 + t * D;
       const uint32_t tP = tmem + (C::SEP_P ? C::TMEM_P + 64 * t : 128 * t);
-      uint32_t kv = 0, qc = 0, pc = 0, oc = 0, qkc = 0;
+      const uint32_t S_FULL = BAR(C::B_S_FULL + t), P_FULL = BAR(C::B_P_FULL + t);
+      const uint32_t O_READY = BAR(C::B_O_READY + t), PV_DONE = BAR(C::B_PV_DONE + t);
+      const uint32_t S_FREE = BAR(C::B_S_FREE + t);
+      uint32_t qc = 0, pc = 0, oc = 0, qkc = 0;
       auto ring_wait = [&](uint32_t k) {
         mbar_wait(KV_FULL(k % C::NS), (k / C::NS) & 1);
         tc_fence_after();
         return sbase + C::OFF_RING + (k % C::NS) * C::TILE;
       };
-      for (int idx = first; idx < p.num_items; idx += stride) {
-        const WorkItem w = decode_item(p, idx);
-        const int N = max(w.n[0], w.n[1]);
-        if (N == 0) continue;
-        const int n = w.n[t];
-        int qs = 0;
-        if (n > 0) {
-          qs = qc % C::QS;
-          mbar_wait(Q_FULL(t, qs), (qc / C::QS) & 1);
-          ++qc;
-          tc_fence_after();
+      // Two cursors walk the same sequence of (item, KV step j): the QK cursor runs one step ahead
+      // of the PV cursor (behind it when P aliases S), across item boundaries, so the next item's
+      // first S is computed while the current item's last P is still being produced.
+      struct Cursor {
+        int idx, j, N, n, qs;
+        uint32_t base;  // ring index of K_0 of the item; K_j = base + 2j, V_j = base + 2j + 1
+        bool valid;
+      };
+      auto seek = [&](Cursor& cu, int idx, uint32_t base) {
+        cu.valid = false;
+        for (; idx < p.num_items; idx += stride) {
+          const WorkItem w = decode_item(p, idx);
+          const int N = max(w.n0, w.n1);
+          if (N == 0) continue;
+          cu.idx = idx;
+          cu.j = 0;
+          cu.N = N;
+          cu.n = w.n(t);
+          cu.base = base;
+          cu.valid = true;
+          return;
         }
-        const uint32_t qoff = C::OFF_Q + (2 * qs + t) * C::TILE;
-        const uint32_t base = kv;  // ring index of K_0 of this item; K_j = base + 2j, V_j = base + 2j + 1
-        kv += 2 * N;
-        // S_t <- Q_t K_j^T (with separate P buffers: once softmax t has read the previous S_t)
-        auto issue_qk = [&](int j) {
-          const uint32_t kidx = base + 2 * j;
+      };
+      auto advance = [&](Cursor& cu) {
+        if (++cu.j == cu.N) seek(cu, cu.idx + stride, cu.base + 2 * cu.N);
+      };
+      Cursor cq, cp;
+      seek(cq, first, 0);
+      cp = cq;
+      // S_t <- Q_t K_j^T (separate P: once the softmax warps have read the previous S_t)
+      auto issue_qk = [&](Cursor& cu) {
+        const uint32_t kidx = cu.base + 2 * cu.j;
+        if (cu.j < cu.n) {
+          if (cu.j == 0) {  // first QK of this item's tile t: its Q tile must have landed
+            cu.qs = qc % C::QS;
+            mbar_wait(Q_FULL(t, cu.qs), (qc / C::QS) & 1);
+            ++qc;
+          }
           const uint32_t sK = ring_wait(kidx);
-          if (j < n) {
-            if (C::SEP_P && qkc > 0) {
-              mbar_wait(S_FREE(t), (qkc - 1) & 1);
-              tc_fence_after();
-            }
-            ++qkc;
-            const uint32_t koff = sK - sbase;
-#pragma unroll
-            for (int kk = 0; kk < D / 16; ++kk) {
-              const uint32_t off = (kk / 4) * C::CHUNK + (kk % 4) * 32;
-              umma_ss_elect(tS, desc0 + ((qoff + off) >> 4), desc0 + ((koff + off) >> 4), IDESC_QK, kk > 0);
-            }
-            umma_commit_elect(S_FULL(t));
-            TRACE_EV(EV_MMA_QK, t * 64 + j);
-            if (j + 1 == n) umma_commit_elect(Q_EMPTY(t, qs));  // last QK of this tile: Q slot reusable
-          }
-          umma_commit_elect(KV_EMPTY(kidx % C::NS));
-        };
-        // O_t (+)= P_t V_j once softmax t wrote P_t and the correction group rescaled O_t
-        auto issue_pv = [&](int j) {
-          const uint32_t vidx = base + 2 * j + 1;
-          const uint32_t sV = ring_wait(vidx);
-          if (j < n) {
-            mbar_wait(P_FULL(t), pc & 1);
-            ++pc;
-            TRACE_EV(EV_MMA_P, t * 64 + j);
-            mbar_wait(O_READY(t), oc & 1);
-            ++oc;
-            TRACE_EV(EV_MMA_O, t * 64 + j);
+          if (C::SEP_P && qkc > 0) {
+            mbar_wait(S_FREE, (qkc - 1) & 1);
             tc_fence_after();
-#pragma unroll
-            for (int kk = 0; kk < 8; ++kk)
-              umma_ts_elect(tO, tP + kk * 8, vdesc0 + ((sV - sbase + kk * 2048) >> 4), IDESC_PV, (j > 0 || kk > 0));
-            umma_commit_elect(PV_DONE(t));
-            TRACE_EV(EV_MMA_PV, t * 64 + j);
           }
-          umma_commit_elect(KV_EMPTY(vidx % C::NS));
-        };
-        issue_qk(0);
-        for (int j = 0; j < N; ++j) {
-          if (C::SEP_P) {  // next scores first: they only need S_t free, not P_t
-            if (j + 1 < N) issue_qk(j + 1);
-            issue_pv(j);
-          } else {  // P_t overwrites S_t: QK_{t,j+1} must follow PV_{t,j} (in-order tensor pipe)
-            issue_pv(j);
-            if (j + 1 < N) issue_qk(j + 1);
+          ++qkc;
+          const uint32_t qoff = C::OFF_Q + (2 * cu.qs + t) * C::TILE;
+          const uint32_t koff = sK - sbase;
+#pragma unroll
+          for (int kk = 0; kk < D / 16; ++kk) {
+            const uint32_t off = (kk / 4) * C::CHUNK + (kk % 4) * 32;
+            umma_ss_elect(tS, desc0 + ((qoff + off) >> 4), desc0 + ((koff + off) >> 4), IDESC_QK, kk > 0);
+          }
+          umma_commit_elect(S_FULL);
+          TRACE_EV(EV_MMA_QK, t * 64 + cu.j);
+          if (cu.j + 1 == cu.n) umma_commit_elect(Q_EMPTY(t, cu.qs));  // last QK of the tile: Q slot reusable
+        } else {
+          ring_wait(kidx);  // K_j unused by this tile: release it once loaded
+        }
+        umma_commit_elect(KV_EMPTY(kidx % C::NS));
+      };
+      // O_t (+)= P_t V_j once the softmax wrote P_t and the correction group rescaled O_t
+      auto issue_pv = [&](Cursor& cu) {
+        const uint32_t vidx = cu.base + 2 * cu.j + 1;
+        const uint32_t sV = ring_wait(vidx);
+        if (cu.j < cu.n) {
+          mbar_wait(P_FULL, pc & 1);
+          ++pc;
+          TRACE_EV(EV_MMA_P, t * 64 + cu.j);
+          mbar_wait(O_READY, oc & 1);
+          ++oc;
+          tc_fence_after();
+#pragma unroll
+          for (int kk = 0; kk < 8; ++kk)
+            umma_ts_elect(tO, tP + kk * 8, vdesc0 + ((sV - sbase + kk * 2048) >> 4), IDESC_PV, (cu.j > 0 || kk > 0));
+          umma_commit_elect(PV_DONE);
+          TRACE_EV(EV_MMA_PV, t * 64 + cu.j);
+        }
+        umma_commit_elect(KV_EMPTY(vidx % C::NS));
+      };
+      if (C::SEP_P) {
+        if (cq.valid) {
+          issue_qk(cq);
+          advance(cq);
+        }
+        while (cp.valid) {
+          if (cq.valid) {
+            issue_qk(cq);
+            advance(cq);
+          }
+          issue_pv(cp);
+          advance(cp);
+        }
+      } else {  // P_t overwrites S_t: QK_{t,g+1} must follow PV_{t,g} (in-order tensor pipe)
+        if (cq.valid) {
+          issue_qk(cq);
+          advance(cq);
+        }
+        while (cp.valid) {
+          issue_pv(cp);
+          advance(cp);
+          if (cq.valid) {
+            issue_qk(cq);
+            advance(cq);
           }
         }
       }
     }
-  } else if (warp < 8) {
-    asm volatile("setmaxnreg.inc.sync.aligned.u32 176;");
-    // ============================================================== softmax group t (a5, a6)
-    // The two groups take turns for the exp2 phase (named barriers 2 + t): while one group
-    // exponentiates, the other loads/reduces its next S and the tensor core runs the first
-    // group's PV and next QK, so MUFU and tensor pipes overlap instead of running in lockstep.
-    const int t = warp >> 2;
-    const int quad = warp & 3;
+  } else if (warp < 16) {
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(C::REG_SOFTMAX));
+    // ============================================================== softmax (a5, a6)
+    const int t = warp >> 3, h = (warp >> 2) & 1, quad = warp & 3;
     const int row = quad * 32 + lane;
-    const uint32_t tS = tmem + (static_cast<uint32_t>(quad * 32) << 16) + 128 * t;
+    const uint32_t lane_off = static_cast<uint32_t>(quad * 32) << 16;
+    const uint32_t tS = tmem + lane_off + 128 * t + 64 * h;  // this warp's 64 S columns
+    const uint32_t tP = tmem + lane_off + (C::SEP_P ? C::TMEM_P + 64 * t : 128 * t) + 32 * h;
+    const uint32_t S_FULL = BAR(C::B_S_FULL + t), P_FULL = BAR(C::B_P_FULL + t);
+    const uint32_t PV_DONE = BAR(C::B_PV_DONE + t), S_FREE = BAR(C::B_S_FREE + t);
+    const uint32_t ST_FULL = BAR(C::B_ST_FULL + t), ST_EMPTY = BAR(C::B_ST_EMPTY + t);
+    const uint32_t L_FULL = BAR(C::B_L_FULL + t);
+    const uint32_t pair_bar = 4 + 4 * t + quad;  // named barrier shared with the other column half
+    // The tiles take turns for the exp phase (named barriers 2, 3; 256 threads per tile): one
+    // tile's two warps per SMSP saturate MUFU while the other tile loads S and reduces its max.
+    const uint32_t my_turn = 2 + t, other_turn = 3 - t;
+    if (t == 1) named_bar_arrive(2, 512);  // tile 0 goes first
     const float c = p.scale_log2;
     const int off = p.seq_kv - p.seq_q;
-    const uint32_t my_turn = 2 + t, other_turn = 3 - t;
-    if (C::TURNS && t == 1) named_bar_arrive(2, 256);  // tile 0 goes first
-    const uint32_t tP = tmem + (static_cast<uint32_t>(quad * 32) << 16) + (C::SEP_P ? C::TMEM_P + 64 * t : 128 * t);
     uint32_t sc = 0, stc = 0, gstep = 0;
     for (int idx = first; idx < p.num_items; idx += stride) {
       const WorkItem w = decode_item(p, idx);
-      const int N = max(w.n[0], w.n[1]);
-      const int n = w.n[t];
+      const int N = max(w.n0, w.n1);
+      const int n = w.n(t);
       const int qi = w.q0 + 128 * t + row;
       int lim = w.kv_valid;  // keys j < lim are visible to this row
       if (p.mask_kind == MASK_CAUSAL) lim = min(lim, qi + off + 1);
+      lim -= 64 * h;         // ... in this warp's column coordinates
       float m_ref = -INFINITY;  // max used as the exp2 reference (lags the true max by < 2^8)
-      float l = 0.f;
+      float l = 0.f;            // this half's share of the row sum
       for (int j = 0; j < N; ++j) {
-        if (j >= n) {  // this tile has no KV tile j: keep the turn order
-          if (C::TURNS) {
-            named_bar_sync(my_turn, 256);
-            named_bar_arrive(other_turn, 256);
-          }
+        if (j >= n) {  // no KV tile j for this tile: pass the turn on
+          named_bar_sync(my_turn, 512);
+          named_bar_arrive(other_turn, 512);
           continue;
         }
         TRACE_EV(EV_S_WAIT, j);
-        mbar_wait(S_FULL(t), sc & 1);
+        mbar_wait(S_FULL, sc & 1);
         ++sc;
         TRACE_EV(EV_S_READY, j);
         tc_fence_after();
-        uint32_t s[128];
-#pragma unroll
-        for (int q = 0; q < 4; ++q) tmem_ld_32x32b_x32(tS + 32 * q, *reinterpret_cast<uint32_t(*)[32]>(&s[32 * q]));
+        uint32_t s[64];
+        tmem_ld_32x32b_x32(tS, *reinterpret_cast<uint32_t(*)[32]>(&s[0]));
+        tmem_ld_32x32b_x32(tS + 32, *reinterpret_cast<uint32_t(*)[32]>(&s[32]));
         tmem_wait_ld();
         reg_fence(s);
-        if (C::SEP_P) {  // S_t is in registers: the tensor core may overwrite it with S_{t,j+1}
+        if (C::SEP_P) {  // S_t read: the tensor core may overwrite it with S_{t,j+1}
           tc_fence_before();
-          mbar_arrive(S_FREE(t));
+          mbar_arrive(S_FREE);
         }
         const int rem = lim - j * 128;
-        if (rem < 128) {  // boundary tile for this row (a5)
+        if (rem < 64) {  // boundary tile for this row (a5)
 #pragma unroll
-          for (int k = 0; k < 128; ++k)
+          for (int k = 0; k < 64; ++k)
             if (k >= rem) s[k] = __float_as_uint(-INFINITY);
         }
-        float mx0 = m_ref, mx1 = -INFINITY;
+        float mx0 = m_ref, mx1 = -INFINITY, mx2 = -INFINITY, mx3 = -INFINITY;
 #pragma unroll
-        for (int k = 0; k < 128; k += 4) {
+        for (int k = 0; k < 64; k += 8) {
           mx0 = fmax3(mx0, __uint_as_float(s[k]), __uint_as_float(s[k + 1]));
           mx1 = fmax3(mx1, __uint_as_float(s[k + 2]), __uint_as_float(s[k + 3]));
+          mx2 = fmax3(mx2, __uint_as_float(s[k + 4]), __uint_as_float(s[k + 5]));
+          mx3 = fmax3(mx3, __uint_as_float(s[k + 6]), __uint_as_float(s[k + 7]));
         }
-        const float m_new = fmaxf(mx0, mx1);
+        // combine with the other column half of this row
+        float* slot = s_pmax + ((gstep & 1) * 4 + 2 * t) * 128;  // [parity][t][half][row]
+        slot[h * 128 + row] = fmaxf(fmaxf(mx0, mx1), fmaxf(mx2, mx3));
+        named_bar_sync(pair_bar, 64);
+        const float m_new = fmaxf(slot[row], slot[128 + row]);
+        TRACE_EV(EV_MAX_DONE, j);
         // Lazy rescale: keep the old reference while the max grows by < 8 in the log2 domain (the
         // p's then stay <= 2^8, exact in fp32 and in fp16/bf16 range); l and O share the reference.
         float alpha = 1.f;
@@ -412,28 +458,28 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           alpha = (m_ref == -INFINITY) ? 0.f : ex2((m_ref - m_new) * c);
           m_ref = m_new;
         }
-        // hand alpha to the correction group (it rescales O_t before PV_{t,j})
-        mbar_wait(ST_EMPTY(t), (stc & 1) ^ 1);
-        s_alpha[t * 128 + row] = (j == 0) ? 1.f : alpha;
-        mbar_arrive(ST_FULL(t));
-        ++stc;
-
+        if (h == 0) {  // hand alpha to the correction group (it rescales O_t before PV_{t,j})
+          mbar_wait(ST_EMPTY, (stc & 1) ^ 1);
+          s_alpha[t * 128 + row] = (j == 0) ? 1.f : alpha;
+          mbar_arrive(ST_FULL);
+          ++stc;
+        }
         const float mc = (m_ref == -INFINITY) ? 0.f : m_ref * c;
-        float2 acc0 = make_float2(0.f, 0.f), acc1 = make_float2(0.f, 0.f);
-        TRACE_EV(EV_MAX_DONE, j);
-        if (C::TURNS) named_bar_sync(my_turn, 256);
-        TRACE_EV(EV_TURN, j);
         if (C::SEP_P && gstep > 0) {  // P_t buffer still read by PV_{t,j-1}?
-          mbar_wait(PV_DONE(t), (gstep - 1) & 1);
+          mbar_wait(PV_DONE, (gstep - 1) & 1);
           tc_fence_after();
         }
         ++gstep;
+        // P = exp2(c*s - c*m_ref) (a6), rounded to the I/O type, stored to TMEM for the PV MMA
+        float2 acc0 = make_float2(0.f, 0.f), acc1 = make_float2(0.f, 0.f);
+        named_bar_sync(my_turn, 512);
+        TRACE_EV(EV_XCHG, j);
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
-          uint32_t pk[32];
+        for (int hh = 0; hh < 2; ++hh) {
+          uint32_t pk[16];
 #pragma unroll
-          for (int u = 0; u < 32; u += 2) {
-            const int k = 64 * h + 2 * u;
+          for (int u = 0; u < 16; u += 2) {
+            const int k = 32 * hh + 2 * u;
             float2 x0 = ffma2(make_float2(__uint_as_float(s[k]), __uint_as_float(s[k + 1])), c, -mc);
             float2 x1 = ffma2(make_float2(__uint_as_float(s[k + 2]), __uint_as_float(s[k + 3])), c, -mc);
             x0.x = ex2(x0.x);
@@ -445,24 +491,23 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             pk[u] = pack2<BF16>(x0.x, x0.y);
             pk[u + 1] = pack2<BF16>(x1.x, x1.y);
           }
-          tmem_st_32x32b_x32(tP + 32 * h, pk);
-          if (C::TURNS && C::HALF_TURN && h == 0) named_bar_arrive(other_turn, 256);
+          tmem_st_32x32b_x16(tP + 16 * hh, pk);
         }
-        if (C::TURNS && !C::HALF_TURN) named_bar_arrive(other_turn, 256);
+        named_bar_arrive(other_turn, 512);
         TRACE_EV(EV_EXP_DONE, j);
         tmem_wait_st();
         tc_fence_before();
-        mbar_arrive(P_FULL(t));
+        mbar_arrive(P_FULL);
         l = l * alpha + ((acc0.x + acc0.y) + (acc1.x + acc1.y));
       }
-      if (w.has[t]) {
-        s_lsum[t * 128 + row] = l;
-        mbar_arrive(L_FULL(t));
+      if (t == 0 || w.has1) {
+        s_lsum[(2 * t + h) * 128 + row] = l;
+        mbar_arrive(L_FULL);
       }
     }
-    if (C::TURNS && t == 0) named_bar_sync(2, 256);  // consume tile 1's last hand-over
+    if (t == 0) named_bar_sync(2, 512);  // consume tile 1's last hand-over
   } else {
-    asm volatile("setmaxnreg.dec.sync.aligned.u32 96;");
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(C::REG_CORR));
     // ================================================================ correction group (a7, a9)
     const int quad = warp & 3;
     const int row = quad * 32 + lane;
@@ -470,23 +515,23 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     uint32_t stc[2] = {0, 0}, pvc[2] = {0, 0}, lc[2] = {0, 0};
     for (int idx = first; idx < p.num_items; idx += stride) {
       const WorkItem w = decode_item(p, idx);
-      const int N = max(w.n[0], w.n[1]);
+      const int N = max(w.n0, w.n1);
       for (int j = 0; j < N; ++j) {
 #pragma unroll
         for (int t = 0; t < 2; ++t) {
-          if (j >= w.n[t]) continue;
-          mbar_wait(ST_FULL(t), stc[t] & 1);
+          if (j >= w.n(t)) continue;
+          mbar_wait(BAR(C::B_ST_FULL + t), stc[t] & 1);
           TRACE_EV(EV_COR_ST, t * 64 + j);
           const float alpha = s_alpha[t * 128 + row];
-          mbar_arrive(ST_EMPTY(t));
+          mbar_arrive(BAR(C::B_ST_EMPTY + t));
           ++stc[t];
           if (j > 0) {
-            mbar_wait(PV_DONE(t), pvc[t] & 1);  // PV_{t,j-1} has landed in O_t
+            mbar_wait(BAR(C::B_PV_DONE + t), pvc[t] & 1);  // PV_{t,j-1} has landed in O_t
             ++pvc[t];
             if (__any_sync(0xffffffffu, alpha != 1.f)) {
               tc_fence_after();
               const uint32_t tO = tmem + lane_off + 256 + t * D;
-#pragma unroll
+#pragma unroll 1
               for (int q = 0; q < D / 32; ++q) {
                 uint32_t o[32];
                 tmem_ld_32x32b_x32(tO + 32 * q, o);
@@ -500,19 +545,20 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             }
           }
           tc_fence_before();
-          mbar_arrive(O_READY(t));
+          mbar_arrive(BAR(C::B_O_READY + t));
           TRACE_EV(EV_COR_ORDY, t * 64 + j);
         }
       }
       // ------------------------------------------------------------ epilogue per tile (a9)
 #pragma unroll 1
       for (int t = 0; t < 2; ++t) {
-        if (!w.has[t]) continue;
-        mbar_wait(L_FULL(t), lc[t] & 1);
+        if (t == 1 && !w.has1) continue;
+        mbar_wait(BAR(C::B_L_FULL + t), lc[t] & 1);
         ++lc[t];
-        const float l = s_lsum[t * 128 + row];
-        if (w.n[t] > 0) {
-          mbar_wait(PV_DONE(t), pvc[t] & 1);  // last PV of this tile
+        const float l = s_lsum[(2 * t) * 128 + row] + s_lsum[(2 * t + 1) * 128 + row];
+        const int n = w.n(t);
+        if (n > 0) {
+          mbar_wait(BAR(C::B_PV_DONE + t), pvc[t] & 1);  // last PV of this tile
           ++pvc[t];
           tc_fence_after();
         }
@@ -521,10 +567,10 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         if (row == 0) tma_store_wait_read0();  // previous store out of this staging buffer done
         named_bar_sync(1, 128);
         const uint32_t tO = tmem + lane_off + 256 + t * D;
-#pragma unroll
+#pragma unroll 1
         for (int q = 0; q < D / 32; ++q) {
           uint32_t o[32];
-          if (w.n[t] > 0) {
+          if (n > 0) {
             tmem_ld_32x32b_x32(tO + 32 * q, o);
             tmem_wait_ld();
             reg_fence(o);
@@ -559,7 +605,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
 
   tc_fence_before();
   __syncthreads();
-  if (warp == 12) {
+  if (warp == 20) {
     tc_fence_after();
     tmem_dealloc(tmem, C::TMEM_COLS);
   }

@@ -17,7 +17,7 @@ import paper_conf_asplos_hagedornfccgg23_b200 as fm  # noqa: E402
 lib = _lib.load()
 lib.fmha_trace_set.argtypes = [ctypes.c_void_p]
 lib.fmha_trace_count.restype = ctypes.c_uint
-EV = {1: "S_WAIT", 2: "S_READY", 3: "MAX_DONE", 4: "TURN", 5: "EXP_DONE", 6: "MMA_P", 7: "MMA_O", 8: "MMA_PV",
+EV = {1: "S_WAIT", 2: "S_READY", 3: "MAX_DONE", 4: "XCHG", 5: "EXP_DONE", 6: "MMA_P", 7: "MMA_O", 8: "MMA_PV",
       9: "MMA_QK", 10: "COR_ST", 11: "COR_PV", 12: "COR_ORDY", 13: "EPI", 14: "TMA_KV", 15: "ITEM"}
 
 cfg = CONFIGS[sys.argv[1] if len(sys.argv) > 1 else "bert_large_512"]
@@ -25,7 +25,7 @@ q, k, v, kl = make_fmha_inputs(cfg)
 dev = torch.device("cuda:0")
 q, k, v = q.to(dev), k.to(dev), v.to(dev)
 kld = None if kl is None else torch.from_numpy(kl).to(dev)
-buf = torch.zeros(16 * 4096, dtype=torch.int64, device=dev)
+buf = torch.zeros(24 * 2048, dtype=torch.int64, device=dev)
 for it in range(3):
     buf.zero_()
     lib.fmha_trace_set(buf.data_ptr())
