@@ -10,7 +10,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "lib", "libb200fmha.so")
+# B200FMHA_LIB may name another build of the same library (tuning variants under lib/)
+LIB_PATH = os.environ.get("B200FMHA_LIB", os.path.join(_HERE, "lib", "libb200fmha.so"))
 
 FMHA_OK = 0
 STATUS_NAMES = {

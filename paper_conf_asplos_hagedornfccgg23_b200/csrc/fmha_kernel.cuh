@@ -112,8 +112,14 @@ struct FmhaCfg {
   static constexpr bool SEP_P = (D == 64);
   static constexpr int TMEM_P = 384;
   // registers after setmaxnreg.  setmaxnreg.inc only draws on the CTA's launch allocation
-  // (80 x 768 = 61440), so 16 x 32 x 96 + 4 x 32 x 56 + 4 x 32 x 40 = 61440 must not be exceeded.
-  static constexpr int REG_SOFTMAX = 96, REG_CORR = 56, REG_MISC = 40;
+  // (80 x 768 = 61440), so 16 x 32 x 96 + 4 x 32 x 48 + 4 x 32 x 48 = 61440 must not be exceeded.
+  static constexpr int REG_SOFTMAX = 96, REG_CORR = 48, REG_MISC = 48;
+  // exp2 of element pairs q (of 32 per half-row) with (q % POLY_MOD) < POLY_CNT runs on the
+  // FMA pipe (exp2_poly2) instead of MUFU: at D = 64 MUFU (16/clk/SM) is the bound.
+#ifndef FMHA_POLY_CNT
+#define FMHA_POLY_CNT 4
+#endif
+  static constexpr int POLY_MOD = 8, POLY_CNT = (D == 64) ? FMHA_POLY_CNT : 0;
   static_assert(16 * 32 * REG_SOFTMAX + 4 * 32 * REG_CORR + 4 * 32 * REG_MISC <= 80 * THREADS, "register pool");
   static_assert(SMEM_ALLOC <= 232448, "shared memory budget");
 };
@@ -482,10 +488,18 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
             const int k = 32 * hh + 2 * u;
             float2 x0 = ffma2(make_float2(__uint_as_float(s[k]), __uint_as_float(s[k + 1])), c, -mc);
             float2 x1 = ffma2(make_float2(__uint_as_float(s[k + 2]), __uint_as_float(s[k + 3])), c, -mc);
-            x0.x = ex2(x0.x);
-            x0.y = ex2(x0.y);
-            x1.x = ex2(x1.x);
-            x1.y = ex2(x1.y);
+            if (((16 * hh + u) % C::POLY_MOD) < C::POLY_CNT) {
+              x0 = exp2_poly2(x0);
+            } else {
+              x0.x = ex2(x0.x);
+              x0.y = ex2(x0.y);
+            }
+            if (((16 * hh + u + 1) % C::POLY_MOD) < C::POLY_CNT) {
+              x1 = exp2_poly2(x1);
+            } else {
+              x1.x = ex2(x1.x);
+              x1.y = ex2(x1.y);
+            }
             acc0 = fadd2(acc0, x0);
             acc1 = fadd2(acc1, x1);
             pk[u] = pack2<BF16>(x0.x, x0.y);

@@ -296,6 +296,26 @@ __device__ __forceinline__ float2 fmul2(float2 a, float2 b) {
   return u64_as_f2(r);
 }
 
+// 2^x for a pair on the FMA/ALU pipes (no MUFU), x <= 8: x = j + f with j = rint(x) taken from the
+// low mantissa bits of x + 1.5*2^23, f in [-1/2, 1/2]; 2^f = 1 + f (c1 + f (c2 + f c3)), fitted for
+// minimax relative error on [-1/2, 1/2] with the constant pinned to 1 (max 1.0e-4, below fp16's
+// half-ulp 2.4e-4); j is added to the exponent field.  x is clamped at -127, where f = 0 and the
+// polynomial is exactly 1.0, so -inf (masked scores) gives exactly +0 -- a fully masked row keeps
+// l = 0 and its O = 0.
+__device__ __forceinline__ float2 exp2_poly2(float2 x) {
+  x.x = fmaxf(x.x, -127.f);
+  x.y = fmaxf(x.y, -127.f);
+  const float2 t = fadd2(x, make_float2(12582912.f, 12582912.f));
+  const float2 jf = fadd2(t, make_float2(-12582912.f, -12582912.f));
+  const float2 f = fadd2(x, make_float2(-jf.x, -jf.y));
+  float2 q = ffma2(f, make_float2(0.055008720606565475f, 0.055008720606565475f),
+                   make_float2(0.24221046268939972f, 0.24221046268939972f));
+  q = ffma2(q, f, make_float2(0.6932829022407532f, 0.6932829022407532f));
+  q = ffma2(q, f, make_float2(1.0f, 1.0f));
+  return make_float2(__int_as_float(__float_as_int(q.x) + (__float_as_int(t.x) << 23)),
+                     __int_as_float(__float_as_int(q.y) + (__float_as_int(t.y) << 23)));
+}
+
 template <bool BF16>
 __device__ __forceinline__ uint32_t pack2(float lo, float hi);
 template <>
