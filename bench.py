@@ -27,7 +27,7 @@ sys.path.insert(0, ROOT)
 import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
-from workloads import CONFIGS, MASK_CAUSAL, MASK_KEY_PADDING, make_fmha_inputs  # noqa: E402
+from workloads import CONFIGS, MASK_CAUSAL, MASK_KEY_PADDING, make_fmha_inputs, shard  # noqa: E402
 
 METRIC = "FMHA fwd TFLOP/s & % of B200 fp16 tensor peak at BERT-large shapes, 1/2/4/8 GPU"
 SPEC_TFLOPS = 2250.0
@@ -142,16 +142,20 @@ def main():
     ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", default="bert_large_512", choices=sorted(CONFIGS))
+    ap.add_argument("--workload", default="bert_large_512", choices=sorted(CONFIGS) + ["mlp"])
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of CPU oracle timing")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--scaling", choices=["weak", "strong"], default="weak",
+                    help="weak: each rank runs the whole config on its own batch; strong: ranks split its batch")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.workload == "mlp":
+        return run_mlp(args, world, rank, local)
     cfg = CONFIGS[args.workload]
 
     if args.impl == "reference":
@@ -166,7 +170,8 @@ def main():
 
     import paper_conf_asplos_hagedornfccgg23_b200 as fm
 
-    q, k, v, kv_len = make_fmha_inputs(cfg, batch_offset=rank * cfg.batch)  # weak scaling: own batch
+    cfg, offset = shard(cfg, rank, world, args.scaling)  # weak: own batch; strong: a slice of it
+    q, k, v, kv_len = make_fmha_inputs(cfg, batch_offset=offset)
     set_bytes = alg_bytes(cfg)
     n_sets = max(1, int(np.ceil(3 * L2_BYTES / set_bytes)))  # rotate > 3x L2 of inputs+outputs
     qd, kd, vd = q.to(dev), k.to(dev), v.to(dev)
@@ -246,7 +251,8 @@ def main():
 
     # ---- check this rank's last output against sampled oracle rows (cheap sanity, not timed)
     from oracle import attention_rows_fp64
-    units = [(0, 0, 0), (cfg.batch - 1, cfg.heads - 1, cfg.seq_q - 1), (cfg.batch // 2, 1, cfg.seq_q // 3)]
+    units = [(0, 0, 0), (cfg.batch - 1, cfg.heads - 1, cfg.seq_q - 1),
+             (cfg.batch // 2, min(1, cfg.heads - 1), cfg.seq_q // 3)]
     ref = attention_rows_fp64(q, k, v, cfg.scale, units, kv_len, causal)
     o_last = sets[(args.steps - 1) % n_sets][3]
     got = np.stack([o_last[b, h, i].double().cpu().numpy() for b, h, i in units])
@@ -267,7 +273,7 @@ def main():
         line = {
             "metric": METRIC, "value": round(value, 2), "unit": "TFLOP/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 5),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None,
             "dtype": "f16" if cfg.dtype == "fp16" else "bf16", "data": "synthetic",
             "config": {"workload": cfg.name, "batch_per_gpu": cfg.batch, "heads": cfg.heads, "seq_q": cfg.seq_q,
                        "seq_kv": cfg.seq_kv, "head_dim": cfg.head_dim,
@@ -289,6 +295,55 @@ def main():
         print(json.dumps(line), flush=True)
     if dist:
         dist.destroy_process_group()
+
+
+def run_mlp(args, world, rank, local):
+    """BASELINE.json config 5: Transformer MLP block, tokens=16384, 1024 -> 4096 (+bias, GELU) -> 1024
+    (+bias), fp16, two gemm_bias_act launches per step."""
+    from workloads import MLP_CONFIG, make_mlp_inputs
+    import paper_conf_asplos_hagedornfccgg23_b200 as fm
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    cfg = MLP_CONFIG
+    x, w1, b1, w2, b2 = (t.to(dev) for t in make_mlp_inputs(cfg))
+    h = torch.empty((cfg.tokens, cfg.d_ff), dtype=torch.float16, device=dev)
+    y = torch.empty((cfg.tokens, cfg.d_model), dtype=torch.float16, device=dev)
+
+    def step():
+        fm.gemm_bias_act(x, w1, b1, act="gelu", out=h)
+        fm.gemm_bias_act(h, w2, b2, act="none", out=y)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    graph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(graph):
+        for _ in range(args.steps):
+            step()
+    graph.replay()
+    torch.cuda.synchronize()
+    stream = torch.cuda.current_stream(dev)
+    sampler = ClockSampler(local)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with sampler:
+        torch.cuda.synchronize()
+        e0.record(stream)
+        graph.replay()
+        e1.record(stream)
+        torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / args.steps
+    flops = 2.0 * cfg.tokens * cfg.d_model * cfg.d_ff * 2
+    peak_burst, _, _, src = measured_peaks()
+    val = flops / (ms * 1e-3) / 1e12
+    if rank == 0:
+        print(json.dumps({"metric": "MLP block (GEMM+bias+GELU, GEMM+bias) TFLOP/s", "value": round(val, 2),
+                          "unit": "TFLOP/s", "n_gpus": 1, "steps": args.steps, "warmup": args.warmup,
+                          "ms_per_step": round(ms, 5), "higher_is_better": True, "dtype": "f16", "data": "synthetic",
+                          "config": {"workload": "mlp", "tokens": cfg.tokens, "d_model": cfg.d_model, "d_ff": cfg.d_ff},
+                          "clocks": sampler.summary(), "gpu_launches": 2 * args.steps,
+                          "roofline": {"bound": "tensor", "achieved": round(val, 2), "peak": peak_burst,
+                                       "unit": "TFLOP/s", "frac": round(val / peak_burst, 4),
+                                       "peak_source": f"{src} bf16 dense burst"}}), flush=True)
 
 
 def run_reference(args, cfg, world, rank):

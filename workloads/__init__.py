@@ -122,6 +122,21 @@ def make_fmha_inputs(cfg: FmhaConfig, batch_offset: int = 0, seed: int = SEED):
     return _round(q, td), _round(k, td), _round(v, td), kv_lengths(cfg, batch_offset, seed)
 
 
+def shard(cfg: FmhaConfig, rank: int, world: int, scaling: str = "weak"):
+    """The multi-GPU partition: every (b, h) is independent, so ranks split by batch.
+    weak:   every rank runs the whole config on its own batch (global batch = world * cfg.batch);
+    strong: the config's batch is split into `world` contiguous ranges (batch must divide).
+    Returns (local config, global batch offset)."""
+    if scaling == "weak":
+        return cfg, rank * cfg.batch
+    if scaling != "strong":
+        raise ValueError(scaling)
+    if cfg.batch % world:
+        raise ValueError(f"batch {cfg.batch} does not split over {world} ranks")
+    b = cfg.batch // world
+    return cfg.with_(batch=b), rank * b
+
+
 def make_mlp_inputs(cfg: MlpConfig = MLP_CONFIG, tokens: int | None = None, seed: int = SEED):
     """Returns (x [T,d_model], w1 [d_ff,d_model], b1 [d_ff], w2 [d_model,d_ff], b2 [d_model])
     as fp16 CPU tensors."""
