@@ -116,6 +116,10 @@ struct FmhaCfg {
   static constexpr int REG_SOFTMAX = 96, REG_CORR = 48, REG_MISC = 48;
   // exp2 of element pairs q (of 32 per half-row) with (q % POLY_MOD) < POLY_CNT runs on the
   // FMA pipe (exp2_poly2) instead of MUFU: at D = 64 MUFU (16/clk/SM) is the bound.
+#ifndef FMHA_TURNS
+#define FMHA_TURNS 1
+#endif
+  static constexpr bool TURNS = FMHA_TURNS;
 #ifndef FMHA_POLY_CNT
 #define FMHA_POLY_CNT 4
 #endif
@@ -403,7 +407,7 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
     // The tiles take turns for the exp phase (named barriers 2, 3; 256 threads per tile): one
     // tile's two warps per SMSP saturate MUFU while the other tile loads S and reduces its max.
     const uint32_t my_turn = 2 + t, other_turn = 3 - t;
-    if (t == 1) named_bar_arrive(2, 512);  // tile 0 goes first
+    if (C::TURNS && t == 1) named_bar_arrive(2, 512);  // tile 0 goes first
     const float c = p.scale_log2;
     const int off = p.seq_kv - p.seq_q;
     uint32_t sc = 0, stc = 0, gstep = 0;
@@ -419,8 +423,10 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
       float l = 0.f;            // this half's share of the row sum
       for (int j = 0; j < N; ++j) {
         if (j >= n) {  // no KV tile j for this tile: pass the turn on
-          named_bar_sync(my_turn, 512);
-          named_bar_arrive(other_turn, 512);
+          if (C::TURNS) {
+            named_bar_sync(my_turn, 512);
+            named_bar_arrive(other_turn, 512);
+          }
           continue;
         }
         TRACE_EV(EV_S_WAIT, j);
@@ -478,7 +484,7 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
         ++gstep;
         // P = exp2(c*s - c*m_ref) (a6), rounded to the I/O type, stored to TMEM for the PV MMA
         float2 acc0 = make_float2(0.f, 0.f), acc1 = make_float2(0.f, 0.f);
-        named_bar_sync(my_turn, 512);
+        if (C::TURNS) named_bar_sync(my_turn, 512);
         TRACE_EV(EV_XCHG, j);
 #pragma unroll
         for (int hh = 0; hh < 2; ++hh) {
@@ -507,7 +513,7 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
           }
           tmem_st_32x32b_x16(tP + 16 * hh, pk);
         }
-        named_bar_arrive(other_turn, 512);
+        if (C::TURNS) named_bar_arrive(other_turn, 512);
         TRACE_EV(EV_EXP_DONE, j);
         tmem_wait_st();
         tc_fence_before();
@@ -519,7 +525,7 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
         mbar_arrive(L_FULL);
       }
     }
-    if (t == 0) named_bar_sync(2, 512);  // consume tile 1's last hand-over
+    if (C::TURNS && t == 0) named_bar_sync(2, 512);  // consume tile 1's last hand-over
   } else {
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(C::REG_CORR));
     // ================================================================ correction group (a7, a9)
