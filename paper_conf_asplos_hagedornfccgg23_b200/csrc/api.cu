@@ -99,14 +99,14 @@ bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) ==
 template <int D, bool BF16>
 int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) {
   using C = b200::FmhaCfg<D>;
-  auto kern = b200::fmha_fwd_sm100<D, BF16>;
-  static bool attr_done[64];
+  auto kern = prm.pair_mode ? b200::fmha_fwd_sm100<D, BF16, true> : b200::fmha_fwd_sm100<D, BF16, false>;
+  static bool attr_done[64][2];
   int dev = 0;
   cudaGetDevice(&dev);
-  if (dev >= 64 || !attr_done[dev]) {
+  if (dev >= 64 || !attr_done[dev][prm.pair_mode]) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_ALLOC);
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(fmha)");
-    if (dev < 64) attr_done[dev] = true;
+    if (dev < 64) attr_done[dev][prm.pair_mode] = true;
   }
   // persistent: one CTA per SM (or fewer when there is less work)
   dim3 grid(static_cast<unsigned>(std::min(prm.num_items, sm_count)), 1, 1);
@@ -155,8 +155,12 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   // scores (-inf) still map to exp2(-inf) = 0 instead of -inf * 0 = NaN.  1e-30 perturbs visible
   // scores by < 1e-25 in the exponent.
   prm.scale_log2 = std::max(scale * 1.4426950408889634f, 1e-30f);
-  const long long items = units * ((prm.num_q_tiles + 1) / 2);
-  if (items > 2147483647LL) return FMHA_ERR_UNSUPPORTED;
+  // odd q-tile counts >= 3 (non-causal): pair tiles across units so no item has an empty second
+  // tile (BERT-large-384: +8%).  With a single q-tile per unit (short sequences) every item is one
+  // latency-bound step and pairing across units measured slower, so those keep pair_mode 0.
+  prm.pair_mode = (kind != FMHA_MASK_CAUSAL && (prm.num_q_tiles & 1) && prm.num_q_tiles >= 3) ? 1 : 0;
+  const long long items = prm.pair_mode ? (units * prm.num_q_tiles + 1) / 2 : units * ((prm.num_q_tiles + 1) / 2);
+  if (items > 2147483647LL || units * prm.num_q_tiles > 2147483647LL) return FMHA_ERR_UNSUPPORTED;
   prm.num_items = static_cast<int>(items);
 
   if (head_dim == 64)

@@ -78,7 +78,10 @@ struct FmhaParams {
   int heads;
   int num_q_tiles;
   int num_units;  // B*H
-  int num_items;  // num_units * ceil(num_q_tiles / 2)
+  int num_items;  // see pair_mode
+  int pair_mode;  // 0: items are q-tiles {2i, 2i+1} of one unit (num_units * ceil(num_q_tiles / 2) items)
+                  // 1: items are tiles {2i, 2i+1} of the flattened (unit, q-tile) list, so a tile pair
+                  //    may straddle two units (odd num_q_tiles, non-causal): no half-empty items
   int mask_kind;
   float scale_log2;  // scale * log2(e)
 };
@@ -102,7 +105,7 @@ struct FmhaCfg {
   // barrier slots
   enum : int {
     B_S_FULL = 0, B_P_FULL = 2, B_O_READY = 4, B_PV_DONE = 6, B_ST_FULL = 8, B_ST_EMPTY = 10, B_L_FULL = 12,
-    B_S_FREE = 14, B_Q_FULL = 16, B_Q_EMPTY = 20, B_KV = 24
+    B_S_FREE = 14, B_Q_FULL = 16, B_Q_EMPTY = 20, B_L_EMPTY = 24, B_KV = 26
   };
   static constexpr int NUM_BARS = B_KV + 2 * NS;
   static constexpr int OFF_TMEMPTR = OFF_BAR + NUM_BARS * 8;
@@ -128,43 +131,76 @@ struct FmhaCfg {
   static_assert(SMEM_ALLOC <= 232448, "shared memory budget");
 };
 
-// One work item = q-tiles {2*pair, 2*pair+1} of unit bh.  Every role decodes items identically.
+// One work item = two 128-row query tiles t = 0, 1.  Every role decodes items identically.
+// shared: both tiles belong to one unit and share every K/V tile; otherwise (pair_mode 1) each tile
+// streams its own K/V through the ring (entries of tile 0 then tile 1 for every step j).
 struct WorkItem {
-  int bh;
-  int q0;        // first query row of tile 0
-  int kv_valid;  // keys >= kv_valid are masked for every row (key padding)
-  int n0, n1;    // KV tiles visited by tile 0 / 1 (0 = tile absent or fully masked)
+  int bh0, bh1;  // units of tile 0 / 1
+  int r0, r1;    // first query row of tile 0 / 1
+  int kv0, kv1;  // keys >= kv_t are masked for every row of tile t (key padding)
+  int n0, n1;    // KV tiles visited by tile t (0 = tile absent or fully masked)
   bool has1;     // tile 1 exists (tile 0 always does)
+  bool shared;
   __device__ __forceinline__ int n(int t) const { return t ? n1 : n0; }
+  __device__ __forceinline__ int bh(int t) const { return t ? bh1 : bh0; }
+  __device__ __forceinline__ int row0(int t) const { return t ? r1 : r0; }
+  __device__ __forceinline__ int kv(int t) const { return t ? kv1 : kv0; }
+  // number of K/V ring entries the item uses, and the ring index of K_{t,j} (V = K + 1)
+  __device__ __forceinline__ int entries() const { return shared ? 2 * max(n0, n1) : 2 * (n0 + n1); }
+  __device__ __forceinline__ int k_index(int t, int j) const {
+    return shared ? 2 * j : 2 * (min(j, n0) + min(j, n1)) + ((t == 1 && j < n0) ? 2 : 0);
+  }
 };
 
+template <bool PAIRX>
 __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
   WorkItem w;
-  const int pairs = (p.num_q_tiles + 1) >> 1;
-  int pr;
-  if (p.mask_kind == MASK_CAUSAL) {  // longest-first: the last query tiles see the most keys
-    pr = pairs - 1 - idx / p.num_units;
-    w.bh = idx % p.num_units;
-  } else {  // both pairs of a (b,h) back to back so K/V are re-read from L2
-    w.bh = idx / pairs;
-    pr = idx % pairs;
+  int qt0;
+  if (!PAIRX) {
+    const int pairs = (p.num_q_tiles + 1) >> 1;
+    int pr;
+    if (p.mask_kind == MASK_CAUSAL) {  // longest-first: the last query tiles see the most keys
+      pr = pairs - 1 - idx / p.num_units;
+      w.bh0 = idx % p.num_units;
+    } else {  // both pairs of a (b,h) back to back so K/V are re-read from L2
+      w.bh0 = idx / pairs;
+      pr = idx % pairs;
+    }
+    qt0 = 2 * pr;
+    w.bh1 = w.bh0;
+    w.has1 = qt0 + 1 < p.num_q_tiles;
+    w.shared = true;
+    w.r0 = qt0 * 128;
+    w.r1 = w.r0 + 128;
+  } else {
+    const int a = 2 * idx, b = 2 * idx + 1;
+    w.bh0 = a / p.num_q_tiles;
+    qt0 = a - w.bh0 * p.num_q_tiles;
+    w.bh1 = b / p.num_q_tiles;
+    const int qt1 = b - w.bh1 * p.num_q_tiles;
+    w.has1 = b < p.num_units * p.num_q_tiles;
+    w.shared = w.has1 && w.bh1 == w.bh0;
+    w.r0 = qt0 * 128;
+    w.r1 = qt1 * 128;
   }
-  w.q0 = pr * 256;
-  w.kv_valid = p.seq_kv;
-  if (p.mask_kind == MASK_KEY_PADDING) w.kv_valid = min(max(__ldg(p.kv_len + w.bh / p.heads), 0), p.seq_kv);
+  w.kv0 = w.kv1 = p.seq_kv;
+  if (p.mask_kind == MASK_KEY_PADDING) {
+    w.kv0 = min(max(__ldg(p.kv_len + w.bh0 / p.heads), 0), p.seq_kv);
+    w.kv1 = w.shared ? w.kv0 : min(max(__ldg(p.kv_len + min(w.bh1, p.num_units - 1) / p.heads), 0), p.seq_kv);
+  }
   const int off = p.seq_kv - p.seq_q;
-  int kv_end0 = w.kv_valid, kv_end1 = w.kv_valid;
+  int kv_end0 = w.kv0, kv_end1 = w.kv1;
   if (p.mask_kind == MASK_CAUSAL) {
-    kv_end0 = min(kv_end0, max(0, w.q0 + 128 + off));
-    kv_end1 = min(kv_end1, max(0, w.q0 + 256 + off));
+    kv_end0 = min(kv_end0, max(0, w.r0 + 128 + off));
+    kv_end1 = min(kv_end1, max(0, w.r1 + 128 + off));
   }
-  w.has1 = 2 * pr + 1 < p.num_q_tiles;
   w.n0 = (kv_end0 + 127) / 128;
   w.n1 = w.has1 ? (kv_end1 + 127) / 128 : 0;
   return w;
 }
 
-template <int D, bool BF16>
+// PAIRX = (pair_mode == 1): items may pair tiles of two units (see FmhaParams::pair_mode).
+template <int D, bool BF16, bool PAIRX>
 __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
   using C = FmhaCfg<D>;
   // Dynamic shared memory starts at the (1024-byte aligned) base of the CTA's shared window; the
@@ -196,6 +232,7 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
       mbar_init(BAR(C::B_ST_FULL + t), 128);  // half-0 softmax threads
       mbar_init(BAR(C::B_ST_EMPTY + t), 128);
       mbar_init(BAR(C::B_L_FULL + t), 256);
+      mbar_init(BAR(C::B_L_EMPTY + t), 128);  // correction threads, after reading the row sums
       mbar_init(BAR(C::B_S_FREE + t), 256);
       for (int q = 0; q < 2; ++q) {
         mbar_init(Q_FULL(t, q), 1);
@@ -231,42 +268,50 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
       const uint64_t keep = policy_evict_last();   // K/V: re-read by the other q-tile pairs
       const uint64_t once = policy_evict_first();  // Q: read once
       uint32_t kv = 0, qc0 = 0, qc1 = 0;
+      auto load_kv = [&](int bh, int j) {
+#pragma unroll
+        for (int m = 0; m < 2; ++m, ++kv) {  // m = 0: K_j, m = 1: V_j
+          const int s = kv % C::NS;
+          mbar_wait_at(KV_EMPTY(s), ((kv / C::NS) & 1) ^ 1, 1, kv, j);
+          TRACE_EV(EV_TMA_KV, m * 64 + j);
+          mbar_arrive_expect_tx_elect(KV_FULL(s), C::TILE);
+          const CUtensorMap* map = m ? &p.tmV : &p.tmK;
+#pragma unroll
+          for (int c = 0; c < D / 64; ++c)
+            tma_load_3d_hint_elect(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64,
+                                   j * 128, bh, keep);
+        }
+      };
       for (int idx = first; idx < p.num_items; idx += stride) {
-        const WorkItem w = decode_item(p, idx);
+        const WorkItem w = decode_item<PAIRX>(p, idx);
         const int N = max(w.n0, w.n1);
 #pragma unroll
         for (int t = 0; t < 2; ++t) {
           if (w.n(t) == 0) continue;
           uint32_t& qc = t ? qc1 : qc0;
           const int qs = qc % C::QS;
-          mbar_wait(Q_EMPTY(t, qs), ((qc / C::QS) & 1) ^ 1);
+          mbar_wait_at(Q_EMPTY(t, qs), ((qc / C::QS) & 1) ^ 1, 2, qc, t);
           mbar_arrive_expect_tx_elect(Q_FULL(t, qs), C::TILE);
 #pragma unroll
           for (int c = 0; c < D / 64; ++c)
             tma_load_3d_hint_elect(sbase + C::OFF_Q + (2 * qs + t) * C::TILE + c * C::CHUNK, &p.tmQ, Q_FULL(t, qs),
-                                   c * 64, w.q0 + 128 * t, w.bh, once);
+                                   c * 64, w.row0(t), w.bh(t), once);
           ++qc;
           TRACE_EV(EV_ITEM, 4 + t);
         }
         for (int j = 0; j < N; ++j) {
-#pragma unroll
-          for (int m = 0; m < 2; ++m, ++kv) {  // m = 0: K_j, m = 1: V_j
-            const int s = kv % C::NS;
-            mbar_wait(KV_EMPTY(s), ((kv / C::NS) & 1) ^ 1);
-            TRACE_EV(EV_TMA_KV, m * 64 + j);
-            mbar_arrive_expect_tx_elect(KV_FULL(s), C::TILE);
-            const CUtensorMap* map = m ? &p.tmV : &p.tmK;
-#pragma unroll
-            for (int c = 0; c < D / 64; ++c)
-              tma_load_3d_hint_elect(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64,
-                                     j * 128, w.bh, keep);
+          if (w.shared) {
+            load_kv(w.bh0, j);
+          } else {
+            if (j < w.n0) load_kv(w.bh0, j);
+            if (j < w.n1) load_kv(w.bh1, j);
           }
         }
       }
     } else if (warp == 20 || warp == 21) {
       // ============================================================ MMA issuers (a4, a8)
       // Warp 20 issues tile 0's MMAs, warp 21 tile 1's, so each tile's chain (QK -> softmax ->
-      // PV) depends only on its own softmax warps.  Both warps release every K/V slot (count 2).
+      // PV) depends only on its own softmax warps.  Both warps release every K/V entry (count 2).
       const int t = warp - 20;
       constexpr uint32_t IDESC_QK = idesc_f16(BF16, 128, 128, false, false);  // Q, K: K-major
       constexpr uint32_t IDESC_PV = idesc_f16(BF16, 128, D, false, true);     // P: K-major (TMEM), V: MN-major
@@ -281,114 +326,144 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
       const uint32_t S_FREE = BAR(C::B_S_FREE + t);
       uint32_t qc = 0, pc = 0, oc = 0, qkc = 0;
       auto ring_wait = [&](uint32_t k) {
-        mbar_wait(KV_FULL(k % C::NS), (k / C::NS) & 1);
+        mbar_wait_at(KV_FULL(k % C::NS), (k / C::NS) & 1, 3, k, 0);
         tc_fence_after();
         return sbase + C::OFF_RING + (k % C::NS) * C::TILE;
       };
       // Two cursors walk the same sequence of (item, KV step j): the QK cursor runs one step ahead
       // of the PV cursor (behind it when P aliases S), across item boundaries, so the next item's
       // first S is computed while the current item's last P is still being produced.
+      struct Ring {  // the part of a WorkItem the ring arithmetic needs
+        int n0, n1;
+        bool shared;
+        __device__ __forceinline__ int n(int t) const { return t ? n1 : n0; }
+        __device__ __forceinline__ int entries() const { return shared ? 2 * max(n0, n1) : 2 * (n0 + n1); }
+        __device__ __forceinline__ int k_index(int t, int j) const {
+          return shared ? 2 * j : 2 * (min(j, n0) + min(j, n1)) + ((t == 1 && j < n0) ? 2 : 0);
+        }
+      };
       struct Cursor {
-        int idx, j, N, n, qs;
-        uint32_t base;  // ring index of K_0 of the item; K_j = base + 2j, V_j = base + 2j + 1
+        Ring w;
+        int idx, j, N, qs;
+        uint32_t base;  // ring index of the item's first K/V entry (WorkItem::k_index)
         bool valid;
       };
       auto seek = [&](Cursor& cu, int idx, uint32_t base) {
         cu.valid = false;
         for (; idx < p.num_items; idx += stride) {
-          const WorkItem w = decode_item(p, idx);
+          const WorkItem w = decode_item<PAIRX>(p, idx);
           const int N = max(w.n0, w.n1);
           if (N == 0) continue;
+          cu.w.n0 = w.n0;
+          cu.w.n1 = w.n1;
+          cu.w.shared = w.shared;
           cu.idx = idx;
           cu.j = 0;
           cu.N = N;
-          cu.n = w.n(t);
           cu.base = base;
           cu.valid = true;
           return;
         }
       };
       auto advance = [&](Cursor& cu) {
-        if (++cu.j == cu.N) seek(cu, cu.idx + stride, cu.base + 2 * cu.N);
+        if (++cu.j == cu.N) seek(cu, cu.idx + stride, cu.base + cu.w.entries());
       };
       Cursor cq, cp;
       seek(cq, first, 0);
       cp = cq;
       // S_t <- Q_t K_j^T (separate P: once the softmax warps have read the previous S_t)
-      auto issue_qk = [&](Cursor& cu) {
-        const uint32_t kidx = cu.base + 2 * cu.j;
-        if (cu.j < cu.n) {
-          if (cu.j == 0) {  // first QK of this item's tile t: its Q tile must have landed
-            cu.qs = qc % C::QS;
-            mbar_wait(Q_FULL(t, cu.qs), (qc / C::QS) & 1);
-            ++qc;
-          }
-          const uint32_t sK = ring_wait(kidx);
-          if (C::SEP_P && qkc > 0) {
-            mbar_wait(S_FREE, (qkc - 1) & 1);
-            tc_fence_after();
-          }
-          ++qkc;
-          const uint32_t qoff = C::OFF_Q + (2 * cu.qs + t) * C::TILE;
-          const uint32_t koff = sK - sbase;
-#pragma unroll
-          for (int kk = 0; kk < D / 16; ++kk) {
-            const uint32_t off = (kk / 4) * C::CHUNK + (kk % 4) * 32;
-            umma_ss_elect(tS, desc0 + ((qoff + off) >> 4), desc0 + ((koff + off) >> 4), IDESC_QK, kk > 0);
-          }
-          umma_commit_elect(S_FULL);
-          TRACE_EV(EV_MMA_QK, t * 64 + cu.j);
-          if (cu.j + 1 == cu.n) umma_commit_elect(Q_EMPTY(t, cu.qs));  // last QK of the tile: Q slot reusable
-        } else {
-          ring_wait(kidx);  // K_j unused by this tile: release it once loaded
-        }
+      // Every K/V ring entry is released exactly once by each MMA warp (KV_EMPTY count 2): a warp
+      // that does not use an entry waits for it to be filled, then commits.  (Two back-to-back
+      // commits from one thread to one barrier are not a reliable way to arrive twice.)
+      auto release = [&](uint32_t kidx) {
+        ring_wait(kidx);
         umma_commit_elect(KV_EMPTY(kidx % C::NS));
       };
-      // O_t (+)= P_t V_j once the softmax wrote P_t and the correction group rescaled O_t
-      auto issue_pv = [&](Cursor& cu) {
-        const uint32_t vidx = cu.base + 2 * cu.j + 1;
-        const uint32_t sV = ring_wait(vidx);
-        if (cu.j < cu.n) {
-          mbar_wait(P_FULL, pc & 1);
-          ++pc;
-          TRACE_EV(EV_MMA_P, t * 64 + cu.j);
-          mbar_wait(O_READY, oc & 1);
-          ++oc;
-          tc_fence_after();
-#pragma unroll
-          for (int kk = 0; kk < 8; ++kk)
-            umma_ts_elect(tO, tP + kk * 8, vdesc0 + ((sV - sbase + kk * 2048) >> 4), IDESC_PV, (cu.j > 0 || kk > 0));
-          umma_commit_elect(PV_DONE);
-          TRACE_EV(EV_MMA_PV, t * 64 + cu.j);
+      // S_t <- Q_t K_{t,j}^T (separate P: once the softmax warps have read the previous S_t)
+      auto qk_entry = [&](Cursor& cu, uint32_t kidx) {
+        const int n = cu.w.n(t);
+        const uint32_t sK = ring_wait(kidx);
+        if (cu.j == 0) {  // first QK of this item's tile t: its Q tile must have landed
+          cu.qs = qc % C::QS;
+          mbar_wait_at(Q_FULL(t, cu.qs), (qc / C::QS) & 1, 4, qc, cu.idx);
+          ++qc;
         }
+        if (C::SEP_P && qkc > 0) {
+          mbar_wait_at(S_FREE, (qkc - 1) & 1, 5, qkc, cu.idx);
+          tc_fence_after();
+        }
+        ++qkc;
+        const uint32_t qoff = C::OFF_Q + (2 * cu.qs + t) * C::TILE;
+        const uint32_t koff = sK - sbase;
+#pragma unroll
+        for (int kk = 0; kk < D / 16; ++kk) {
+          const uint32_t off = (kk / 4) * C::CHUNK + (kk % 4) * 32;
+          umma_ss_elect(tS, desc0 + ((qoff + off) >> 4), desc0 + ((koff + off) >> 4), IDESC_QK, kk > 0);
+        }
+        umma_commit_elect(S_FULL);
+        TRACE_EV(EV_MMA_QK, t * 64 + cu.j);
+        if (cu.j + 1 == n) umma_commit_elect(Q_EMPTY(t, cu.qs));  // last QK of the tile: Q slot reusable
+        umma_commit_elect(KV_EMPTY(kidx % C::NS));
+      };
+      // O_t (+)= P_t V_{t,j} once the softmax wrote P_t and the correction group rescaled O_t
+      auto pv_entry = [&](Cursor& cu, uint32_t vidx) {
+        const uint32_t sV = ring_wait(vidx);
+        mbar_wait_at(P_FULL, pc & 1, 6, pc, cu.idx);
+        ++pc;
+        TRACE_EV(EV_MMA_P, t * 64 + cu.j);
+        mbar_wait_at(O_READY, oc & 1, 7, oc, cu.idx);
+        ++oc;
+        tc_fence_after();
+#pragma unroll
+        for (int kk = 0; kk < 8; ++kk)
+          umma_ts_elect(tO, tP + kk * 8, vdesc0 + ((sV - sbase + kk * 2048) >> 4), IDESC_PV, (cu.j > 0 || kk > 0));
+        umma_commit_elect(PV_DONE);
+        TRACE_EV(EV_MMA_PV, t * 64 + cu.j);
         umma_commit_elect(KV_EMPTY(vidx % C::NS));
       };
-      if (C::SEP_P) {
+      // walk the ring entries of step j in ring order: use this tile's, release the rest
+      auto issue_qk = [&](Cursor& cu) {
+        for (int u = 0; u < (cu.w.shared ? 1 : 2); ++u) {
+          const int uu = cu.w.shared ? t : u;  // tile whose entry this is
+          if (cu.j >= cu.w.n(uu)) {
+            if (cu.w.shared) release(cu.base + cu.w.k_index(t, cu.j));
+            continue;
+          }
+          const uint32_t kidx = cu.base + cu.w.k_index(uu, cu.j);
+          if (uu == t) qk_entry(cu, kidx);
+          else release(kidx);
+        }
+      };
+      auto issue_pv = [&](Cursor& cu) {
+        for (int u = 0; u < (cu.w.shared ? 1 : 2); ++u) {
+          const int uu = cu.w.shared ? t : u;
+          if (cu.j >= cu.w.n(uu)) {
+            if (cu.w.shared) release(cu.base + cu.w.k_index(t, cu.j) + 1);
+            continue;
+          }
+          const uint32_t vidx = cu.base + cu.w.k_index(uu, cu.j) + 1;
+          if (uu == t) pv_entry(cu, vidx);
+          else release(vidx);
+        }
+      };
+      // One loop, one call site each (keeps the issuing code small).  With separate P the QK
+      // cursor leads (QK of step s+1 before PV of step s); with P over S it follows.
+      bool started = false;
+      while (cp.valid) {
+        if (!C::SEP_P && started) {
+          issue_pv(cp);
+          advance(cp);
+          if (!cp.valid) break;
+        }
         if (cq.valid) {
           issue_qk(cq);
           advance(cq);
         }
-        while (cp.valid) {
-          if (cq.valid) {
-            issue_qk(cq);
-            advance(cq);
-          }
+        if (C::SEP_P && started) {
           issue_pv(cp);
           advance(cp);
         }
-      } else {  // P_t overwrites S_t: QK_{t,g+1} must follow PV_{t,g} (in-order tensor pipe)
-        if (cq.valid) {
-          issue_qk(cq);
-          advance(cq);
-        }
-        while (cp.valid) {
-          issue_pv(cp);
-          advance(cp);
-          if (cq.valid) {
-            issue_qk(cq);
-            advance(cq);
-          }
-        }
+        started = true;
       }
     }
   } else if (warp < 16) {
@@ -402,7 +477,7 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
     const uint32_t S_FULL = BAR(C::B_S_FULL + t), P_FULL = BAR(C::B_P_FULL + t);
     const uint32_t PV_DONE = BAR(C::B_PV_DONE + t), S_FREE = BAR(C::B_S_FREE + t);
     const uint32_t ST_FULL = BAR(C::B_ST_FULL + t), ST_EMPTY = BAR(C::B_ST_EMPTY + t);
-    const uint32_t L_FULL = BAR(C::B_L_FULL + t);
+    const uint32_t L_FULL = BAR(C::B_L_FULL + t), L_EMPTY = BAR(C::B_L_EMPTY + t);
     const uint32_t pair_bar = 4 + 4 * t + quad;  // named barrier shared with the other column half
     // The tiles take turns for the exp phase (named barriers 2, 3; 256 threads per tile): one
     // tile's two warps per SMSP saturate MUFU while the other tile loads S and reduces its max.
@@ -410,13 +485,15 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
     if (C::TURNS && t == 1) named_bar_arrive(2, 512);  // tile 0 goes first
     const float c = p.scale_log2;
     const int off = p.seq_kv - p.seq_q;
-    uint32_t sc = 0, stc = 0, gstep = 0;
+    // g = real steps this warp has done so far: the phase count of S_FULL, ST_EMPTY, PV_DONE and
+    // the max-exchange slot parity are all g (one counter keeps the 96-register budget)
+    uint32_t g = 0, lc = 0;
     for (int idx = first; idx < p.num_items; idx += stride) {
-      const WorkItem w = decode_item(p, idx);
+      const WorkItem w = decode_item<PAIRX>(p, idx);
       const int N = max(w.n0, w.n1);
       const int n = w.n(t);
-      const int qi = w.q0 + 128 * t + row;
-      int lim = w.kv_valid;  // keys j < lim are visible to this row
+      const int qi = w.row0(t) + row;
+      int lim = w.kv(t);  // keys j < lim are visible to this row
       if (p.mask_kind == MASK_CAUSAL) lim = min(lim, qi + off + 1);
       lim -= 64 * h;         // ... in this warp's column coordinates
       float m_ref = -INFINITY;  // max used as the exp2 reference (lags the true max by < 2^8)
@@ -430,8 +507,7 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
           continue;
         }
         TRACE_EV(EV_S_WAIT, j);
-        mbar_wait(S_FULL, sc & 1);
-        ++sc;
+        mbar_wait_at(S_FULL, g & 1, 8, g, idx);
         TRACE_EV(EV_S_READY, j);
         tc_fence_after();
         uint32_t s[64];
@@ -458,7 +534,7 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
           mx3 = fmax3(mx3, __uint_as_float(s[k + 6]), __uint_as_float(s[k + 7]));
         }
         // combine with the other column half of this row
-        float* slot = s_pmax + ((gstep & 1) * 4 + 2 * t) * 128;  // [parity][t][half][row]
+        float* slot = s_pmax + ((g & 1) * 4 + 2 * t) * 128;  // [parity][t][half][row]
         slot[h * 128 + row] = fmaxf(fmaxf(mx0, mx1), fmaxf(mx2, mx3));
         named_bar_sync(pair_bar, 64);
         const float m_new = fmaxf(slot[row], slot[128 + row]);
@@ -471,17 +547,16 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
           m_ref = m_new;
         }
         if (h == 0) {  // hand alpha to the correction group (it rescales O_t before PV_{t,j})
-          mbar_wait(ST_EMPTY, (stc & 1) ^ 1);
+          mbar_wait_at(ST_EMPTY, (g & 1) ^ 1, 9, g, idx);
           s_alpha[t * 128 + row] = (j == 0) ? 1.f : alpha;
           mbar_arrive(ST_FULL);
-          ++stc;
         }
         const float mc = (m_ref == -INFINITY) ? 0.f : m_ref * c;
-        if (C::SEP_P && gstep > 0) {  // P_t buffer still read by PV_{t,j-1}?
-          mbar_wait(PV_DONE, (gstep - 1) & 1);
+        if (C::SEP_P && g > 0) {  // P_t buffer still read by PV_{t,j-1}?
+          mbar_wait_at(PV_DONE, (g - 1) & 1, 10, g, idx);
           tc_fence_after();
         }
-        ++gstep;
+        ++g;
         // P = exp2(c*s - c*m_ref) (a6), rounded to the I/O type, stored to TMEM for the PV MMA
         float2 acc0 = make_float2(0.f, 0.f), acc1 = make_float2(0.f, 0.f);
         if (C::TURNS) named_bar_sync(my_turn, 512);
@@ -521,6 +596,12 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
         l = l * alpha + ((acc0.x + acc0.y) + (acc1.x + acc1.y));
       }
       if (t == 0 || w.has1) {
+        // the correction group has read the previous item's sums (without this wait the softmax can
+        // run two items ahead and L_FULL's phase parity would alias)
+#ifndef FMHA_NO_LEMPTY
+        mbar_wait_at(L_EMPTY, (lc & 1) ^ 1, 15, lc, idx);
+#endif
+        ++lc;
         s_lsum[(2 * t + h) * 128 + row] = l;
         mbar_arrive(L_FULL);
       }
@@ -534,19 +615,19 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
     const uint32_t lane_off = static_cast<uint32_t>(quad * 32) << 16;
     uint32_t stc[2] = {0, 0}, pvc[2] = {0, 0}, lc[2] = {0, 0};
     for (int idx = first; idx < p.num_items; idx += stride) {
-      const WorkItem w = decode_item(p, idx);
+      const WorkItem w = decode_item<PAIRX>(p, idx);
       const int N = max(w.n0, w.n1);
       for (int j = 0; j < N; ++j) {
 #pragma unroll
         for (int t = 0; t < 2; ++t) {
           if (j >= w.n(t)) continue;
-          mbar_wait(BAR(C::B_ST_FULL + t), stc[t] & 1);
+          mbar_wait_at(BAR(C::B_ST_FULL + t), stc[t] & 1, 11, stc[t], idx);
           TRACE_EV(EV_COR_ST, t * 64 + j);
           const float alpha = s_alpha[t * 128 + row];
           mbar_arrive(BAR(C::B_ST_EMPTY + t));
           ++stc[t];
           if (j > 0) {
-            mbar_wait(BAR(C::B_PV_DONE + t), pvc[t] & 1);  // PV_{t,j-1} has landed in O_t
+            mbar_wait_at(BAR(C::B_PV_DONE + t), pvc[t] & 1, 12, pvc[t], idx);  // PV_{t,j-1} has landed in O_t
             ++pvc[t];
             if (__any_sync(0xffffffffu, alpha != 1.f)) {
               tc_fence_after();
@@ -573,12 +654,13 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
 #pragma unroll 1
       for (int t = 0; t < 2; ++t) {
         if (t == 1 && !w.has1) continue;
-        mbar_wait(BAR(C::B_L_FULL + t), lc[t] & 1);
+        mbar_wait_at(BAR(C::B_L_FULL + t), lc[t] & 1, 13, lc[t], idx);
         ++lc[t];
         const float l = s_lsum[(2 * t) * 128 + row] + s_lsum[(2 * t + 1) * 128 + row];
+        mbar_arrive(BAR(C::B_L_EMPTY + t));
         const int n = w.n(t);
         if (n > 0) {
-          mbar_wait(BAR(C::B_PV_DONE + t), pvc[t] & 1);  // last PV of this tile
+          mbar_wait_at(BAR(C::B_PV_DONE + t), pvc[t] & 1, 14, pvc[t], idx);  // last PV of this tile
           ++pvc[t];
           tc_fence_after();
         }
@@ -615,7 +697,7 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
         if (row == 0) {
 #pragma unroll
           for (int c2 = 0; c2 < D / 64; ++c2)
-            tma_store_3d(&p.tmO, stg + c2 * C::CHUNK, c2 * 64, w.q0 + 128 * t, w.bh);
+            tma_store_3d(&p.tmO, stg + c2 * C::CHUNK, c2 * 64, w.row0(t), w.bh(t));
           tma_store_commit();
         }
       }

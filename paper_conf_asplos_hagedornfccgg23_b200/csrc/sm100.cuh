@@ -9,6 +9,7 @@
 #include <cuda.h>
 #include <cuda_fp16.h>
 #include <cuda_bf16.h>
+#include <cstdio>
 
 #include "tmem_ops.cuh"
 
@@ -46,10 +47,42 @@ __device__ __forceinline__ bool mbar_try_wait(uint32_t bar, uint32_t parity) {
       : "memory");
   return ok != 0;
 }
-// Wait until the phase with the given parity has completed.
+// Wait until the phase with the given parity has completed.  Debug builds (-DB200_HANG_CHECK=1)
+// report the stuck barrier (smem offset, parity, block, warp) and trap instead of spinning forever.
+#ifndef B200_HANG_CHECK
+#define B200_HANG_CHECK 0
+#endif
 __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+#if B200_HANG_CHECK
+  long long spins = 0;
+  while (!mbar_try_wait(bar, parity)) {
+    ++spins;
+    if (spins == (1ll << 22) && (threadIdx.x & 31) == 0)  // report, keep waiting so every stuck warp reports
+      printf("HANG block %d warp %d bar_off 0x%x parity %u\n", blockIdx.x, threadIdx.x >> 5, bar & 0xFFFFF, parity);
+    if (spins == (1ll << 24)) __trap();
+  }
+#else
   while (!mbar_try_wait(bar, parity)) {
   }
+#endif
+}
+
+// Same, tagged with a call site and two counters for the hang report (debug builds only).
+__device__ __forceinline__ void mbar_wait_at(uint32_t bar, uint32_t parity, int site, int a, int b) {
+#if B200_HANG_CHECK
+  long long spins = 0;
+  while (!mbar_try_wait(bar, parity)) {
+    ++spins;
+    if (spins == (1ll << 22) && (threadIdx.x & 31) == 0)
+      printf("HANG block %d warp %d site %d a %d b %d parity %u\n", blockIdx.x, threadIdx.x >> 5, site, a, b, parity);
+    if (spins == (1ll << 24)) __trap();
+  }
+#else
+  (void)site;
+  (void)a;
+  (void)b;
+  mbar_wait(bar, parity);
+#endif
 }
 
 // ------------------------------------------------------------------ TMA
