@@ -163,3 +163,25 @@ def test_from_host_entry_point_matches(name):
     fm.fmha_fwd_from_host(pq, pk, pv, out, ws, kv_len=klh, causal=cfg.mask == MASK_CAUSAL, scale=cfg.scale)
     torch.cuda.synchronize()
     assert torch.equal(out, o.cpu())
+
+
+# ------------------------------------------------------------------ regression: pipeline deadlocks
+@pytest.mark.timeout(240)
+@pytest.mark.parametrize("name,batch", [("bert_base_pad", 32), ("bert_large_384", 32), ("bert_large_512", 8)])
+def test_back_to_back_launches_do_not_hang(name, batch):
+    """Many items per persistent CTA, many launches back to back: exercises the K/V ring release
+    (each MMA warp commits once per entry) and the L_FULL / L_EMPTY hand-off that used to run two
+    phases ahead when items are a single step long.  A hang fails this test by timeout."""
+    cfg = CONFIGS[name].with_(batch=batch)
+    q, k, v, kl = make_fmha_inputs(cfg)
+    qd, kd, vd = q.to(DEV), k.to(DEV), v.to(DEV)
+    kld = None if kl is None else torch.from_numpy(kl).to(DEV)
+    out = torch.empty_like(qd)
+    first = None
+    for i in range(30):
+        fm.fmha_fwd(qd, kd, vd, kv_len=kld, scale=cfg.scale, out=out)
+        if i == 0:
+            torch.cuda.synchronize()
+            first = out.clone()
+    torch.cuda.synchronize()
+    assert torch.equal(out, first)
