@@ -124,9 +124,20 @@ struct FmhaCfg {
 #endif
   static constexpr bool TURNS = FMHA_TURNS;
 #ifndef FMHA_POLY_CNT
-#define FMHA_POLY_CNT 4
+#define FMHA_POLY_CNT 3
 #endif
-  static constexpr int POLY_MOD = 8, POLY_CNT = (D == 64) ? FMHA_POLY_CNT : 0;
+#ifndef FMHA_POLY_MOD
+#define FMHA_POLY_MOD 8
+#endif
+  static constexpr int POLY_MOD = FMHA_POLY_MOD, POLY_CNT = (D == 64) ? FMHA_POLY_CNT : 0;
+#ifndef FMHA_POLY_MASK
+#define FMHA_POLY_MASK 0
+#endif
+  // optional explicit 8-bit pattern over (pair index % 8); 0 = use POLY_MOD / POLY_CNT
+  static constexpr unsigned POLY_MASK = FMHA_POLY_MASK;
+  static __host__ __device__ constexpr bool poly_pair(int q) {
+    return D != 64 ? false : (POLY_MASK ? ((POLY_MASK >> (q % 8)) & 1u) != 0 : (q % POLY_MOD) < POLY_CNT);
+  }
   static_assert(16 * 32 * REG_SOFTMAX + 4 * 32 * REG_CORR + 4 * 32 * REG_MISC <= 80 * THREADS, "register pool");
   static_assert(SMEM_ALLOC <= 232448, "shared memory budget");
 };
@@ -552,14 +563,19 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
           mbar_arrive(ST_FULL);
         }
         const float mc = (m_ref == -INFINITY) ? 0.f : m_ref * c;
+        TRACE_EV(EV_COR_ST, j);  // after the stats hand-off
         if (C::SEP_P && g > 0) {  // P_t buffer still read by PV_{t,j-1}?
           mbar_wait_at(PV_DONE, (g - 1) & 1, 10, g, idx);
           tc_fence_after();
         }
+        TRACE_EV(EV_COR_PV, j);  // after the PV_DONE wait
         ++g;
         // P = exp2(c*s - c*m_ref) (a6), rounded to the I/O type, stored to TMEM for the PV MMA
         float2 acc0 = make_float2(0.f, 0.f), acc1 = make_float2(0.f, 0.f);
         if (C::TURNS) named_bar_sync(my_turn, 512);
+#if FMHA_TRACE
+        if (*reinterpret_cast<volatile float*>(s_lsum) == 12345.f) m_ref += 1.f;  // force the deferred barrier block here
+#endif
         TRACE_EV(EV_XCHG, j);
 #pragma unroll
         for (int hh = 0; hh < 2; ++hh) {
@@ -569,13 +585,23 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
             const int k = 32 * hh + 2 * u;
             float2 x0 = ffma2(make_float2(__uint_as_float(s[k]), __uint_as_float(s[k + 1])), c, -mc);
             float2 x1 = ffma2(make_float2(__uint_as_float(s[k + 2]), __uint_as_float(s[k + 3])), c, -mc);
-            if (((16 * hh + u) % C::POLY_MOD) < C::POLY_CNT) {
+#ifdef FMHA_FAKE_EXP  // timing experiment only: exponentials replaced by a trivial op (wrong results)
+            if (true) {
+              x0 = fadd2(x0, make_float2(1.f, 1.f));
+            } else
+#endif
+            if (C::poly_pair(16 * hh + u)) {
               x0 = exp2_poly2(x0);
             } else {
               x0.x = ex2(x0.x);
               x0.y = ex2(x0.y);
             }
-            if (((16 * hh + u + 1) % C::POLY_MOD) < C::POLY_CNT) {
+#ifdef FMHA_FAKE_EXP
+            if (true) {
+              x1 = fadd2(x1, make_float2(1.f, 1.f));
+            } else
+#endif
+            if (C::poly_pair(16 * hh + u + 1)) {
               x1 = exp2_poly2(x1);
             } else {
               x1.x = ex2(x1.x);
@@ -591,6 +617,7 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
         if (C::TURNS) named_bar_arrive(other_turn, 512);
         TRACE_EV(EV_EXP_DONE, j);
         tmem_wait_st();
+        TRACE_EV(EV_EPI, j);  // P stores landed
         tc_fence_before();
         mbar_arrive(P_FULL);
         l = l * alpha + ((acc0.x + acc0.y) + (acc1.x + acc1.y));
