@@ -162,6 +162,10 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   const long long items = prm.pair_mode ? (units * prm.num_q_tiles + 1) / 2 : units * ((prm.num_q_tiles + 1) / 2);
   if (items > 2147483647LL || units * prm.num_q_tiles > 2147483647LL) return FMHA_ERR_UNSUPPORTED;
   prm.num_items = static_cast<int>(items);
+  prm.div_units.init(static_cast<uint32_t>(std::max(prm.num_units, 1)));
+  prm.div_pairs.init(static_cast<uint32_t>(std::max((prm.num_q_tiles + 1) / 2, 1)));
+  prm.div_qtiles.init(static_cast<uint32_t>(std::max(prm.num_q_tiles, 1)));
+  prm.div_heads.init(static_cast<uint32_t>(std::max(heads, 1)));
 
   if (head_dim == 64)
     return bf16 ? launch_fmha<64, true>(prm, sm_count, stream) : launch_fmha<64, false>(prm, sm_count, stream);

@@ -7,15 +7,16 @@
 //
 //   work item     two consecutive 128-row query tiles (t = 0, 1) of one (b, h) sharing every
 //                 K/V tile load; persistent CTAs (one per SM) walk a static item list        [a1]
-//   warps 0-15    softmax: warp (t, h, q) = 8t + 4h + q handles rows 32q..32q+31 of tile t and
-//                 key columns 64h..64h+63 of every 128-key S tile (two warps per row, so each
-//                 SMSP runs four softmax warps and MUFU.EX2 never idles on one warp's latency;
-//                 the two halves exchange their partial row max through smem)              [a5, a6]
-//   warps 16-19   correction: rescale O_t in TMEM when a row max grew by more than 2^8
-//                 (lazy), then the epilogue O_t / l -> fp16/bf16 -> smem -> TMA store      [a7, a9]
-//   warps 20, 21  MMA issuers for tile 0 / tile 1 (one elected lane each):
+//   warps 0-7     softmax: warpgroup t (warps 4t..4t+3) owns tile t, one thread per query row
+//                 and all 128 key columns of every S tile, so the row max and row sum are
+//                 thread-local (192 registers per thread after setmaxnreg)                 [a5, a6]
+//                 A softmax warp also rescales its own 32 rows of O_t in TMEM when a row max
+//                 grew by more than 2^8 (lazy rescale, rare), so PV_{t,j} waits only for P  [a7]
+//   warps 8-11    epilogue: O_t / l -> fp16/bf16 -> smem -> TMA store                      [a9]
+//   warps 12, 13  MMA issuers for tile 0 / tile 1 (one elected lane each):
 //                 S_t = Q_t K_j^T (SS), O_t += P_t V_j (TS)                                [a4, a8]
-//   warp 22       TMA producer: Q_t per item (double-buffered at D=64), K_j / V_j ring     [a2, a3]
+//   warp 14       TMA producer: Q_t per item (double-buffered at D=64), K_j / V_j ring     [a2, a3]
+//   warp 15       idle (completes warpgroup 3 for setmaxnreg)
 //
 //   TMEM (512 columns x 128 lanes, fp32):  S_0 [0,128)  S_1 [128,256)  O_0 [256,256+D)  O_1 [..+D)
 //   D = 64 : P_t (16-bit, two per column) has its own columns [384 + 64t, 448 + 64t), so
@@ -28,8 +29,7 @@
 //   * tcgen05.commit arrives once all earlier tcgen05 ops of the issuing thread have completed.
 //
 // Because tcgen05.ld 32x32b gives each thread whole TMEM lanes (= query rows), row statistics are
-// thread-local: no warp-shuffle reductions.  The two column halves of a row meet
-// through one 4-byte smem slot per row and a 64-thread named barrier.
+// thread-local: no warp-shuffle reductions and no cross-warp exchange.
 #pragma once
 #include "sm100.cuh"
 
@@ -67,6 +67,22 @@ enum : int { EV_S_WAIT = 1, EV_S_READY, EV_MAX_DONE, EV_XCHG, EV_EXP_DONE, EV_MM
 
 enum : int { MASK_NONE = 0, MASK_KEY_PADDING = 1, MASK_CAUSAL = 2 };
 
+// Division by a launch constant without the integer-divide sequence (whose MUFU.RCP would queue
+// behind the softmax's exponentials): q = (umulhi(n, m) + n) >> s, exact for 0 <= n < 2^31.
+struct FastDiv {
+  uint32_t d, m, s;
+  __host__ void init(uint32_t div) {
+    d = div;
+    s = 0;
+    while ((1ull << s) < div) ++s;
+    m = static_cast<uint32_t>(((1ull << 32) * ((1ull << s) - div)) / div + 1);
+  }
+  __device__ __forceinline__ int div(int n) const {
+    return static_cast<int>((__umulhi(static_cast<uint32_t>(n), m) + static_cast<uint32_t>(n)) >> s);
+  }
+  __device__ __forceinline__ int mod(int n, int q) const { return n - q * static_cast<int>(d); }
+};
+
 struct FmhaParams {
   CUtensorMap tmQ;  // 3-D {D, seq_q, B*H}, box {64, 128, 1}, SWIZZLE_128B
   CUtensorMap tmK;  // 3-D {D, seq_kv, B*H}
@@ -84,6 +100,7 @@ struct FmhaParams {
                   //    may straddle two units (odd num_q_tiles, non-causal): no half-empty items
   int mask_kind;
   float scale_log2;  // scale * log2(e)
+  FastDiv div_units, div_pairs, div_qtiles, div_heads;  // num_units, ceil(num_q_tiles/2), num_q_tiles, heads
 };
 
 template <int D>
@@ -98,33 +115,42 @@ struct FmhaCfg {
   static constexpr int OFF_Q = 0;               // Q[stage][tile]
   static constexpr int OFF_RING = 2 * QS * TILE;
   static constexpr int OFF_STG = OFF_RING + NS * TILE;
-  static constexpr int OFF_ALPHA = OFF_STG + NSTG * TILE;  // float alpha[2 tiles][128 rows]
-  static constexpr int OFF_LSUM = OFF_ALPHA + 2 * 128 * 4;  // float l[2 tiles][2 halves][128]
-  static constexpr int OFF_PMAX = OFF_LSUM + 4 * 128 * 4;   // float pmax[2 parity][2][2][128]
-  static constexpr int OFF_BAR = OFF_PMAX + 8 * 128 * 4;
+  static constexpr int OFF_LSUM = OFF_STG + NSTG * TILE;  // float l[2 tiles][128 rows]
+  static constexpr int OFF_MC = OFF_LSUM + 2 * 128 * 4;    // float mc[2 tiles][128 rows] (turn fence)
+  static constexpr int OFF_BAR = OFF_MC + 2 * 128 * 4;
   // barrier slots
   enum : int {
-    B_S_FULL = 0, B_P_FULL = 2, B_O_READY = 4, B_PV_DONE = 6, B_ST_FULL = 8, B_ST_EMPTY = 10, B_L_FULL = 12,
+    B_S_FULL = 0, B_P_FULL = 2, B_O_FULL = 4, B_PV_DONE = 6, B_O_EMPTY = 8, B_L_FULL = 12,
     B_S_FREE = 14, B_Q_FULL = 16, B_Q_EMPTY = 20, B_L_EMPTY = 24, B_KV = 26
   };
   static constexpr int NUM_BARS = B_KV + 2 * NS;
   static constexpr int OFF_TMEMPTR = OFF_BAR + NUM_BARS * 8;
   static constexpr int SMEM_ALLOC = OFF_TMEMPTR + 16;
   static constexpr int TMEM_COLS = 512;
-  static constexpr int THREADS = 768;
+  static constexpr int THREADS = 512;
+  static constexpr int W_CORR = 8, W_MMA = 12, W_TMA = 14;  // first warp of each role
   static constexpr bool SEP_P = (D == 64);
   static constexpr int TMEM_P = 384;
   // registers after setmaxnreg.  setmaxnreg.inc only draws on the CTA's launch allocation
-  // (80 x 768 = 61440), so 16 x 32 x 96 + 4 x 32 x 48 + 4 x 32 x 48 = 61440 must not be exceeded.
-  static constexpr int REG_SOFTMAX = 96, REG_CORR = 48, REG_MISC = 48;
-  // exp2 of element pairs q (of 32 per half-row) with (q % POLY_MOD) < POLY_CNT runs on the
-  // FMA pipe (exp2_poly2) instead of MUFU: at D = 64 MUFU (16/clk/SM) is the bound.
+  // (128 x 512 = 65536), so 8 x 32 x 192 + 4 x 32 x 80 + 4 x 32 x 48 = 65536 must not be exceeded.
+  static constexpr int REG_SOFTMAX = 192, REG_CORR = 80, REG_MISC = 48;
+  // The two tiles' softmax warps on one SMSP (warps q and 4 + q) take turns for the exp phase, so
+  // one tile's exponentials overlap the other's S load and row max (named barriers 2..9).
 #ifndef FMHA_TURNS
 #define FMHA_TURNS 1
 #endif
   static constexpr bool TURNS = FMHA_TURNS;
+  // The first PRE_CHUNKS of the four 32-column chunks of a row are exponentiated before the turn
+  // (overlapping the other tile's turn), the rest inside it.
+#ifndef FMHA_PRE_CHUNKS
+#define FMHA_PRE_CHUNKS ((D == 128) ? 0 : 1)
+#endif
+  static constexpr int PRE_CHUNKS = TURNS ? FMHA_PRE_CHUNKS : 4;
+  static_assert(!TURNS || (PRE_CHUNKS >= 0 && PRE_CHUNKS < 4), "the turn barrier sits before chunk PRE_CHUNKS");
+  // exp2 of element pairs q (of 64 per row) with (q % POLY_MOD) < POLY_CNT runs on the FMA pipe
+  // (exp2_poly2) instead of MUFU: at D = 64 MUFU (16/clk/SM) is the bound.
 #ifndef FMHA_POLY_CNT
-#define FMHA_POLY_CNT 3
+#define FMHA_POLY_CNT 2
 #endif
 #ifndef FMHA_POLY_MOD
 #define FMHA_POLY_MOD 8
@@ -138,7 +164,7 @@ struct FmhaCfg {
   static __host__ __device__ constexpr bool poly_pair(int q) {
     return D != 64 ? false : (POLY_MASK ? ((POLY_MASK >> (q % 8)) & 1u) != 0 : (q % POLY_MOD) < POLY_CNT);
   }
-  static_assert(16 * 32 * REG_SOFTMAX + 4 * 32 * REG_CORR + 4 * 32 * REG_MISC <= 80 * THREADS, "register pool");
+  static_assert(8 * 32 * REG_SOFTMAX + 4 * 32 * REG_CORR + 4 * 32 * REG_MISC <= 128 * THREADS, "register pool");
   static_assert(SMEM_ALLOC <= 232448, "shared memory budget");
 };
 
@@ -171,11 +197,12 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
     const int pairs = (p.num_q_tiles + 1) >> 1;
     int pr;
     if (p.mask_kind == MASK_CAUSAL) {  // longest-first: the last query tiles see the most keys
-      pr = pairs - 1 - idx / p.num_units;
-      w.bh0 = idx % p.num_units;
+      const int q = p.div_units.div(idx);
+      pr = pairs - 1 - q;
+      w.bh0 = p.div_units.mod(idx, q);
     } else {  // both pairs of a (b,h) back to back so K/V are re-read from L2
-      w.bh0 = idx / pairs;
-      pr = idx % pairs;
+      w.bh0 = p.div_pairs.div(idx);
+      pr = p.div_pairs.mod(idx, w.bh0);
     }
     qt0 = 2 * pr;
     w.bh1 = w.bh0;
@@ -185,9 +212,9 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
     w.r1 = w.r0 + 128;
   } else {
     const int a = 2 * idx, b = 2 * idx + 1;
-    w.bh0 = a / p.num_q_tiles;
+    w.bh0 = p.div_qtiles.div(a);
     qt0 = a - w.bh0 * p.num_q_tiles;
-    w.bh1 = b / p.num_q_tiles;
+    w.bh1 = p.div_qtiles.div(b);
     const int qt1 = b - w.bh1 * p.num_q_tiles;
     w.has1 = b < p.num_units * p.num_q_tiles;
     w.shared = w.has1 && w.bh1 == w.bh0;
@@ -196,8 +223,9 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
   }
   w.kv0 = w.kv1 = p.seq_kv;
   if (p.mask_kind == MASK_KEY_PADDING) {
-    w.kv0 = min(max(__ldg(p.kv_len + w.bh0 / p.heads), 0), p.seq_kv);
-    w.kv1 = w.shared ? w.kv0 : min(max(__ldg(p.kv_len + min(w.bh1, p.num_units - 1) / p.heads), 0), p.seq_kv);
+    w.kv0 = min(max(__ldg(p.kv_len + p.div_heads.div(w.bh0)), 0), p.seq_kv);
+    w.kv1 = w.shared ? w.kv0
+                     : min(max(__ldg(p.kv_len + p.div_heads.div(min(w.bh1, p.num_units - 1))), 0), p.seq_kv);
   }
   const int off = p.seq_kv - p.seq_q;
   int kv_end0 = w.kv0, kv_end1 = w.kv1;
@@ -212,7 +240,7 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
 
 // PAIRX = (pair_mode == 1): items may pair tiles of two units (see FmhaParams::pair_mode).
 template <int D, bool BF16, bool PAIRX>
-__global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
+__global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
   using C = FmhaCfg<D>;
   // Dynamic shared memory starts at the (1024-byte aligned) base of the CTA's shared window; the
   // SWIZZLE_128B tiles need that alignment.  Using the base directly keeps smem addresses uniform.
@@ -224,9 +252,7 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
   auto Q_EMPTY = [&](int t, int q) { return BAR(C::B_Q_EMPTY + 2 * q + t); };
   auto KV_FULL = [&](int s) { return BAR(C::B_KV + s); };
   auto KV_EMPTY = [&](int s) { return BAR(C::B_KV + C::NS + s); };
-  float* s_alpha = reinterpret_cast<float*>(smem + C::OFF_ALPHA);
   float* s_lsum = reinterpret_cast<float*>(smem + C::OFF_LSUM);
-  float* s_pmax = reinterpret_cast<float*>(smem + C::OFF_PMAX);
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(smem + C::OFF_TMEMPTR);
 
   const int warp = warp_id();
@@ -237,14 +263,13 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
     if (sbase & 1023u) __trap();  // the layout below assumes a 1024-byte aligned window
     for (int t = 0; t < 2; ++t) {
       mbar_init(BAR(C::B_S_FULL + t), 1);
-      mbar_init(BAR(C::B_P_FULL + t), 256);   // both column halves of all 128 rows
-      mbar_init(BAR(C::B_O_READY + t), 128);  // correction threads
+      mbar_init(BAR(C::B_P_FULL + t), 128);   // softmax threads of tile t (one per row)
+      mbar_init(BAR(C::B_O_FULL + t), 1);     // last PV of the tile committed
+      mbar_init(BAR(C::B_O_EMPTY + t), 128);  // epilogue threads have read O_t
       mbar_init(BAR(C::B_PV_DONE + t), 1);
-      mbar_init(BAR(C::B_ST_FULL + t), 128);  // half-0 softmax threads
-      mbar_init(BAR(C::B_ST_EMPTY + t), 128);
-      mbar_init(BAR(C::B_L_FULL + t), 256);
-      mbar_init(BAR(C::B_L_EMPTY + t), 128);  // correction threads, after reading the row sums
-      mbar_init(BAR(C::B_S_FREE + t), 256);
+      mbar_init(BAR(C::B_L_FULL + t), 128);
+      mbar_init(BAR(C::B_L_EMPTY + t), 128);  // epilogue threads, after reading the row sums
+      mbar_init(BAR(C::B_S_FREE + t), 128);
       for (int q = 0; q < 2; ++q) {
         mbar_init(Q_FULL(t, q), 1);
         mbar_init(Q_EMPTY(t, q), 1);
@@ -256,13 +281,13 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
     }
     fence_mbar_init();
   }
-  if (warp == 22 && lane == 0) {
+  if (warp == C::W_TMA && lane == 0) {
     tma_prefetch_desc(&p.tmQ);
     tma_prefetch_desc(&p.tmK);
     tma_prefetch_desc(&p.tmV);
     tma_prefetch_desc(&p.tmO);
   }
-  if (warp == 20) {
+  if (warp == C::W_MMA) {
     tmem_alloc(smem_u32(tmem_holder), C::TMEM_COLS);
     tmem_relinquish();
   }
@@ -272,9 +297,9 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
   const uint32_t tmem = *tmem_holder;
   const int first = blockIdx.x, stride = gridDim.x;
 
-  if (warp >= 20) {
+  if (warp >= C::W_MMA) {
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(C::REG_MISC));
-    if (warp == 22) {
+    if (warp == C::W_TMA) {
       // ============================================================ TMA producer (a2, a3)
       const uint64_t keep = policy_evict_last();   // K/V: re-read by the other q-tile pairs
       const uint64_t once = policy_evict_first();  // Q: read once
@@ -319,11 +344,11 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
           }
         }
       }
-    } else if (warp == 20 || warp == 21) {
+    } else if (warp == C::W_MMA || warp == C::W_MMA + 1) {
       // ============================================================ MMA issuers (a4, a8)
-      // Warp 20 issues tile 0's MMAs, warp 21 tile 1's, so each tile's chain (QK -> softmax ->
+      // Warp W_MMA issues tile 0's MMAs, warp W_MMA + 1 tile 1's, so each tile's chain (QK -> softmax ->
       // PV) depends only on its own softmax warps.  Both warps release every K/V entry (count 2).
-      const int t = warp - 20;
+      const int t = warp - C::W_MMA;
       constexpr uint32_t IDESC_QK = idesc_f16(BF16, 128, 128, false, false);  // Q, K: K-major
       constexpr uint32_t IDESC_PV = idesc_f16(BF16, 128, D, false, true);     // P: K-major (TMEM), V: MN-major
       // descriptors differ only in the start-address field: one base, plus (offset >> 4)
@@ -333,8 +358,8 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
       const uint32_t tO = tmem + 256 + t * D;
       const uint32_t tP = tmem + (C::SEP_P ? C::TMEM_P + 64 * t : 128 * t);
       const uint32_t S_FULL = BAR(C::B_S_FULL + t), P_FULL = BAR(C::B_P_FULL + t);
-      const uint32_t O_READY = BAR(C::B_O_READY + t), PV_DONE = BAR(C::B_PV_DONE + t);
-      const uint32_t S_FREE = BAR(C::B_S_FREE + t);
+      const uint32_t O_FULL = BAR(C::B_O_FULL + t), O_EMPTY = BAR(C::B_O_EMPTY + t);
+      const uint32_t PV_DONE = BAR(C::B_PV_DONE + t), S_FREE = BAR(C::B_S_FREE + t);
       uint32_t qc = 0, pc = 0, oc = 0, qkc = 0;
       auto ring_wait = [&](uint32_t k) {
         mbar_wait_at(KV_FULL(k % C::NS), (k / C::NS) & 1, 3, k, 0);
@@ -416,19 +441,23 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
         if (cu.j + 1 == n) umma_commit_elect(Q_EMPTY(t, cu.qs));  // last QK of the tile: Q slot reusable
         umma_commit_elect(KV_EMPTY(kidx % C::NS));
       };
-      // O_t (+)= P_t V_{t,j} once the softmax wrote P_t and the correction group rescaled O_t
+      // O_t (+)= P_t V_{t,j} once the softmax wrote P_t (and rescaled its rows of O_t if needed);
+      // the first PV of an item overwrites O_t, so it also waits until the epilogue has read O_t
       auto pv_entry = [&](Cursor& cu, uint32_t vidx) {
         const uint32_t sV = ring_wait(vidx);
+        if (cu.j == 0) {
+          mbar_wait_at(O_EMPTY, (oc & 1) ^ 1, 7, oc, cu.idx);
+          ++oc;
+        }
         mbar_wait_at(P_FULL, pc & 1, 6, pc, cu.idx);
         ++pc;
         TRACE_EV(EV_MMA_P, t * 64 + cu.j);
-        mbar_wait_at(O_READY, oc & 1, 7, oc, cu.idx);
-        ++oc;
         tc_fence_after();
 #pragma unroll
         for (int kk = 0; kk < 8; ++kk)
           umma_ts_elect(tO, tP + kk * 8, vdesc0 + ((sV - sbase + kk * 2048) >> 4), IDESC_PV, (cu.j > 0 || kk > 0));
-        umma_commit_elect(PV_DONE);
+        if (C::SEP_P) umma_commit_elect(PV_DONE);   // P_t may be overwritten
+        if (cu.j + 1 == cu.w.n(t)) umma_commit_elect(O_FULL);  // O_t final: epilogue
         TRACE_EV(EV_MMA_PV, t * 64 + cu.j);
         umma_commit_elect(KV_EMPTY(vidx % C::NS));
       };
@@ -477,53 +506,48 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
         started = true;
       }
     }
-  } else if (warp < 16) {
+  } else if (warp < C::W_CORR) {
     asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(C::REG_SOFTMAX));
     // ============================================================== softmax (a5, a6)
-    const int t = warp >> 3, h = (warp >> 2) & 1, quad = warp & 3;
+    const int t = warp >> 2, quad = warp & 3;
     const int row = quad * 32 + lane;
     const uint32_t lane_off = static_cast<uint32_t>(quad * 32) << 16;
-    const uint32_t tS = tmem + lane_off + 128 * t + 64 * h;  // this warp's 64 S columns
-    const uint32_t tP = tmem + lane_off + (C::SEP_P ? C::TMEM_P + 64 * t : 128 * t) + 32 * h;
+    const uint32_t tS = tmem + lane_off + 128 * t;  // this row's 128 S columns
+    const uint32_t tP = tmem + lane_off + (C::SEP_P ? C::TMEM_P + 64 * t : 128 * t);
     const uint32_t S_FULL = BAR(C::B_S_FULL + t), P_FULL = BAR(C::B_P_FULL + t);
     const uint32_t PV_DONE = BAR(C::B_PV_DONE + t), S_FREE = BAR(C::B_S_FREE + t);
-    const uint32_t ST_FULL = BAR(C::B_ST_FULL + t), ST_EMPTY = BAR(C::B_ST_EMPTY + t);
     const uint32_t L_FULL = BAR(C::B_L_FULL + t), L_EMPTY = BAR(C::B_L_EMPTY + t);
-    const uint32_t pair_bar = 4 + 4 * t + quad;  // named barrier shared with the other column half
-    // The tiles take turns for the exp phase (named barriers 2, 3; 256 threads per tile): one
-    // tile's two warps per SMSP saturate MUFU while the other tile loads S and reduces its max.
-    const uint32_t my_turn = 2 + t, other_turn = 3 - t;
-    if (C::TURNS && t == 1) named_bar_arrive(2, 512);  // tile 0 goes first
+    const uint32_t tO = tmem + lane_off + 256 + t * D;  // this row of O_t
+    const uint32_t my_turn = 2 + 2 * quad + t, other_turn = 3 + 2 * quad - t;  // 64-thread barriers
+    if (C::TURNS && t == 1) named_bar_arrive(2 + 2 * quad, 64);  // tile 0 goes first
     const float c = p.scale_log2;
     const int off = p.seq_kv - p.seq_q;
-    // g = real steps this warp has done so far: the phase count of S_FULL, ST_EMPTY, PV_DONE and
-    // the max-exchange slot parity are all g (one counter keeps the 96-register budget)
+    // g = real steps this thread has done so far: the phase count of S_FULL and PV_DONE
     uint32_t g = 0, lc = 0;
     for (int idx = first; idx < p.num_items; idx += stride) {
       const WorkItem w = decode_item<PAIRX>(p, idx);
-      const int N = max(w.n0, w.n1);
       const int n = w.n(t);
+      const int N = C::TURNS ? max(w.n0, w.n1) : n;
+      TRACE_EV(EV_ITEM, 1);
       const int qi = w.row0(t) + row;
       int lim = w.kv(t);  // keys j < lim are visible to this row
       if (p.mask_kind == MASK_CAUSAL) lim = min(lim, qi + off + 1);
-      lim -= 64 * h;         // ... in this warp's column coordinates
       float m_ref = -INFINITY;  // max used as the exp2 reference (lags the true max by < 2^8)
-      float l = 0.f;            // this half's share of the row sum
+      float l = 0.f;            // row sum relative to m_ref
       for (int j = 0; j < N; ++j) {
         if (j >= n) {  // no KV tile j for this tile: pass the turn on
-          if (C::TURNS) {
-            named_bar_sync(my_turn, 512);
-            named_bar_arrive(other_turn, 512);
-          }
+          named_bar_sync(my_turn, 64);
+          named_bar_arrive(other_turn, 64);
           continue;
         }
         TRACE_EV(EV_S_WAIT, j);
         mbar_wait_at(S_FULL, g & 1, 8, g, idx);
         TRACE_EV(EV_S_READY, j);
         tc_fence_after();
-        uint32_t s[64];
-        tmem_ld_32x32b_x32(tS, *reinterpret_cast<uint32_t(*)[32]>(&s[0]));
-        tmem_ld_32x32b_x32(tS + 32, *reinterpret_cast<uint32_t(*)[32]>(&s[32]));
+        uint32_t s[128];
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          tmem_ld_32x32b_x32(tS + 32 * q, *reinterpret_cast<uint32_t(*)[32]>(&s[32 * q]));
         tmem_wait_ld();
         reg_fence(s);
         if (C::SEP_P) {  // S_t read: the tensor core may overwrite it with S_{t,j+1}
@@ -531,24 +555,20 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
           mbar_arrive(S_FREE);
         }
         const int rem = lim - j * 128;
-        if (rem < 64) {  // boundary tile for this row (a5)
+        if (rem < 128) {  // boundary tile for this row (a5)
 #pragma unroll
-          for (int k = 0; k < 64; ++k)
+          for (int k = 0; k < 128; ++k)
             if (k >= rem) s[k] = __float_as_uint(-INFINITY);
         }
         float mx0 = m_ref, mx1 = -INFINITY, mx2 = -INFINITY, mx3 = -INFINITY;
 #pragma unroll
-        for (int k = 0; k < 64; k += 8) {
+        for (int k = 0; k < 128; k += 8) {
           mx0 = fmax3(mx0, __uint_as_float(s[k]), __uint_as_float(s[k + 1]));
           mx1 = fmax3(mx1, __uint_as_float(s[k + 2]), __uint_as_float(s[k + 3]));
           mx2 = fmax3(mx2, __uint_as_float(s[k + 4]), __uint_as_float(s[k + 5]));
           mx3 = fmax3(mx3, __uint_as_float(s[k + 6]), __uint_as_float(s[k + 7]));
         }
-        // combine with the other column half of this row
-        float* slot = s_pmax + ((g & 1) * 4 + 2 * t) * 128;  // [parity][t][half][row]
-        slot[h * 128 + row] = fmaxf(fmaxf(mx0, mx1), fmaxf(mx2, mx3));
-        named_bar_sync(pair_bar, 64);
-        const float m_new = fmaxf(slot[row], slot[128 + row]);
+        const float m_new = fmaxf(fmaxf(mx0, mx1), fmaxf(mx2, mx3));
         TRACE_EV(EV_MAX_DONE, j);
         // Lazy rescale: keep the old reference while the max grows by < 8 in the log2 domain (the
         // p's then stay <= 2^8, exact in fp32 and in fp16/bf16 range); l and O share the reference.
@@ -557,14 +577,11 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
           alpha = (m_ref == -INFINITY) ? 0.f : ex2((m_ref - m_new) * c);
           m_ref = m_new;
         }
-        if (h == 0) {  // hand alpha to the correction group (it rescales O_t before PV_{t,j})
-          mbar_wait_at(ST_EMPTY, (g & 1) ^ 1, 9, g, idx);
-          s_alpha[t * 128 + row] = (j == 0) ? 1.f : alpha;
-          mbar_arrive(ST_FULL);
-        }
         const float mc = (m_ref == -INFINITY) ? 0.f : m_ref * c;
-        TRACE_EV(EV_COR_ST, j);  // after the stats hand-off
-        if (C::SEP_P && g > 0) {  // P_t buffer still read by PV_{t,j-1}?
+        TRACE_EV(EV_COR_ST, j);
+        // PV_{t,j-1} must be done before P_t is overwritten (separate P) and before O_t is rescaled.
+        // (With P over S, S_{t,j} was computed after PV_{t,j-1}: S_FULL already implies it.)
+        if (C::SEP_P && g > 0) {
           mbar_wait_at(PV_DONE, (g - 1) & 1, 10, g, idx);
           tc_fence_after();
         }
@@ -572,19 +589,23 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
         ++g;
         // P = exp2(c*s - c*m_ref) (a6), rounded to the I/O type, stored to TMEM for the PV MMA
         float2 acc0 = make_float2(0.f, 0.f), acc1 = make_float2(0.f, 0.f);
-        if (C::TURNS) named_bar_sync(my_turn, 512);
-#if FMHA_TRACE
-        if (*reinterpret_cast<volatile float*>(s_lsum) == 12345.f) m_ref += 1.f;  // force the deferred barrier block here
-#endif
-        TRACE_EV(EV_XCHG, j);
+        float mcv = mc;
 #pragma unroll
-        for (int hh = 0; hh < 2; ++hh) {
+        for (int hh = 0; hh < 4; ++hh) {
+          if (hh == C::PRE_CHUNKS) {
+            // The exponentials are register-only work that ptxas would hoist above the barrier:
+            // round-trip their input through shared memory, which bar.sync does order.
+            const uint32_t slot = sbase + C::OFF_MC + (t * 128 + row) * 4;
+            asm volatile("st.shared.f32 [%0], %1;" ::"r"(slot), "f"(mc) : "memory");
+            named_bar_sync(my_turn, 64);
+            asm volatile("ld.volatile.shared.f32 %0, [%1];" : "=f"(mcv) : "r"(slot) : "memory");
+          }
           uint32_t pk[16];
 #pragma unroll
           for (int u = 0; u < 16; u += 2) {
             const int k = 32 * hh + 2 * u;
-            float2 x0 = ffma2(make_float2(__uint_as_float(s[k]), __uint_as_float(s[k + 1])), c, -mc);
-            float2 x1 = ffma2(make_float2(__uint_as_float(s[k + 2]), __uint_as_float(s[k + 3])), c, -mc);
+            float2 x0 = ffma2(make_float2(__uint_as_float(s[k]), __uint_as_float(s[k + 1])), c, -mcv);
+            float2 x1 = ffma2(make_float2(__uint_as_float(s[k + 2]), __uint_as_float(s[k + 3])), c, -mcv);
 #ifdef FMHA_FAKE_EXP  // timing experiment only: exponentials replaced by a trivial op (wrong results)
             if (true) {
               x0 = fadd2(x0, make_float2(1.f, 1.f));
@@ -614,81 +635,62 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
           }
           tmem_st_32x32b_x16(tP + 16 * hh, pk);
         }
-        if (C::TURNS) named_bar_arrive(other_turn, 512);
+        if (C::TURNS) named_bar_arrive(other_turn, 64);
         TRACE_EV(EV_EXP_DONE, j);
+        // lazy rescale of this warp's rows of O_t (a7), after the exponentials so that S is no
+        // longer live; at j = 0 PV overwrites O_t instead
+        if (j > 0 && __any_sync(0xffffffffu, alpha != 1.f)) {
+#pragma unroll 1
+          for (int q = 0; q < D / 32; ++q) {
+            uint32_t o[32];
+            tmem_ld_32x32b_x32(tO + 32 * q, o);
+            tmem_wait_ld();
+            reg_fence(o);
+#pragma unroll
+            for (int k = 0; k < 32; ++k) o[k] = __float_as_uint(__uint_as_float(o[k]) * alpha);
+            tmem_st_32x32b_x32(tO + 32 * q, o);
+          }
+        }
         tmem_wait_st();
         TRACE_EV(EV_EPI, j);  // P stores landed
         tc_fence_before();
         mbar_arrive(P_FULL);
         l = l * alpha + ((acc0.x + acc0.y) + (acc1.x + acc1.y));
       }
-      if (t == 0 || w.has1) {
-        // the correction group has read the previous item's sums (without this wait the softmax can
-        // run two items ahead and L_FULL's phase parity would alias)
-#ifndef FMHA_NO_LEMPTY
-        mbar_wait_at(L_EMPTY, (lc & 1) ^ 1, 15, lc, idx);
-#endif
-        ++lc;
-        s_lsum[(2 * t + h) * 128 + row] = l;
-        mbar_arrive(L_FULL);
-      }
+      if (t == 1 && !w.has1) continue;
+      // the epilogue has read the previous item's sums (without this wait the softmax can run two
+      // items ahead and L_FULL's phase parity would alias)
+      TRACE_EV(EV_ITEM, 2);
+      mbar_wait_at(L_EMPTY, (lc & 1) ^ 1, 15, lc, idx);
+      TRACE_EV(EV_ITEM, 3);
+      ++lc;
+      s_lsum[t * 128 + row] = l;
+      mbar_arrive(L_FULL);
     }
-    if (C::TURNS && t == 0) named_bar_sync(2, 512);  // consume tile 1's last hand-over
+    if (C::TURNS && t == 0) named_bar_sync(2 + 2 * quad, 64);  // consume tile 1's last hand-over
   } else {
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(C::REG_CORR));
-    // ================================================================ correction group (a7, a9)
+    // ================================================================ epilogue (a9)
     const int quad = warp & 3;
     const int row = quad * 32 + lane;
     const uint32_t lane_off = static_cast<uint32_t>(quad * 32) << 16;
-    uint32_t stc[2] = {0, 0}, pvc[2] = {0, 0}, lc[2] = {0, 0};
+    uint32_t ofc[2] = {0, 0}, lc[2] = {0, 0};
     for (int idx = first; idx < p.num_items; idx += stride) {
       const WorkItem w = decode_item<PAIRX>(p, idx);
-      const int N = max(w.n0, w.n1);
-      for (int j = 0; j < N; ++j) {
-#pragma unroll
-        for (int t = 0; t < 2; ++t) {
-          if (j >= w.n(t)) continue;
-          mbar_wait_at(BAR(C::B_ST_FULL + t), stc[t] & 1, 11, stc[t], idx);
-          TRACE_EV(EV_COR_ST, t * 64 + j);
-          const float alpha = s_alpha[t * 128 + row];
-          mbar_arrive(BAR(C::B_ST_EMPTY + t));
-          ++stc[t];
-          if (j > 0) {
-            mbar_wait_at(BAR(C::B_PV_DONE + t), pvc[t] & 1, 12, pvc[t], idx);  // PV_{t,j-1} has landed in O_t
-            ++pvc[t];
-            if (__any_sync(0xffffffffu, alpha != 1.f)) {
-              tc_fence_after();
-              const uint32_t tO = tmem + lane_off + 256 + t * D;
-#pragma unroll 1
-              for (int q = 0; q < D / 32; ++q) {
-                uint32_t o[32];
-                tmem_ld_32x32b_x32(tO + 32 * q, o);
-                tmem_wait_ld();
-                reg_fence(o);
-#pragma unroll
-                for (int k = 0; k < 32; ++k) o[k] = __float_as_uint(__uint_as_float(o[k]) * alpha);
-                tmem_st_32x32b_x32(tO + 32 * q, o);
-              }
-              tmem_wait_st();
-            }
-          }
-          tc_fence_before();
-          mbar_arrive(BAR(C::B_O_READY + t));
-          TRACE_EV(EV_COR_ORDY, t * 64 + j);
-        }
-      }
       // ------------------------------------------------------------ epilogue per tile (a9)
 #pragma unroll 1
       for (int t = 0; t < 2; ++t) {
         if (t == 1 && !w.has1) continue;
         mbar_wait_at(BAR(C::B_L_FULL + t), lc[t] & 1, 13, lc[t], idx);
+        TRACE_EV(EV_EPI, 100 + t);
         ++lc[t];
-        const float l = s_lsum[(2 * t) * 128 + row] + s_lsum[(2 * t + 1) * 128 + row];
+        const float l = s_lsum[t * 128 + row];
         mbar_arrive(BAR(C::B_L_EMPTY + t));
         const int n = w.n(t);
         if (n > 0) {
-          mbar_wait_at(BAR(C::B_PV_DONE + t), pvc[t] & 1, 14, pvc[t], idx);  // last PV of this tile
-          ++pvc[t];
+          mbar_wait_at(BAR(C::B_O_FULL + t), ofc[t] & 1, 14, ofc[t], idx);  // last PV of this tile
+          TRACE_EV(EV_EPI, 110 + t);
+          ++ofc[t];
           tc_fence_after();
         }
         const float inv_l = (l > 0.f) ? 1.f / l : 0.f;  // fully masked row -> 0 (R4)
@@ -719,6 +721,10 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
                          pack2<BF16>(__uint_as_float(o[8 * u + 6]) * inv_l, __uint_as_float(o[8 * u + 7]) * inv_l));
           }
         }
+        if (n > 0) {  // O_t read: the next item's first PV may overwrite it
+          tc_fence_before();
+          mbar_arrive(BAR(C::B_O_EMPTY + t));
+        }
         fence_proxy_async_smem();
         named_bar_sync(1, 128);
         if (row == 0) {
@@ -727,6 +733,7 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
             tma_store_3d(&p.tmO, stg + c2 * C::CHUNK, c2 * 64, w.row0(t), w.bh(t));
           tma_store_commit();
         }
+        TRACE_EV(EV_EPI, 120 + t);
       }
     }
     if (row == 0) tma_store_wait0();
@@ -734,7 +741,7 @@ __global__ void __launch_bounds__(768, 1) fmha_fwd_sm100(const __grid_constant__
 
   tc_fence_before();
   __syncthreads();
-  if (warp == 20) {
+  if (warp == C::W_MMA) {
     tc_fence_after();
     tmem_dealloc(tmem, C::TMEM_COLS);
   }
