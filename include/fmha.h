@@ -80,6 +80,25 @@ FMHA_API int fmha_fwd(const void* Q, const void* K, const void* V, void* O, cons
 FMHA_API int fmha_fwd_bf16(const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask, int batch,
                   int heads, int seq_q, int seq_kv, int head_dim, float scale, fmha_stream_t stream);
 
+/* Variable-length packed input: the MLPerf BERT inference format the paper's FMHA serves
+ * (SURVEY.md §8(f) f2).  A batch of num_seqs sequences is stored back to back:
+ *   QKV        DEVICE [total_tokens, 3, heads, head_dim]  (Q, K, V of token t, e.g. the output of one
+ *              fused QKV projection GEMM: row t = [q_h0 .. q_hH-1 | k_h0 .. | v_h0 ..])
+ *   O          DEVICE [total_tokens, heads, head_dim]
+ *   cu_seqlens DEVICE int32 [num_seqs + 1]: sequence s is tokens [cu_seqlens[s], cu_seqlens[s+1]);
+ *              cu_seqlens[0] = 0, nondecreasing, cu_seqlens[num_seqs] = total_tokens (not checked:
+ *              out-of-range values make the kernel read or write outside the buffers).
+ *   max_seqlen HOST int >= every sequence length (sizes the work decomposition; larger is legal).
+ * For every sequence s, head h and token i of s:
+ *     O[i,h,:] = sum_{j in s} softmax_j( scale * <Q[i,h,:], K[j,h,:]> + mask ) * V[j,h,:]
+ * with mask = none (causal = 0) or j <= i (causal = 1, positions within the sequence).  Tokens of
+ * different sequences never attend to each other; zero-length sequences are allowed.
+ * dtype: 0 = fp16, 1 = bf16.  Precision, ownership, errors: as fmha_fwd.  QKV and O 16-byte
+ * aligned, cu_seqlens 4-byte aligned. */
+FMHA_API int fmha_fwd_varlen(const void* QKV, void* O, const int32_t* cu_seqlens, int num_seqs, int max_seqlen,
+                             int total_tokens, int heads, int head_dim, float scale, int causal, int dtype,
+                             fmha_stream_t stream);
+
 /* End-to-end variant: Q/K/V/O and kv_len are HOST buffers (pinned memory for asynchronous copies).
  * Copies Q, K, V (and kv_len) host->device into `workspace`, runs the same kernel, copies O
  * device->host, all enqueued on `stream` (no synchronisation: the caller syncs before reading O).

@@ -17,7 +17,8 @@ recorded in DESIGN.md §3 where the paper is silent.
 
 Modules
 -------
-fmha   numpy fp64, unfused GEMM -> softmax -> GEMM per (batch, head)   [pinned]
+fmha   numpy fp64, unfused GEMM -> softmax -> GEMM per (batch, head);
+       the same per (sequence, head) of a packed variable-length batch   [pinned]
 brute  pure-Python scalar loops with math.fsum, tiny shapes only        [pinned]
 gemm   numpy fp64 act(A @ W^T + b)                                      [pinned]
 
@@ -27,13 +28,14 @@ torch's fp64 CPU ``scaled_dot_product_attention``.  There is no "parity
 unpinned" function in this package.
 """
 
-from .fmha import attention_fp64, attention_rows_fp64, softmax_probs_fp64, fmha_flops
+from .fmha import attention_fp64, attention_rows_fp64, attention_varlen_fp64, softmax_probs_fp64, fmha_flops
 from .brute import attention_brute
 from .gemm import gemm_bias_act_fp64, gelu_erf, gelu_tanh, relu
 
 __all__ = [
     "attention_fp64",
     "attention_rows_fp64",
+    "attention_varlen_fp64",
     "softmax_probs_fp64",
     "fmha_flops",
     "attention_brute",

@@ -125,6 +125,29 @@ def attention_rows_fp64(q, k, v, scale: float, units, kv_len=None,
     return np.stack(res) if res else np.zeros((0, v.shape[-1]))
 
 
+def attention_varlen_fp64(qkv, cu_seqlens, scale: float, causal: bool = False) -> np.ndarray:
+    """Variable-length packed attention (MLPerf BERT inference layout; R17).
+
+    ``qkv`` [T, 3, H, D] holds Q, K, V of every token; sequence s is tokens
+    cu_seqlens[s] .. cu_seqlens[s+1]-1.  Each sequence is an independent problem:
+    for every head h, steps 1-7 above on Q = qkv[a:b, 0, h], K = qkv[a:b, 1, h],
+    V = qkv[a:b, 2, h] (causal: key j visible to query i iff j <= i, positions
+    within the sequence).  Returns float64 O [T, H, D]."""
+    x = _as_f64(qkv)
+    t_, three, h_, d = x.shape
+    assert three == 3
+    cu = [int(c) for c in cu_seqlens]
+    out = np.zeros((t_, h_, d), dtype=np.float64)
+    for s in range(len(cu) - 1):
+        a, b = cu[s], cu[s + 1]
+        if b <= a:
+            continue
+        for h in range(h_):
+            p = softmax_probs_fp64(x[a:b, 0, h], x[a:b, 1, h], scale, None, causal)
+            out[a:b, h] = p @ x[a:b, 2, h]                   # step 7 (GEMM #2)
+    return out
+
+
 def fmha_flops(batch: int, heads: int, sq: int, skv: int, d: int, kv_len=None,
                causal: bool = False) -> float:
     """Algorithmic flops: 4*D per visible (i,j) pair (2*D for Q.K, 2*D for P.V).

@@ -6,6 +6,7 @@ kernels behind the ABI.  There is no CPU or library fallback: without the built 
 sm_100 device these functions raise.
 
     fmha_fwd(q, k, v, kv_len=None, causal=False, scale=None, out=None) -> O
+    fmha_fwd_varlen(qkv, cu_seqlens, max_seqlen, causal=False, scale=None, out=None) -> O
     fmha_fwd_from_host(q, k, v, ..., workspace) -> O  (host tensors; copies inside the call)
     gemm_bias_act(a, w, bias=None, act="none", out=None) -> C
 """
@@ -20,7 +21,7 @@ import torch
 from . import _lib
 from ._lib import FmhaError, FmhaMask
 
-__all__ = ["fmha_fwd", "fmha_fwd_from_host", "gemm_bias_act", "workspace_bytes", "FmhaError",
+__all__ = ["fmha_fwd", "fmha_fwd_varlen", "fmha_fwd_from_host", "gemm_bias_act", "workspace_bytes", "FmhaError",
            "MASK_NONE", "MASK_KEY_PADDING", "MASK_CAUSAL", "ACTS", "version"]
 
 MASK_NONE, MASK_KEY_PADDING, MASK_CAUSAL = 0, 1, 2
@@ -73,6 +74,34 @@ def fmha_fwd(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, kv_len: torch.Te
     st = fn(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), ctypes.byref(m), b, h, sq, skv, d,
             scale, _stream_ptr(q.device))
     _lib.check(st, "fmha_fwd")
+    return out
+
+
+def fmha_fwd_varlen(qkv: torch.Tensor, cu_seqlens: torch.Tensor, max_seqlen: int, causal: bool = False,
+                    scale: float | None = None, out: torch.Tensor | None = None) -> torch.Tensor:
+    """Packed variable-length FMHA (MLPerf BERT layout): qkv [T,3,H,D] contiguous CUDA fp16/bf16,
+    cu_seqlens CUDA int32 [num_seqs+1] (sequence s = tokens cu[s]..cu[s+1]-1), max_seqlen a host
+    int >= every length.  Returns O [T,H,D].  Calls ``fmha_fwd_varlen`` of the C ABI."""
+    lib = _lib.load()
+    if qkv.dtype not in (torch.float16, torch.bfloat16):
+        raise TypeError("qkv must be fp16 or bf16")
+    if not qkv.is_cuda or not cu_seqlens.is_cuda:
+        raise TypeError("qkv and cu_seqlens must be CUDA tensors (no CPU fallback)")
+    if qkv.dim() != 4 or qkv.shape[1] != 3 or not qkv.is_contiguous():
+        raise ValueError("qkv must be contiguous [T,3,H,D]")
+    if cu_seqlens.dtype != torch.int32 or cu_seqlens.dim() != 1 or cu_seqlens.numel() < 1:
+        raise ValueError("cu_seqlens must be a CUDA int32 tensor [num_seqs+1]")
+    t, _, h, d = qkv.shape
+    cu_seqlens = cu_seqlens.contiguous()
+    if out is None:
+        out = torch.empty((t, h, d), dtype=qkv.dtype, device=qkv.device)
+    elif out.shape != (t, h, d) or out.dtype != qkv.dtype or not out.is_contiguous():
+        raise ValueError("out must be contiguous [T,H,D] of qkv's dtype")
+    scale = 1.0 / math.sqrt(d) if scale is None else float(scale)
+    st = lib.fmha_fwd_varlen(qkv.data_ptr(), out.data_ptr(), cu_seqlens.data_ptr(), cu_seqlens.numel() - 1,
+                             int(max_seqlen), t, h, d, scale, int(bool(causal)),
+                             0 if qkv.dtype == torch.float16 else 1, _stream_ptr(qkv.device))
+    _lib.check(st, "fmha_fwd_varlen")
     return out
 
 

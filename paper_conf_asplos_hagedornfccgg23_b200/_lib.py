@@ -27,6 +27,7 @@ STATUS_NAMES = {
 EXPORTED_SYMBOLS = (
     "fmha_fwd",
     "fmha_fwd_bf16",
+    "fmha_fwd_varlen",
     "fmha_workspace_bytes",
     "fmha_fwd_from_host",
     "gemm_bias_act",
@@ -66,6 +67,9 @@ def load() -> ctypes.CDLL:
         f = getattr(lib, name)
         f.argtypes = [vp, vp, vp, vp, mp, i32, i32, i32, i32, i32, f32, vp]
         f.restype = i32
+    if hasattr(lib, "fmha_fwd_varlen"):  # absent only in old tuning builds (B200FMHA_LIB A/B runs)
+        lib.fmha_fwd_varlen.argtypes = [vp, vp, vp, i32, i32, i32, i32, i32, f32, i32, i32, vp]
+        lib.fmha_fwd_varlen.restype = i32
     lib.fmha_workspace_bytes.argtypes = [i32] * 5
     lib.fmha_workspace_bytes.restype = sz
     lib.fmha_fwd_from_host.argtypes = [i32, vp, vp, vp, vp, mp, vp, sz, i32, i32, i32, i32, i32, f32, vp]

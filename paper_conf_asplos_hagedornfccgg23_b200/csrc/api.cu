@@ -94,19 +94,49 @@ int make_map_3d(CUtensorMap* m, const void* base, bool bf16, uint64_t cols, uint
   return FMHA_OK;
 }
 
+// 3-D tile map over token-major [T, (3,) H, D] data (varlen packed mode): dims {D, H, T}, token
+// stride `tok_stride` elements, box {64, 1, 128}: one head's 128-token x 64-d block (the same
+// 128 rows x 128 B SWIZZLE_128B smem tile as the dense map).  Tokens >= T read as zero.
+int make_map_thd(CUtensorMap* m, const void* base, bool bf16, uint64_t d, uint64_t heads, uint64_t tokens,
+                 uint64_t tok_stride) {
+  EncodeTiledFn enc = get_encode_fn();
+  if (!enc) {
+    snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "cuTensorMapEncodeTiled entry point unavailable");
+    return FMHA_ERR_CUDA;
+  }
+  cuuint64_t dims[3] = {d, heads, tokens};
+  cuuint64_t strides[2] = {d * 2, tok_stride * 2};
+  cuuint32_t box[3] = {64, 1, 128};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = enc(m, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 3,
+                   const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) {
+    snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "cuTensorMapEncodeTiled failed (%d)", int(r));
+    return FMHA_ERR_CUDA;
+  }
+  return FMHA_OK;
+}
+
 bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
 template <int D, bool BF16>
 int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) {
   using C = b200::FmhaCfg<D>;
-  auto kern = prm.pair_mode ? b200::fmha_fwd_sm100<D, BF16, true> : b200::fmha_fwd_sm100<D, BF16, false>;
-  static bool attr_done[64][2];
+  const int mode = prm.cu_seqlens ? (prm.sched ? b200::MODE_VARLEN_SCHED : b200::MODE_VARLEN)
+                                  : (prm.pair_mode ? b200::MODE_PAIRX : b200::MODE_DENSE);
+  void (*kern)(b200::FmhaParams) = mode == b200::MODE_DENSE    ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_DENSE>
+                                   : mode == b200::MODE_PAIRX  ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_PAIRX>
+                                   : mode == b200::MODE_VARLEN ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_VARLEN>
+                                                               : b200::fmha_fwd_sm100<D, BF16, b200::MODE_VARLEN_SCHED>;
+  static bool attr_done[64][4];
   int dev = 0;
   cudaGetDevice(&dev);
-  if (dev >= 64 || !attr_done[dev][prm.pair_mode]) {
+  if (dev >= 64 || !attr_done[dev][mode]) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_ALLOC);
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(fmha)");
-    if (dev < 64) attr_done[dev][prm.pair_mode] = true;
+    if (dev < 64) attr_done[dev][mode] = true;
   }
   // persistent: one CTA per SM (or fewer when there is less work)
   dim3 grid(static_cast<unsigned>(std::min(prm.num_items, sm_count)), 1, 1);
@@ -145,6 +175,7 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   if ((st = make_map_3d(&prm.tmV, V, bf16, head_dim, seq_kv, units, 128)) != FMHA_OK) return st;
   if ((st = make_map_3d(&prm.tmO, O, bf16, head_dim, seq_q, units, 128)) != FMHA_OK) return st;
   prm.kv_len = (kind == FMHA_MASK_KEY_PADDING) ? mask->kv_len : nullptr;
+  prm.cu_seqlens = nullptr;
   prm.seq_q = seq_q;
   prm.seq_kv = seq_kv;
   prm.heads = heads;
@@ -174,6 +205,59 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
 
 size_t round_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
+int fmha_varlen_common(bool bf16, const void* QKV, void* O, const int32_t* cu_seqlens, int num_seqs, int max_seqlen,
+                       int total_tokens, int heads, int head_dim, float scale, int causal, cudaStream_t stream) {
+  g_last_cuda_error[0] = 0;
+  if (num_seqs < 0 || max_seqlen < 0 || total_tokens < 0 || heads < 0) return FMHA_ERR_INVALID_ARG;
+  if (!std::isfinite(scale)) return FMHA_ERR_INVALID_ARG;
+  if (head_dim != 64 && head_dim != 128) return FMHA_ERR_UNSUPPORTED;
+  if (scale < 0.f || (causal != 0 && causal != 1)) return FMHA_ERR_UNSUPPORTED;
+  const long long units = static_cast<long long>(num_seqs) * heads;
+  if (units == 0 || max_seqlen == 0 || total_tokens == 0) return FMHA_OK;
+  if (!QKV || !O || !cu_seqlens) return FMHA_ERR_INVALID_ARG;
+  if (!aligned16(QKV) || !aligned16(O) || (reinterpret_cast<uintptr_t>(cu_seqlens) & 3u)) return FMHA_ERR_MISALIGNED;
+  if (units > 2147483647LL || static_cast<long long>(total_tokens) * 3 * heads * head_dim > (1LL << 40))
+    return FMHA_ERR_INVALID_ARG;
+  int sm_count = 0;
+  int st = check_device(&sm_count);
+  if (st != FMHA_OK) return st;
+
+  b200::FmhaParams prm;
+  memset(&prm, 0, sizeof(prm));
+  const uint64_t hd = static_cast<uint64_t>(heads) * head_dim;
+  const uint8_t* base = static_cast<const uint8_t*>(QKV);
+  if ((st = make_map_thd(&prm.tmQ, base, bf16, head_dim, heads, total_tokens, 3 * hd)) != FMHA_OK) return st;
+  if ((st = make_map_thd(&prm.tmK, base + 2 * hd, bf16, head_dim, heads, total_tokens, 3 * hd)) != FMHA_OK) return st;
+  if ((st = make_map_thd(&prm.tmV, base + 4 * hd, bf16, head_dim, heads, total_tokens, 3 * hd)) != FMHA_OK) return st;
+  if ((st = make_map_thd(&prm.tmO, O, bf16, head_dim, heads, total_tokens, hd)) != FMHA_OK) return st;
+  prm.kv_len = nullptr;
+  prm.cu_seqlens = cu_seqlens;
+  prm.o_ptr = static_cast<uint8_t*>(O);
+  prm.o_row_elems = static_cast<int>(hd);
+  prm.seq_q = prm.seq_kv = max_seqlen;  // self-attention within each sequence: causal offset 0
+  prm.heads = heads;
+  prm.num_q_tiles = (max_seqlen + 127) / 128;
+  prm.num_units = static_cast<int>(units);
+  prm.mask_kind = causal ? FMHA_MASK_CAUSAL : FMHA_MASK_NONE;
+  prm.scale_log2 = std::max(scale * 1.4426950408889634f, 1e-30f);
+  prm.pair_mode = 0;  // both tiles of an item belong to one (sequence, head)
+  prm.num_seqs = num_seqs;
+  prm.max_level = prm.num_q_tiles;
+  // non-causal items cost ceil(len/128) KV steps: visit them in decreasing-cost order, dealt in snake
+  // order over the CTAs (see fmha_kernel.cuh).  Causal keeps the static longest-pair-first order.
+  prm.sched = (!causal && num_seqs <= b200::SCHED_MAX_SEQS && prm.max_level <= b200::SCHED_MAX_LEVELS) ? 1 : 0;
+  const long long items = units * ((prm.num_q_tiles + 1) / 2);
+  if (items > 2147483647LL) return FMHA_ERR_UNSUPPORTED;
+  prm.num_items = static_cast<int>(items);
+  prm.div_units.init(static_cast<uint32_t>(std::max(prm.num_units, 1)));
+  prm.div_pairs.init(static_cast<uint32_t>(std::max((prm.num_q_tiles + 1) / 2, 1)));
+  prm.div_qtiles.init(static_cast<uint32_t>(std::max(prm.num_q_tiles, 1)));
+  prm.div_heads.init(static_cast<uint32_t>(std::max(heads, 1)));
+  if (head_dim == 64)
+    return bf16 ? launch_fmha<64, true>(prm, sm_count, stream) : launch_fmha<64, false>(prm, sm_count, stream);
+  return bf16 ? launch_fmha<128, true>(prm, sm_count, stream) : launch_fmha<128, false>(prm, sm_count, stream);
+}
+
 }  // namespace
 
 namespace b200 {
@@ -197,6 +281,14 @@ int fmha_fwd_bf16(const void* Q, const void* K, const void* V, void* O, const fm
                   int heads, int seq_q, int seq_kv, int head_dim, float scale, fmha_stream_t stream) {
   return fmha_common(true, Q, K, V, O, mask, batch, heads, seq_q, seq_kv, head_dim, scale,
                      reinterpret_cast<cudaStream_t>(stream));
+}
+
+int fmha_fwd_varlen(const void* QKV, void* O, const int32_t* cu_seqlens, int num_seqs, int max_seqlen,
+                    int total_tokens, int heads, int head_dim, float scale, int causal, int dtype,
+                    fmha_stream_t stream) {
+  if (dtype != 0 && dtype != 1) return FMHA_ERR_UNSUPPORTED;
+  return fmha_varlen_common(dtype == 1, QKV, O, cu_seqlens, num_seqs, max_seqlen, total_tokens, heads, head_dim,
+                            scale, causal, reinterpret_cast<cudaStream_t>(stream));
 }
 
 size_t fmha_workspace_bytes(int batch, int heads, int seq_q, int seq_kv, int head_dim) {

@@ -31,6 +31,8 @@
 // Because tcgen05.ld 32x32b gives each thread whole TMEM lanes (= query rows), row statistics are
 // thread-local: no warp-shuffle reductions and no cross-warp exchange.
 #pragma once
+#include <type_traits>
+
 #include "sm100.cuh"
 
 // Debug timeline (build with -DFMHA_TRACE=1, see Makefile target `trace`): lane 0 of each warp of
@@ -83,12 +85,32 @@ struct FastDiv {
   __device__ __forceinline__ int mod(int n, int q) const { return n - q * static_cast<int>(d); }
 };
 
+// Cost-sorted schedule (sched mode 1, varlen non-causal): every (sequence, head, q-tile pair) item
+// costs `level` = ceil(len / 128) KV steps.  Items are ordered by decreasing level (sequences of one
+// level by index, then head, then pair) and dealt to the CTAs in snake order (CTA c takes positions
+// c, 2G-1-c, 2G+c, ...), a near-LPT balance.  Each CTA builds the same table in shared memory.
+#ifdef SCHED_SMALL
+constexpr int SCHED_MAX_LEVELS = 4, SCHED_MAX_SEQS = 32;
+#else
+constexpr int SCHED_MAX_LEVELS = 64, SCHED_MAX_SEQS = 1024;
+#endif
+
 struct FmhaParams {
   CUtensorMap tmQ;  // 3-D {D, seq_q, B*H}, box {64, 128, 1}, SWIZZLE_128B
   CUtensorMap tmK;  // 3-D {D, seq_kv, B*H}
   CUtensorMap tmV;
   CUtensorMap tmO;  // same geometry as Q
   const int32_t* kv_len;
+  // Variable-length packed mode (fmha_fwd_varlen): sequence b of the batch is
+  // tokens [cu_seqlens[b], cu_seqlens[b+1]) of QKV [T, 3, H, D] / O [T, H, D]; the tensor maps are
+  // {D, H, T}, so a tile coordinate is (d, h, token) instead of (d, row, b*H + h).  Rows past the
+  // sequence's end are never stored (partial tiles are written row by row, not by TMA).
+  const int32_t* cu_seqlens;  // nullptr: dense [B, H, S, D] mode
+  uint8_t* o_ptr;             // O base (varlen partial-tile stores)
+  int o_row_elems;            // elements between consecutive tokens of O (H * D)
+  int sched;                  // 0: item idx = blockIdx.x + k * gridDim.x;  1: cost-sorted (above)
+  int num_seqs;               // varlen
+  int max_level;              // ceil(max_seqlen / 128) (sched 1: <= SCHED_MAX_LEVELS)
   int seq_q;
   int seq_kv;
   int heads;
@@ -125,15 +147,23 @@ struct FmhaCfg {
   };
   static constexpr int NUM_BARS = B_KV + 2 * NS;
   static constexpr int OFF_TMEMPTR = OFF_BAR + NUM_BARS * 8;
-  static constexpr int SMEM_ALLOC = OFF_TMEMPTR + 16;
+  static constexpr int OFF_SCHED = OFF_TMEMPTR + 16;  // SchedTable (sched mode 1 only)
+  static constexpr int SMEM_ALLOC = OFF_SCHED + 4 * (2 * (SCHED_MAX_LEVELS + 2) + SCHED_MAX_SEQS);
   static constexpr int TMEM_COLS = 512;
   static constexpr int THREADS = 512;
   static constexpr int W_CORR = 8, W_MMA = 12, W_TMA = 14;  // first warp of each role
   static constexpr bool SEP_P = (D == 64);
   static constexpr int TMEM_P = 384;
   // registers after setmaxnreg.  setmaxnreg.inc only draws on the CTA's launch allocation
-  // (128 x 512 = 65536), so 8 x 32 x 192 + 4 x 32 x 80 + 4 x 32 x 48 = 65536 must not be exceeded.
-  static constexpr int REG_SOFTMAX = 192, REG_CORR = 80, REG_MISC = 48;
+  // (128 x 512 = 65536), so 8 x 32 x 192 + 4 x 32 x 56 + 4 x 32 x 72 = 65536 must not be exceeded
+  // (56 / 72: the MMA and TMA warps spill at 48, and those spills cost 2-12%).
+#ifndef FMHA_REG_CORR
+#define FMHA_REG_CORR 56
+#endif
+#ifndef FMHA_REG_MISC
+#define FMHA_REG_MISC 72
+#endif
+  static constexpr int REG_SOFTMAX = 192, REG_CORR = FMHA_REG_CORR, REG_MISC = FMHA_REG_MISC;
   // The two tiles' softmax warps on one SMSP (warps q and 4 + q) take turns for the exp phase, so
   // one tile's exponentials overlap the other's S load and row max (named barriers 2..9).
 #ifndef FMHA_TURNS
@@ -176,12 +206,22 @@ struct WorkItem {
   int r0, r1;    // first query row of tile 0 / 1
   int kv0, kv1;  // keys >= kv_t are masked for every row of tile t (key padding)
   int n0, n1;    // KV tiles visited by tile t (0 = tile absent or fully masked)
-  bool has1;     // tile 1 exists (tile 0 always does)
+  bool has0;     // tile 0 exists (always, except for varlen tiles past the sequence's end)
+  bool has1;     // tile 1 exists
+  int tok0, tok1;  // varlen: first token of the sequence of tile 0 / 1; len = its length
+  int len0, len1;
+  int head;        // varlen: h of unit bh0
+  // TMA coordinates (c1, c2) of the 128-row block starting at row r of tile t (c0 = d)
+  __device__ __forceinline__ int c1(bool varlen, int t, int r) const { return varlen ? head : r; }
+  __device__ __forceinline__ int c2(bool varlen, int t, int r) const { return varlen ? tok(t) + r : bh(t); }
   bool shared;
   __device__ __forceinline__ int n(int t) const { return t ? n1 : n0; }
   __device__ __forceinline__ int bh(int t) const { return t ? bh1 : bh0; }
   __device__ __forceinline__ int row0(int t) const { return t ? r1 : r0; }
   __device__ __forceinline__ int kv(int t) const { return t ? kv1 : kv0; }
+  __device__ __forceinline__ bool has(int t) const { return t ? has1 : has0; }
+  __device__ __forceinline__ int tok(int t) const { return t ? tok1 : tok0; }
+  __device__ __forceinline__ int len(int t) const { return t ? len1 : len0; }
   // number of K/V ring entries the item uses, and the ring index of K_{t,j} (V = K + 1)
   __device__ __forceinline__ int entries() const { return shared ? 2 * max(n0, n1) : 2 * (n0 + n1); }
   __device__ __forceinline__ int k_index(int t, int j) const {
@@ -189,7 +229,7 @@ struct WorkItem {
   }
 };
 
-template <bool PAIRX>
+template <bool PAIRX, bool VL>
 __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
   WorkItem w;
   int qt0;
@@ -221,7 +261,20 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
     w.r0 = qt0 * 128;
     w.r1 = qt1 * 128;
   }
+  w.has0 = true;
   w.kv0 = w.kv1 = p.seq_kv;
+  w.tok0 = w.tok1 = 0;
+  w.head = 0;
+  w.len0 = w.len1 = p.seq_q;
+  if constexpr (VL) {  // varlen (pair_mode 0): both tiles belong to unit bh0 = b * H + h
+    const int b = p.div_heads.div(w.bh0);
+    w.tok0 = w.tok1 = __ldg(p.cu_seqlens + b);
+    w.len0 = w.len1 = __ldg(p.cu_seqlens + b + 1) - w.tok0;
+    w.kv0 = w.kv1 = w.len0;
+    w.head = w.bh0 - b * p.heads;
+    w.has0 = w.r0 < w.len0;
+    w.has1 = w.has1 && w.r1 < w.len0;
+  }
   if (p.mask_kind == MASK_KEY_PADDING) {
     w.kv0 = min(max(__ldg(p.kv_len + p.div_heads.div(w.bh0)), 0), p.seq_kv);
     w.kv1 = w.shared ? w.kv0
@@ -233,15 +286,102 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
     kv_end0 = min(kv_end0, max(0, w.r0 + 128 + off));
     kv_end1 = min(kv_end1, max(0, w.r1 + 128 + off));
   }
-  w.n0 = (kv_end0 + 127) / 128;
+  w.n0 = w.has0 ? (kv_end0 + 127) / 128 : 0;
   w.n1 = w.has1 ? (kv_end1 + 127) / 128 : 0;
   return w;
 }
 
-// PAIRX = (pair_mode == 1): items may pair tiles of two units (see FmhaParams::pair_mode).
-template <int D, bool BF16, bool PAIRX>
+// Shared-memory table of sched mode 1: items_end[l] = number of items of level >= l (levels
+// descending), seq_start[l] = first entry of level l in seq_by_level, seq_by_level = sequence indices
+// sorted by decreasing level (ascending index within a level).
+struct SchedTable {
+  int items_end[SCHED_MAX_LEVELS + 2];
+  int seq_start[SCHED_MAX_LEVELS + 2];
+  int seq_by_level[SCHED_MAX_SEQS];
+};
+
+// Built by one full warp before the CTA's first __syncthreads.  Deterministic (no order-dependent
+// atomics), so every CTA derives the same order.
+__device__ __forceinline__ void build_sched(const FmhaParams& p, SchedTable* tb, int lane) {
+  const int L = p.max_level;
+  for (int l = lane; l <= L + 1; l += 32) tb->items_end[l] = tb->seq_start[l] = 0;
+  __syncwarp();
+  auto level_of = [&](int sq) {
+    if (sq >= p.num_seqs) return -1;
+    const int len = __ldg(p.cu_seqlens + sq + 1) - __ldg(p.cu_seqlens + sq);
+    return len <= 0 ? -1 : min((len + 127) >> 7, L);
+  };
+  for (int base = 0; base < p.num_seqs; base += 32) {  // sequences per level (into seq_start)
+    const int lv = level_of(base + lane);
+    if (lv > 0) atomicAdd(&tb->seq_start[lv], 1);
+  }
+  __syncwarp();
+  if (lane == 0) {  // prefix over descending levels
+    int seqs = 0, items = 0;
+    for (int l = L; l >= 1; --l) {
+      const int c = tb->seq_start[l];
+      tb->seq_start[l] = seqs;
+      seqs += c;
+      items += c * p.heads * ((l + 1) >> 1);
+      tb->items_end[l] = items;
+    }
+    tb->items_end[L + 1] = 0;
+    tb->items_end[0] = items;  // total
+  }
+  __syncwarp();
+  for (int base = 0; base < p.num_seqs; base += 32) {  // stable scatter, 32 sequences at a time
+    const int sq = base + lane;
+    const int lv = level_of(sq);
+    const unsigned same = __match_any_sync(0xffffffffu, lv);
+    if (lv > 0) {
+      const int rank = __popc(same & ((1u << lane) - 1u));
+      tb->seq_by_level[tb->seq_start[lv] + rank] = sq;
+    }
+    __syncwarp();
+    if (lv > 0 && lane == __ffs(same) - 1) tb->seq_start[lv] += __popc(same);
+    __syncwarp();
+  }
+  if (lane == 0) {  // undo the scatter's advance: seq_start[l] = first entry of level l again
+    int seqs = 0;
+    for (int l = L; l >= 1; --l) {
+      const int end = tb->seq_start[l];
+      tb->seq_start[l] = seqs;
+      seqs = end;
+    }
+  }
+  __syncwarp();
+}
+
+// The k-th work item of this CTA: its index in decode_item's numbering, or -1 when exhausted.
+template <bool SCHED>
+__device__ __forceinline__ int item_at(const FmhaParams& p, const SchedTable* tb, int k) {
+  const int G = gridDim.x, c = blockIdx.x;
+  if constexpr (!SCHED) {
+    const long long idx = c + static_cast<long long>(k) * G;
+    return idx < p.num_items ? static_cast<int>(idx) : -1;
+  } else {
+    const long long pos = static_cast<long long>(k) * G + ((k & 1) ? G - 1 - c : c);
+    if (pos >= tb->items_end[0]) return -1;
+    int l = p.max_level;
+    while (pos >= tb->items_end[l]) --l;  // items_end grows as l decreases
+    const int r = static_cast<int>(pos) - tb->items_end[l + 1];
+    const int pairs_l = (l + 1) >> 1, per = p.heads * pairs_l;
+    const int si = r / per, rem = r - si * per;
+    const int h = rem / pairs_l, pr = rem - h * pairs_l;
+    const int sq = tb->seq_by_level[tb->seq_start[l] + si];
+    return (sq * p.heads + h) * ((p.num_q_tiles + 1) >> 1) + pr;
+  }
+}
+
+// Kernel instances (MODE): dense [B,H,S,D]; dense with cross-unit tile pairing (pair_mode 1, see
+// FmhaParams::pair_mode); varlen packed; varlen packed with the cost-sorted schedule.  Separate
+// instances keep the varlen and scheduling code out of the dense kernels entirely.
+enum : int { MODE_DENSE = 0, MODE_PAIRX = 1, MODE_VARLEN = 2, MODE_VARLEN_SCHED = 3 };
+
+template <int D, bool BF16, int MODE>
 __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
   using C = FmhaCfg<D>;
+  constexpr bool PAIRX = MODE == MODE_PAIRX, VL = MODE >= MODE_VARLEN, SCHED = MODE == MODE_VARLEN_SCHED;
   // Dynamic shared memory starts at the (1024-byte aligned) base of the CTA's shared window; the
   // SWIZZLE_128B tiles need that alignment.  Using the base directly keeps smem addresses uniform.
   extern __shared__ __align__(1024) uint8_t smem[];
@@ -291,11 +431,13 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     tmem_alloc(smem_u32(tmem_holder), C::TMEM_COLS);
     tmem_relinquish();
   }
+  const SchedTable* sched = reinterpret_cast<const SchedTable*>(smem + C::OFF_SCHED);
+  if (SCHED && warp == C::W_TMA + 1) build_sched(p, reinterpret_cast<SchedTable*>(smem + C::OFF_SCHED), lane);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_holder;
-  const int first = blockIdx.x, stride = gridDim.x;
+  // this CTA's k-th item: item_at<SCHED>(p, sched, k) (-1 when exhausted)
 
   if (warp >= C::W_MMA) {
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(C::REG_MISC));
@@ -304,7 +446,8 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       const uint64_t keep = policy_evict_last();   // K/V: re-read by the other q-tile pairs
       const uint64_t once = policy_evict_first();  // Q: read once
       uint32_t kv = 0, qc0 = 0, qc1 = 0;
-      auto load_kv = [&](int bh, int j) {
+      constexpr bool vl = VL;
+      auto load_kv = [&](const WorkItem& w, int t, int j) {
 #pragma unroll
         for (int m = 0; m < 2; ++m, ++kv) {  // m = 0: K_j, m = 1: V_j
           const int s = kv % C::NS;
@@ -315,11 +458,11 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
 #pragma unroll
           for (int c = 0; c < D / 64; ++c)
             tma_load_3d_hint_elect(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64,
-                                   j * 128, bh, keep);
+                                   w.c1(vl, t, j * 128), w.c2(vl, t, j * 128), keep);
         }
       };
-      for (int idx = first; idx < p.num_items; idx += stride) {
-        const WorkItem w = decode_item<PAIRX>(p, idx);
+      for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
+        const WorkItem w = decode_item<PAIRX, VL>(p, idx);
         const int N = max(w.n0, w.n1);
 #pragma unroll
         for (int t = 0; t < 2; ++t) {
@@ -331,16 +474,16 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
 #pragma unroll
           for (int c = 0; c < D / 64; ++c)
             tma_load_3d_hint_elect(sbase + C::OFF_Q + (2 * qs + t) * C::TILE + c * C::CHUNK, &p.tmQ, Q_FULL(t, qs),
-                                   c * 64, w.row0(t), w.bh(t), once);
+                                   c * 64, w.c1(vl, t, w.row0(t)), w.c2(vl, t, w.row0(t)), once);
           ++qc;
           TRACE_EV(EV_ITEM, 4 + t);
         }
         for (int j = 0; j < N; ++j) {
           if (w.shared) {
-            load_kv(w.bh0, j);
+            load_kv(w, 0, j);
           } else {
-            if (j < w.n0) load_kv(w.bh0, j);
-            if (j < w.n1) load_kv(w.bh1, j);
+            if (j < w.n0) load_kv(w, 0, j);
+            if (j < w.n1) load_kv(w, 1, j);
           }
         }
       }
@@ -380,20 +523,21 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       };
       struct Cursor {
         Ring w;
-        int idx, j, N, qs;
+        int idx, k, j, N, qs;
         uint32_t base;  // ring index of the item's first K/V entry (WorkItem::k_index)
         bool valid;
       };
-      auto seek = [&](Cursor& cu, int idx, uint32_t base) {
+      auto seek = [&](Cursor& cu, int k, uint32_t base) {
         cu.valid = false;
-        for (; idx < p.num_items; idx += stride) {
-          const WorkItem w = decode_item<PAIRX>(p, idx);
+        for (int idx; (idx = item_at<SCHED>(p, sched, k)) >= 0; ++k) {
+          const WorkItem w = decode_item<PAIRX, VL>(p, idx);
           const int N = max(w.n0, w.n1);
           if (N == 0) continue;
           cu.w.n0 = w.n0;
           cu.w.n1 = w.n1;
           cu.w.shared = w.shared;
           cu.idx = idx;
+          cu.k = k;
           cu.j = 0;
           cu.N = N;
           cu.base = base;
@@ -402,10 +546,10 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         }
       };
       auto advance = [&](Cursor& cu) {
-        if (++cu.j == cu.N) seek(cu, cu.idx + stride, cu.base + cu.w.entries());
+        if (++cu.j == cu.N) seek(cu, cu.k + 1, cu.base + cu.w.entries());
       };
       Cursor cq, cp;
-      seek(cq, first, 0);
+      seek(cq, 0, 0);
       cp = cq;
       // S_t <- Q_t K_j^T (separate P: once the softmax warps have read the previous S_t)
       // Every K/V ring entry is released exactly once by each MMA warp (KV_EMPTY count 2): a warp
@@ -524,14 +668,16 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     const int off = p.seq_kv - p.seq_q;
     // g = real steps this thread has done so far: the phase count of S_FULL and PV_DONE
     uint32_t g = 0, lc = 0;
-    for (int idx = first; idx < p.num_items; idx += stride) {
-      const WorkItem w = decode_item<PAIRX>(p, idx);
+    for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
+      const WorkItem w = decode_item<PAIRX, VL>(p, idx);
       const int n = w.n(t);
       const int N = C::TURNS ? max(w.n0, w.n1) : n;
       TRACE_EV(EV_ITEM, 1);
       const int qi = w.row0(t) + row;
       int lim = w.kv(t);  // keys j < lim are visible to this row
       if (p.mask_kind == MASK_CAUSAL) lim = min(lim, qi + off + 1);
+      if (qi >= w.len(t)) lim = 0;  // row past the sequence's end: never stored, so no work
+      const int lim_w = __reduce_max_sync(0xffffffffu, lim);  // keys >= lim_w: masked for the warp
       float m_ref = -INFINITY;  // max used as the exp2 reference (lags the true max by < 2^8)
       float l = 0.f;            // row sum relative to m_ref
       for (int j = 0; j < N; ++j) {
@@ -555,6 +701,8 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           mbar_arrive(S_FREE);
         }
         const int rem = lim - j * 128;
+        // 32-key chunks no row of this warp can see are skipped: their P is stored as zeros
+        const int rem_w = lim_w - j * 128;
         if (rem < 128) {  // boundary tile for this row (a5)
 #pragma unroll
           for (int k = 0; k < 128; ++k)
@@ -590,6 +738,10 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         // P = exp2(c*s - c*m_ref) (a6), rounded to the I/O type, stored to TMEM for the PV MMA
         float2 acc0 = make_float2(0.f, 0.f), acc1 = make_float2(0.f, 0.f);
         float mcv = mc;
+        // two instances: no chunk test at all on unmasked steps (the common case), so ptxas can
+        // interleave the chunks freely; per-chunk skipping on steps with masked columns
+        auto exp_phase = [&](auto skip_tag) {
+          constexpr bool SKIP = decltype(skip_tag)::value;
 #pragma unroll
         for (int hh = 0; hh < 4; ++hh) {
           if (hh == C::PRE_CHUNKS) {
@@ -601,6 +753,12 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             asm volatile("ld.volatile.shared.f32 %0, [%1];" : "=f"(mcv) : "r"(slot) : "memory");
           }
           uint32_t pk[16];
+          if (SKIP && 32 * hh >= rem_w) {
+#pragma unroll
+            for (int u = 0; u < 16; ++u) pk[u] = 0u;
+            tmem_st_32x32b_x16(tP + 16 * hh, pk);
+            continue;
+          }
 #pragma unroll
           for (int u = 0; u < 16; u += 2) {
             const int k = 32 * hh + 2 * u;
@@ -635,6 +793,11 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           }
           tmem_st_32x32b_x16(tP + 16 * hh, pk);
         }
+        };
+        if (rem_w >= 128)
+          exp_phase(std::false_type{});
+        else
+          exp_phase(std::true_type{});
         if (C::TURNS) named_bar_arrive(other_turn, 64);
         TRACE_EV(EV_EXP_DONE, j);
         // lazy rescale of this warp's rows of O_t (a7), after the exponentials so that S is no
@@ -657,7 +820,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         mbar_arrive(P_FULL);
         l = l * alpha + ((acc0.x + acc0.y) + (acc1.x + acc1.y));
       }
-      if (t == 1 && !w.has1) continue;
+      if (!w.has(t)) continue;
       // the epilogue has read the previous item's sums (without this wait the softmax can run two
       // items ahead and L_FULL's phase parity would alias)
       TRACE_EV(EV_ITEM, 2);
@@ -675,12 +838,12 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     const int row = quad * 32 + lane;
     const uint32_t lane_off = static_cast<uint32_t>(quad * 32) << 16;
     uint32_t ofc[2] = {0, 0}, lc[2] = {0, 0};
-    for (int idx = first; idx < p.num_items; idx += stride) {
-      const WorkItem w = decode_item<PAIRX>(p, idx);
+    for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
+      const WorkItem w = decode_item<PAIRX, VL>(p, idx);
       // ------------------------------------------------------------ epilogue per tile (a9)
 #pragma unroll 1
       for (int t = 0; t < 2; ++t) {
-        if (t == 1 && !w.has1) continue;
+        if (!w.has(t)) continue;
         mbar_wait_at(BAR(C::B_L_FULL + t), lc[t] & 1, 13, lc[t], idx);
         TRACE_EV(EV_EPI, 100 + t);
         ++lc[t];
@@ -694,6 +857,9 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           tc_fence_after();
         }
         const float inv_l = (l > 0.f) ? 1.f / l : 0.f;  // fully masked row -> 0 (R4)
+        // varlen tile that crosses its sequence's end: a TMA store would overwrite the next
+        // sequence's rows, so each thread stores its own row (if inside the sequence) instead
+        const bool rowwise = VL && w.row0(t) + 128 > w.len(t);
         const uint32_t stg = sbase + C::OFF_STG + (t % C::NSTG) * C::TILE;
         if (row == 0) tma_store_wait_read0();  // previous store out of this staging buffer done
         named_bar_sync(1, 128);
@@ -714,24 +880,32 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
 #pragma unroll
           for (int u = 0; u < 4; ++u) {
             const int unit = ((col0 % 64) / 8) + u;
-            st_shared_v4(box + ((unit ^ (row & 7)) << 4),
-                         pack2<BF16>(__uint_as_float(o[8 * u + 0]) * inv_l, __uint_as_float(o[8 * u + 1]) * inv_l),
-                         pack2<BF16>(__uint_as_float(o[8 * u + 2]) * inv_l, __uint_as_float(o[8 * u + 3]) * inv_l),
-                         pack2<BF16>(__uint_as_float(o[8 * u + 4]) * inv_l, __uint_as_float(o[8 * u + 5]) * inv_l),
-                         pack2<BF16>(__uint_as_float(o[8 * u + 6]) * inv_l, __uint_as_float(o[8 * u + 7]) * inv_l));
+            const uint32_t v0 = pack2<BF16>(__uint_as_float(o[8 * u + 0]) * inv_l, __uint_as_float(o[8 * u + 1]) * inv_l);
+            const uint32_t v1 = pack2<BF16>(__uint_as_float(o[8 * u + 2]) * inv_l, __uint_as_float(o[8 * u + 3]) * inv_l);
+            const uint32_t v2 = pack2<BF16>(__uint_as_float(o[8 * u + 4]) * inv_l, __uint_as_float(o[8 * u + 5]) * inv_l);
+            const uint32_t v3 = pack2<BF16>(__uint_as_float(o[8 * u + 6]) * inv_l, __uint_as_float(o[8 * u + 7]) * inv_l);
+            if (!rowwise) {
+              st_shared_v4(box + ((unit ^ (row & 7)) << 4), v0, v1, v2, v3);
+            } else if (row < w.len(t) - w.row0(t)) {  // varlen partial tile: rows inside the sequence
+              const size_t tokn = static_cast<size_t>(w.tok(t) + w.row0(t) + row);
+              st_global_v4(p.o_ptr + 2 * (tokn * p.o_row_elems + w.head * D + col0 + 8 * u), v0, v1, v2, v3);
+            }
           }
         }
         if (n > 0) {  // O_t read: the next item's first PV may overwrite it
           tc_fence_before();
           mbar_arrive(BAR(C::B_O_EMPTY + t));
         }
-        fence_proxy_async_smem();
-        named_bar_sync(1, 128);
-        if (row == 0) {
+        if (!rowwise) {
+          fence_proxy_async_smem();
+          named_bar_sync(1, 128);
+          if (row == 0) {
+            constexpr bool vl = VL;
 #pragma unroll
-          for (int c2 = 0; c2 < D / 64; ++c2)
-            tma_store_3d(&p.tmO, stg + c2 * C::CHUNK, c2 * 64, w.row0(t), w.bh(t));
-          tma_store_commit();
+            for (int c2 = 0; c2 < D / 64; ++c2)
+              tma_store_3d(&p.tmO, stg + c2 * C::CHUNK, c2 * 64, w.c1(vl, t, w.row0(t)), w.c2(vl, t, w.row0(t)));
+            tma_store_commit();
+          }
         }
         TRACE_EV(EV_EPI, 120 + t);
       }

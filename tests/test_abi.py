@@ -70,6 +70,16 @@ def test_validation_codes(lib):
     assert lib.gemm_bias_act(16, 16, None, 16, 4, 8, 12, 0, None) == 2  # K % 8
     assert lib.gemm_bias_act(16, 16, None, 16, 4, 8, 16, 9, None) == 2  # act
     assert lib.gemm_bias_act(16, 16, None, 16, 0, 8, 16, 0, None) == 0
+    # varlen: validation before any device access
+    vl = lib.fmha_fwd_varlen
+    assert vl(16, 16, 16, 2, 8, 16, 2, 96, 0.1, 0, 0, None) == 2       # head_dim
+    assert vl(16, 16, 16, 2, 8, 16, 2, 64, -1.0, 0, 0, None) == 2      # negative scale
+    assert vl(16, 16, 16, 2, 8, 16, 2, 64, 0.1, 2, 0, None) == 2       # causal flag
+    assert vl(16, 16, 16, 2, 8, 16, 2, 64, 0.1, 0, 5, None) == 2       # dtype
+    assert vl(None, 16, 16, 2, 8, 16, 2, 64, 0.1, 0, 0, None) == 1     # null QKV
+    assert vl(24, 16, 16, 2, 8, 16, 2, 64, 0.1, 0, 0, None) == 3       # misaligned
+    assert vl(16, 16, 16, -1, 8, 16, 2, 64, 0.1, 0, 0, None) == 1
+    assert vl(None, None, None, 0, 8, 16, 2, 64, 0.1, 0, 0, None) == 0  # no sequences
     assert lib.fmha_workspace_bytes(2, 3, 100, 50, 64) >= 2 * (2 * 3 * 100 * 64 * 2) + 2 * (2 * 3 * 50 * 64 * 2)
 
 

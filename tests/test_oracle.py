@@ -15,7 +15,7 @@ import numpy as np
 import pytest
 import torch
 
-from oracle import (attention_brute, attention_fp64, attention_rows_fp64, fmha_flops,
+from oracle import (attention_brute, attention_fp64, attention_rows_fp64, attention_varlen_fp64, fmha_flops,
                     gemm_bias_act_fp64, gelu_erf, gelu_tanh, softmax_probs_fp64)
 from oracle.gemm import ACT_GELU_ERF, ACT_GELU_TANH, ACT_NONE, ACT_RELU
 from workloads import CONFIGS, make_fmha_inputs
@@ -252,3 +252,59 @@ def test_workloads_shard_reproducible():
     assert list(kl[2:]) == list(kl2)
     assert kl[0] == 16 and all(16 >= x >= 16 for x in kl[:1])
     assert q.dtype == torch.float16
+
+
+# ---------------------------------------------------------------- varlen packed layout (f2)
+def _brute_varlen(x, cu, scale, causal):
+    """Pin for attention_varlen_fp64 via the pure-Python brute force, one sequence at a time."""
+    t, _, h_, d = x.shape
+    out = np.zeros((t, h_, d))
+    for s in range(len(cu) - 1):
+        a, b = int(cu[s]), int(cu[s + 1])
+        if b <= a:
+            continue
+        q = [[[list(map(float, x[i, 0, h])) for i in range(a, b)] for h in range(h_)]]
+        k = [[[list(map(float, x[i, 1, h])) for i in range(a, b)] for h in range(h_)]]
+        v = [[[list(map(float, x[i, 2, h])) for i in range(a, b)] for h in range(h_)]]
+        o = attention_brute(q, k, v, scale, None, causal)[0]
+        for h in range(h_):
+            out[a:b, h] = np.array(o[h])
+    return out
+
+
+@pytest.mark.parametrize("causal", [False, True])
+def test_varlen_brute_force(causal):
+    lens = [3, 0, 5, 1, 4]
+    cu = np.concatenate([[0], np.cumsum(lens)]).astype(np.int32)
+    x = rnd((int(cu[-1]), 3, 2, 4), 7)
+    o = attention_varlen_fp64(x, cu, 0.5, causal)
+    np.testing.assert_allclose(o, _brute_varlen(x, cu, 0.5, causal), atol=1e-13, rtol=0)
+
+
+def test_varlen_equal_lengths_is_dense_layout():
+    """Equal lengths: the packed problem is the dense [B,H,S,D] one with Q/K/V transposed."""
+    b, s, h, d = 3, 7, 2, 8
+    x = rnd((b * s, 3, h, d), 11)
+    cu = np.arange(0, b * s + 1, s, dtype=np.int32)
+    o = attention_varlen_fp64(x, cu, 1 / math.sqrt(d))
+    xs = x.reshape(b, s, 3, h, d).transpose(2, 0, 3, 1, 4)  # [3, B, H, S, D]
+    od = attention_fp64(xs[0], xs[1], xs[2], 1 / math.sqrt(d))  # [B, H, S, D]
+    np.testing.assert_allclose(o, od.transpose(0, 2, 1, 3).reshape(b * s, h, d), atol=1e-14, rtol=0)
+
+
+def test_varlen_sequences_do_not_interact():
+    """Garbage in one sequence's tokens leaves every other sequence's output unchanged, and the
+    first token of a causal sequence returns its own V (closed form)."""
+    lens = [6, 9, 4]
+    cu = np.concatenate([[0], np.cumsum(lens)]).astype(np.int32)
+    x = rnd((int(cu[-1]), 3, 2, 8), 5)
+    o = attention_varlen_fp64(x, cu, 0.3)
+    y = x.copy()
+    y[cu[1]:cu[2]] = rnd((lens[1], 3, 2, 8), 6, sigma=50.0)
+    o2 = attention_varlen_fp64(y, cu, 0.3)
+    keep = np.r_[cu[0]:cu[1], cu[2]:cu[3]]
+    np.testing.assert_array_equal(o[keep], o2[keep])
+    assert not np.allclose(o[cu[1]:cu[2]], o2[cu[1]:cu[2]])
+    oc = attention_varlen_fp64(x, cu, 0.3, causal=True)
+    for s in range(3):
+        np.testing.assert_array_equal(oc[cu[s]], x[cu[s], 2])

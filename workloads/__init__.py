@@ -14,7 +14,12 @@ Recipe:
   * drawn in float32, then rounded to fp16 / bf16 with round-to-nearest-even;
   * key padding (BERT-base config): kv_len[b] ~ U{32..S}, with kv_len[0] = S so
     at least one batch is unpadded;
-  * MLP: A ~ U(-1, 1), W ~ N(0, 1/K), b ~ U(-1, 1).
+  * MLP: A ~ U(-1, 1), W ~ N(0, 1/K), b ~ U(-1, 1);
+  * packed variable-length batches (MLPerf BERT inference layout):
+    sequence lengths ~ round(N(175, 75^2)) clipped to [32, max_seqlen], with
+    sequence 0 at max_seqlen (SQuAD v1.1 tokenised for MLPerf BERT averages ~170
+    tokens with a 384 cap -- an assumption); Q, K, V of each
+    (sequence, head) drawn like the dense configs' (b, h) slices.
 """
 
 from __future__ import annotations
@@ -79,6 +84,70 @@ class MlpConfig:
 
 
 MLP_CONFIG = MlpConfig("mlp", 6, 16384, 1024, 4096)
+
+
+@dataclass(frozen=True)
+class VarlenConfig:
+    """A packed variable-length batch: QKV [T, 3, H, D], cu_seqlens [num_seqs + 1]."""
+    name: str
+    cfg_id: int
+    num_seqs: int
+    heads: int
+    max_seqlen: int
+    head_dim: int
+    dtype: str = "fp16"
+    causal: bool = False
+    mean_len: float = 175.0
+    sd_len: float = 75.0
+    min_len: int = 32
+
+    @property
+    def scale(self) -> float:
+        return float(np.float32(1.0 / np.sqrt(self.head_dim)))
+
+    @property
+    def torch_dtype(self):
+        return torch.float16 if self.dtype == "fp16" else torch.bfloat16
+
+    def with_(self, **kw) -> "VarlenConfig":
+        return replace(self, **kw)
+
+
+# MLPerf-style BERT-large inference batch (the paper's workload, P:L489): 32 sequences, 16 heads,
+# D = 64, max 384 tokens, packed without padding
+VARLEN_CONFIGS = {
+    "bert_large_varlen": VarlenConfig("bert_large_varlen", 8, 32, 16, 384, 64),
+}
+
+
+def varlen_lengths(cfg: VarlenConfig, seq_offset: int = 0, seed: int = SEED) -> np.ndarray:
+    out = np.empty(cfg.num_seqs, dtype=np.int64)
+    for s in range(cfg.num_seqs):
+        gs = s + seq_offset
+        if gs == 0:
+            out[s] = cfg.max_seqlen
+        else:
+            x = _rng(cfg.cfg_id, 9, gs, 0, seed).normal(cfg.mean_len, cfg.sd_len)
+            out[s] = int(np.clip(np.rint(x), min(cfg.min_len, cfg.max_seqlen), cfg.max_seqlen))
+    return out
+
+
+def make_varlen_inputs(cfg: VarlenConfig, seq_offset: int = 0, seed: int = SEED, lengths=None):
+    """Returns (qkv [T,3,H,D] CPU tensor in cfg's dtype, cu_seqlens int32 numpy [num_seqs+1]).
+    Global sequence index = s + seq_offset.  ``lengths`` overrides the drawn lengths."""
+    lens = varlen_lengths(cfg, seq_offset, seed) if lengths is None else np.asarray(lengths, dtype=np.int64)
+    cu = np.zeros(len(lens) + 1, dtype=np.int32)
+    cu[1:] = np.cumsum(lens)
+    t, h_, d = int(cu[-1]), cfg.heads, cfg.head_dim
+    x = np.empty((t, 3, h_, d), dtype=np.float32)
+    for s in range(len(lens)):
+        a, b = int(cu[s]), int(cu[s + 1])
+        gs = s + seq_offset
+        for h in range(h_):
+            x[a:b, 0, h] = _rng(cfg.cfg_id, 0, gs, h, seed).standard_normal((b - a, d), dtype=np.float32)
+            x[a:b, 1, h] = _rng(cfg.cfg_id, 1, gs, h, seed).standard_normal((b - a, d), dtype=np.float32)
+            x[a:b, 2, h] = _rng(cfg.cfg_id, 2, gs, h, seed).uniform(-1.0, 1.0, (b - a, d)).astype(np.float32)
+    return _round(x, cfg.torch_dtype), cu
 
 
 def _round(x32: np.ndarray, tdtype) -> torch.Tensor:
