@@ -120,6 +120,26 @@ typedef enum { ACT_NONE = 0, ACT_RELU = 1, ACT_GELU_ERF = 2, ACT_GELU_TANH = 3 }
 FMHA_API int gemm_bias_act(const void* A, const void* W, const void* bias, void* C, int M, int N, int K, int act,
                   fmha_stream_t stream);
 
+/* End-to-end synthetic Transformer layer (the paper's end-to-end use of its
+ * fused kernels), fp16, tokens packed as in fmha_fwd_varlen:
+ *     QKV = X Wqkv^T + bqkv        X [T, d_model], Wqkv [3 d_model, d_model] (rows: Q heads, K heads,
+ *                                  V heads, so QKV is the [T, 3, heads, head_dim] layout)
+ *     A   = fmha_varlen(QKV)       per-sequence attention, [T, heads, head_dim] = [T, d_model]
+ *     Z   = A Wo^T + bo            Wo [d_model, d_model]
+ *     H   = GELU_erf(Z W1^T + b1)  W1 [d_ff, d_model]
+ *     Y   = H W2^T + b2            W2 [d_model, d_ff], Y [T, d_model]
+ * (no residual adds or LayerNorm: DESIGN.md R18).  Five launches on `stream` (three of them the
+ * gemm_bias_act kernel, one fmha).  head_dim = d_model / heads must be 64 or 128; d_model and d_ff
+ * multiples of 8; biases may be NULL.  Intermediates live in `workspace` (DEVICE, 256-byte aligned,
+ * >= transformer_layer_workspace_bytes(T, d_model, d_ff) bytes).  Errors: as the component calls;
+ * the first failing launch's status is returned and later stages are not launched. */
+FMHA_API size_t transformer_layer_workspace_bytes(int tokens, int d_model, int d_ff);
+FMHA_API int transformer_layer_fwd(const void* X, const void* Wqkv, const void* bqkv, const void* Wo,
+                                   const void* bo, const void* W1, const void* b1, const void* W2, const void* b2,
+                                   void* Y, const int32_t* cu_seqlens, int num_seqs, int max_seqlen, int tokens,
+                                   int d_model, int heads, int d_ff, float scale, int causal, void* workspace,
+                                   size_t workspace_bytes, fmha_stream_t stream);
+
 /* Human-readable text for a status code (static storage). */
 FMHA_API const char* fmha_status_string(int status);
 /* Text of the last CUDA error seen by this thread inside the library ("" if none). */

@@ -9,6 +9,7 @@ sm_100 device these functions raise.
     fmha_fwd_varlen(qkv, cu_seqlens, max_seqlen, causal=False, scale=None, out=None) -> O
     fmha_fwd_from_host(q, k, v, ..., workspace) -> O  (host tensors; copies inside the call)
     gemm_bias_act(a, w, bias=None, act="none", out=None) -> C
+    transformer_layer(x, weights, cu_seqlens, max_seqlen, heads, ...) -> Y  (5 launches, one call)
 """
 
 from __future__ import annotations
@@ -21,7 +22,7 @@ import torch
 from . import _lib
 from ._lib import FmhaError, FmhaMask
 
-__all__ = ["fmha_fwd", "fmha_fwd_varlen", "fmha_fwd_from_host", "gemm_bias_act", "workspace_bytes", "FmhaError",
+__all__ = ["fmha_fwd", "fmha_fwd_varlen", "fmha_fwd_from_host", "gemm_bias_act", "transformer_layer", "layer_workspace_bytes", "workspace_bytes", "FmhaError",
            "MASK_NONE", "MASK_KEY_PADDING", "MASK_CAUSAL", "ACTS", "version"]
 
 MASK_NONE, MASK_KEY_PADDING, MASK_CAUSAL = 0, 1, 2
@@ -151,4 +152,41 @@ def gemm_bias_act(a: torch.Tensor, w: torch.Tensor, bias: torch.Tensor | None = 
     st = lib.gemm_bias_act(a.data_ptr(), w.data_ptr(), None if bias is None else bias.contiguous().data_ptr(),
                            out.data_ptr(), m_, n_, k_, ACTS[act], _stream_ptr(a.device))
     _lib.check(st, "gemm_bias_act")
+    return out
+
+
+def layer_workspace_bytes(tokens: int, d_model: int, d_ff: int) -> int:
+    return int(_lib.load().transformer_layer_workspace_bytes(tokens, d_model, d_ff))
+
+
+def transformer_layer(x: torch.Tensor, wqkv: torch.Tensor, bqkv, wo: torch.Tensor, bo, w1: torch.Tensor, b1,
+                      w2: torch.Tensor, b2, cu_seqlens: torch.Tensor, max_seqlen: int, heads: int,
+                      causal: bool = False, scale: float | None = None, out: torch.Tensor | None = None,
+                      workspace: torch.Tensor | None = None) -> torch.Tensor:
+    """Y = MLP(out_proj(FMHA(QKV_proj(x)))) for packed tokens x [T, d_model] (fp16 CUDA), one call to
+    ``transformer_layer_fwd`` of the C ABI (DESIGN.md R18).  Weights in nn.Linear layout [out, in];
+    biases [out] or None."""
+    lib = _lib.load()
+    ts = [x, wqkv, wo, w1, w2] + [b for b in (bqkv, bo, b1, b2) if b is not None]
+    if any(t.dtype != torch.float16 or not t.is_cuda or not t.is_contiguous() for t in ts):
+        raise TypeError("transformer_layer takes contiguous fp16 CUDA tensors")
+    t_, d = x.shape
+    d_ff = w1.shape[0]
+    if wqkv.shape != (3 * d, d) or wo.shape != (d, d) or w1.shape != (d_ff, d) or w2.shape != (d, d_ff):
+        raise ValueError("weight shapes must be Wqkv [3d,d], Wo [d,d], W1 [d_ff,d], W2 [d,d_ff]")
+    if cu_seqlens.dtype != torch.int32 or not cu_seqlens.is_cuda:
+        raise ValueError("cu_seqlens must be a CUDA int32 tensor")
+    if out is None:
+        out = torch.empty((t_, d), dtype=torch.float16, device=x.device)
+    need = layer_workspace_bytes(t_, d, d_ff)
+    if workspace is None or workspace.numel() * workspace.element_size() < need:
+        workspace = torch.empty(need, dtype=torch.uint8, device=x.device)
+    scale = 1.0 / math.sqrt(d // heads) if scale is None else float(scale)
+    ptr = lambda b: None if b is None else b.data_ptr()
+    st = lib.transformer_layer_fwd(x.data_ptr(), wqkv.data_ptr(), ptr(bqkv), wo.data_ptr(), ptr(bo), w1.data_ptr(),
+                                   ptr(b1), w2.data_ptr(), ptr(b2), out.data_ptr(), cu_seqlens.data_ptr(),
+                                   cu_seqlens.numel() - 1, int(max_seqlen), t_, d, heads, d_ff, scale,
+                                   int(bool(causal)), workspace.data_ptr(),
+                                   workspace.numel() * workspace.element_size(), _stream_ptr(x.device))
+    _lib.check(st, "transformer_layer_fwd")
     return out

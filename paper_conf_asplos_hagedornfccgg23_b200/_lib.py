@@ -31,6 +31,8 @@ EXPORTED_SYMBOLS = (
     "fmha_workspace_bytes",
     "fmha_fwd_from_host",
     "gemm_bias_act",
+    "transformer_layer_workspace_bytes",
+    "transformer_layer_fwd",
     "fmha_status_string",
     "fmha_last_cuda_error",
     "fmha_version",
@@ -76,6 +78,11 @@ def load() -> ctypes.CDLL:
     lib.fmha_fwd_from_host.restype = i32
     lib.gemm_bias_act.argtypes = [vp, vp, vp, vp, i32, i32, i32, i32, vp]
     lib.gemm_bias_act.restype = i32
+    if hasattr(lib, "transformer_layer_fwd"):  # absent only in old tuning builds
+        lib.transformer_layer_workspace_bytes.argtypes = [i32, i32, i32]
+        lib.transformer_layer_workspace_bytes.restype = sz
+        lib.transformer_layer_fwd.argtypes = [vp] * 10 + [vp, i32, i32, i32, i32, i32, i32, f32, i32, vp, sz, vp]
+        lib.transformer_layer_fwd.restype = i32
     for name in ("fmha_status_string",):
         getattr(lib, name).argtypes = [i32]
         getattr(lib, name).restype = ctypes.c_char_p

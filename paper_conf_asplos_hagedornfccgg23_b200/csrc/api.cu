@@ -291,6 +291,43 @@ int fmha_fwd_varlen(const void* QKV, void* O, const int32_t* cu_seqlens, int num
                             scale, causal, reinterpret_cast<cudaStream_t>(stream));
 }
 
+size_t transformer_layer_workspace_bytes(int tokens, int d_model, int d_ff) {
+  if (tokens < 0 || d_model < 0 || d_ff < 0) return 0;
+  const size_t t = static_cast<size_t>(tokens);
+  return round_up(t * 3 * d_model * 2, 256) + 2 * round_up(t * d_model * 2, 256) + round_up(t * d_ff * 2, 256);
+}
+
+int transformer_layer_fwd(const void* X, const void* Wqkv, const void* bqkv, const void* Wo, const void* bo,
+                          const void* W1, const void* b1, const void* W2, const void* b2, void* Y,
+                          const int32_t* cu_seqlens, int num_seqs, int max_seqlen, int tokens, int d_model,
+                          int heads, int d_ff, float scale, int causal, void* workspace, size_t workspace_bytes,
+                          fmha_stream_t stream) {
+  g_last_cuda_error[0] = 0;
+  if (tokens < 0 || d_model <= 0 || heads <= 0 || d_ff <= 0 || num_seqs < 0 || max_seqlen < 0)
+    return FMHA_ERR_INVALID_ARG;
+  if (d_model % heads != 0) return FMHA_ERR_INVALID_ARG;
+  const int head_dim = d_model / heads;
+  if (head_dim != 64 && head_dim != 128) return FMHA_ERR_UNSUPPORTED;
+  if (tokens == 0) return FMHA_OK;
+  if (!X || !Wqkv || !Wo || !W1 || !W2 || !Y || !cu_seqlens || !workspace) return FMHA_ERR_INVALID_ARG;
+  if (workspace_bytes < transformer_layer_workspace_bytes(tokens, d_model, d_ff)) return FMHA_ERR_INVALID_ARG;
+  if ((reinterpret_cast<uintptr_t>(workspace) & 255u) != 0) return FMHA_ERR_MISALIGNED;
+  const size_t t = static_cast<size_t>(tokens);
+  uint8_t* w = static_cast<uint8_t*>(workspace);
+  uint8_t* qkv = w;                                       // [T, 3, H, D]
+  uint8_t* attn = qkv + round_up(t * 3 * d_model * 2, 256);  // [T, H, D] = [T, d_model]
+  uint8_t* z = attn + round_up(t * d_model * 2, 256);     // [T, d_model]
+  uint8_t* h = z + round_up(t * d_model * 2, 256);        // [T, d_ff]
+  int st;
+  if ((st = gemm_bias_act(X, Wqkv, bqkv, qkv, tokens, 3 * d_model, d_model, ACT_NONE, stream)) != FMHA_OK) return st;
+  if ((st = fmha_varlen_common(false, qkv, attn, cu_seqlens, num_seqs, max_seqlen, tokens, heads, head_dim, scale,
+                               causal, reinterpret_cast<cudaStream_t>(stream))) != FMHA_OK)
+    return st;
+  if ((st = gemm_bias_act(attn, Wo, bo, z, tokens, d_model, d_model, ACT_NONE, stream)) != FMHA_OK) return st;
+  if ((st = gemm_bias_act(z, W1, b1, h, tokens, d_ff, d_model, ACT_GELU_ERF, stream)) != FMHA_OK) return st;
+  return gemm_bias_act(h, W2, b2, Y, tokens, d_model, d_ff, ACT_NONE, stream);
+}
+
 size_t fmha_workspace_bytes(int batch, int heads, int seq_q, int seq_kv, int head_dim) {
   if (batch < 0 || heads < 0 || seq_q < 0 || seq_kv < 0 || head_dim < 0) return 0;
   const size_t u = static_cast<size_t>(batch) * heads;

@@ -308,3 +308,30 @@ def test_varlen_sequences_do_not_interact():
     oc = attention_varlen_fp64(x, cu, 0.3, causal=True)
     for s in range(3):
         np.testing.assert_array_equal(oc[cu[s]], x[cu[s], 2])
+
+
+# ---------------------------------------------------------------- synthetic Transformer layer (f1)
+def test_layer_matches_torch_fp64_composition():
+    """Library special case: the same five stages written with torch's float64 CPU linear, SDPA and
+    erf-GELU, rounding every stored intermediate to fp16 (R18)."""
+    from oracle import transformer_layer_fp64
+    from workloads import LayerConfig, make_layer_inputs
+    import torch.nn.functional as F
+    cfg = LayerConfig("tiny_layer", 31, 3, 0, 16, 2, 32)
+    (x, wqkv, bqkv, wo, bo, w1, b1, w2, b2), cu = make_layer_inputs(cfg, lengths=[5, 9, 3])
+    y = transformer_layer_fp64(x, wqkv, bqkv, wo, bo, w1, b1, w2, b2, cu, cfg.heads, cfg.scale)
+    d64 = lambda t: t.double()
+    r16 = lambda t: t.half().double()
+    qkv = r16(F.linear(d64(x), d64(wqkv), d64(bqkv))).view(-1, 3, 2, 8)
+    a = torch.zeros(qkv.shape[0], 2, 8, dtype=torch.float64)
+    for s in range(3):
+        lo, hi = int(cu[s]), int(cu[s + 1])
+        q, k, v = (qkv[lo:hi, i].transpose(0, 1) for i in range(3))
+        a[lo:hi] = F.scaled_dot_product_attention(q, k, v, scale=float(np.float32(cfg.scale))).transpose(0, 1)
+    z = r16(F.linear(r16(a.reshape(-1, 16)), d64(wo), d64(bo)))
+    h = r16(F.gelu(F.linear(z, d64(w1), d64(b1))))
+    yt = F.linear(h, d64(w2), d64(b2))
+    # fp16 rounding can flip on ~1e-16 differences between the two fp64 evaluations: allow one fp16
+    # ulp of an intermediate, propagated (tiny next to the GPU tolerance)
+    np.testing.assert_allclose(y, yt.numpy(), atol=2e-3, rtol=0)
+    assert np.abs(y - yt.numpy()).mean() < 1e-6

@@ -228,3 +228,49 @@ def make_gemm_inputs(m: int, n: int, k: int, seed: int = SEED, cfg_id: int = 7):
     b = r(2).uniform(-1, 1, n).astype(np.float32)
     td = torch.float16
     return _round(a, td), _round(w, td), _round(b, td)
+
+
+@dataclass(frozen=True)
+class LayerConfig:
+    """Synthetic Transformer layer: packed tokens of num_seqs sequences."""
+    name: str
+    cfg_id: int
+    num_seqs: int
+    seq_len: int          # every sequence's length (equal lengths) unless lengths are passed
+    d_model: int
+    heads: int
+    d_ff: int
+    causal: bool = False
+
+    @property
+    def head_dim(self) -> int:
+        return self.d_model // self.heads
+
+    @property
+    def scale(self) -> float:
+        return float(np.float32(1.0 / np.sqrt(self.head_dim)))
+
+    def with_(self, **kw) -> "LayerConfig":
+        return replace(self, **kw)
+
+
+# BERT-large layer at BASELINE.json config 5's token count: 32 sequences x 512 tokens = 16384 tokens,
+# d_model 1024, 16 heads (D = 64), d_ff 4096 (BJ configs 3 and 5)
+LAYER_CONFIGS = {
+    "bert_layer": LayerConfig("bert_layer", 10, 32, 512, 1024, 16, 4096),
+}
+
+
+def make_layer_inputs(cfg: LayerConfig, lengths=None, seed: int = SEED):
+    """Returns (x, wqkv, bqkv, wo, bo, w1, b1, w2, b2) fp16 CPU tensors and cu_seqlens (int32 numpy).
+    x ~ U(-1, 1) [T, d]; every W ~ N(0, 1/fan_in) in nn.Linear layout [out, in]; biases ~ U(-1, 1)."""
+    lens = np.full(cfg.num_seqs, cfg.seq_len, dtype=np.int64) if lengths is None else np.asarray(lengths)
+    cu = np.zeros(len(lens) + 1, dtype=np.int32)
+    cu[1:] = np.cumsum(lens)
+    t, d, f = int(cu[-1]), cfg.d_model, cfg.d_ff
+    r = lambda tid: _rng(cfg.cfg_id, tid, 0, 0, seed)
+    w = lambda tid, o, i: (r(tid).standard_normal((o, i), dtype=np.float32) / np.sqrt(i)).astype(np.float32)
+    b = lambda tid, o: r(tid).uniform(-1, 1, o).astype(np.float32)
+    arrs = [r(0).uniform(-1, 1, (t, d)).astype(np.float32), w(1, 3 * d, d), b(2, 3 * d), w(3, d, d), b(4, d),
+            w(5, f, d), b(6, f), w(7, d, f), b(8, d)]
+    return tuple(_round(a, torch.float16) for a in arrs), cu
