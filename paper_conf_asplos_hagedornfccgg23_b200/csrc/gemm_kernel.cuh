@@ -14,6 +14,7 @@
 #pragma once
 #include <cstdio>
 #include <cstring>
+#include <algorithm>
 
 #include "sm100.cuh"
 
@@ -22,12 +23,35 @@ namespace b200 {
 struct GemmParams {
   CUtensorMap tmA;  // {K, M, 1} box {64, 128, 1}
   CUtensorMap tmW;  // {K, N, 1} box {64, 256, 1}
+  CUtensorMap tmW2;  // {K, N, 1} box {64, 128, 1} (half tiles)
   CUtensorMap tmC;  // {N, M, 1} box {64, 128, 1}
   const __half* bias;
   int M, N, K;
   int act;
   int tiles_m, tiles_n;
+  // Work units: big tiles u < split_from are 128 x 256 (u / tiles_n, u % tiles_n); the last
+  // (num_units - split_from) / 2 big tiles are split into two 128 x 128 half tiles each, so a last
+  // wave that would hold r <= G/2 big tiles holds 2r half tiles instead and takes half as long.
+  int split_from, num_units;
 };
+
+struct GemmUnit {
+  int m0, n0, width;  // output rows m0.., columns n0..n0+width-1 (width 256 or 128)
+};
+__device__ __forceinline__ GemmUnit gemm_unit(const GemmParams& p, int u) {
+  GemmUnit g;
+  if (u < p.split_from) {
+    g.m0 = (u / p.tiles_n) * 128;
+    g.n0 = (u % p.tiles_n) * 256;
+    g.width = 256;
+  } else {
+    const int h = u - p.split_from, b = p.split_from + (h >> 1);
+    g.m0 = (b / p.tiles_n) * 128;
+    g.n0 = (b % p.tiles_n) * 256 + (h & 1) * 128;
+    g.width = 128;
+  }
+  return g;
+}
 
 struct GemmCfg {
   static constexpr int BM = 128, BN = 256, BK = 64;
@@ -47,10 +71,30 @@ struct GemmCfg {
   static_assert(SMEM_ALLOC <= 232448, "shared memory budget");
 };
 
+// GELU_erf(x) = x * Phi(x), Phi(x) = 0.5 * (1 + erf(x / sqrt 2)).  erf by Abramowitz & Stegun 7.1.26
+// (|error| <= 1.5e-7): for z = |x| / sqrt 2, 1 - erf(z) = t (a1 + t (a2 + t (a3 + t (a4 + t a5)))) e^(-z^2),
+// t = 1 / (1 + p z).  q = (1 - erf(z)) / 2 gives Phi = q for x < 0 (no cancellation) and 1 - q for
+// x >= 0.  Branch-free: one MUFU.RCP, one MUFU.EX2 and ~12 FMA-pipe ops per element, against ~25
+// instructions and a divergent branch for erff; the approximate rcp/ex2 add < 1e-6 relative, far
+// below the fp16 output rounding (R15 tolerance).
+__device__ __forceinline__ float gelu_erf_fast(float x) {
+  const float z = fabsf(x) * 0.70710678118654752f;
+  float t;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(t) : "f"(fmaf(0.3275911f, z, 1.f)));
+  float poly = fmaf(t, 1.061405429f, -1.453152027f);
+  poly = fmaf(t, poly, 1.421413741f);
+  poly = fmaf(t, poly, -0.284496736f);
+  poly = fmaf(t, poly, 0.254829592f);
+  poly *= t;
+  const float e = ex2(-1.4426950408889634f * z * z);
+  const float q = 0.5f * poly * e;
+  return x * (x < 0.f ? q : 1.f - q);
+}
+
 template <int ACT>
 __device__ __forceinline__ float apply_act(float x) {
   if (ACT == 1) return fmaxf(x, 0.f);
-  if (ACT == 2) return 0.5f * x * (1.f + erff(x * 0.70710678118654752f));
+  if (ACT == 2) return gelu_erf_fast(x);
   if (ACT == 3) return 0.5f * x * (1.f + tanhf(0.7978845608028654f * (x + 0.044715f * x * x * x)));
   return x;
 }
@@ -68,7 +112,7 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(smem + C::OFF_TMEMPTR);
   const int warp = warp_id(), lane = lane_id();
   const int nk = (p.K + C::BK - 1) / C::BK;
-  const int num_tiles = p.tiles_m * p.tiles_n;
+  const int num_tiles = p.num_units;
 
   if (threadIdx.x == 0) {
     if (sbase & 1023u) __trap();
@@ -85,6 +129,7 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&p.tmA);
     tma_prefetch_desc(&p.tmW);
+    tma_prefetch_desc(&p.tmW2);
     tma_prefetch_desc(&p.tmC);
   }
   if (warp == 1) {
@@ -101,19 +146,21 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
     uint32_t it = 0;
     const uint64_t keep = policy_evict_last();  // A rows and W are re-read by other tiles (all fit in L2)
     for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
-      const int m0 = (tile / p.tiles_n) * C::BM, n0 = (tile % p.tiles_n) * C::BN;
+      const GemmUnit g = gemm_unit(p, tile);
+      const bool half = g.width == 128;
       for (int kb = 0; kb < nk; ++kb, ++it) {
         const int s = it % C::STAGES;
         mbar_wait(EMPTY(s), ((it / C::STAGES) & 1) ^ 1);
-        mbar_arrive_expect_tx_elect(FULL(s), C::STAGE_BYTES);
+        mbar_arrive_expect_tx_elect(FULL(s), half ? C::A_BYTES + C::B_BYTES / 2 : C::STAGE_BYTES);
         const uint32_t sA = sbase + s * C::STAGE_BYTES;
-        tma_load_3d_hint_elect(sA, &p.tmA, FULL(s), kb * C::BK, m0, 0, keep);
-        tma_load_3d_hint_elect(sA + C::A_BYTES, &p.tmW, FULL(s), kb * C::BK, n0, 0, keep);
+        tma_load_3d_hint_elect(sA, &p.tmA, FULL(s), kb * C::BK, g.m0, 0, keep);
+        tma_load_3d_hint_elect(sA + C::A_BYTES, half ? &p.tmW2 : &p.tmW, FULL(s), kb * C::BK, g.n0, 0, keep);
       }
     }
   } else if (warp == 1) {
     // ---------------------------------------------------------------- MMA issuer
     constexpr uint32_t IDESC = idesc_f16(false, C::BM, C::BN, false, false);
+    constexpr uint32_t IDESC_HALF = idesc_f16(false, C::BM, C::BN / 2, false, false);
     const uint64_t desc0 = sdesc_sw128(sbase, 16, 1024);
     uint32_t it = 0, tc = 0;
     for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++tc) {
@@ -121,6 +168,7 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
       mbar_wait(ACC_EMPTY(b), ((tc >> 1) & 1) ^ 1);  // epilogue drained this accumulator
       tc_fence_after();
       const uint32_t tacc = tmem + 256 * b;
+      const uint32_t idesc = tile < p.split_from ? IDESC : IDESC_HALF;
       for (int kb = 0; kb < nk; ++kb, ++it) {
         const int s = it % C::STAGES;
         mbar_wait(FULL(s), (it / C::STAGES) & 1);
@@ -128,7 +176,7 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
         const uint32_t aoff = s * C::STAGE_BYTES, boff = aoff + C::A_BYTES;
 #pragma unroll
         for (int kk = 0; kk < C::BK / 16; ++kk)
-          umma_ss_elect(tacc, desc0 + ((aoff + kk * 32) >> 4), desc0 + ((boff + kk * 32) >> 4), IDESC,
+          umma_ss_elect(tacc, desc0 + ((aoff + kk * 32) >> 4), desc0 + ((boff + kk * 32) >> 4), idesc,
                         (kb > 0 || kk > 0));
         umma_commit_elect(EMPTY(s));
       }
@@ -142,7 +190,9 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
     const uint32_t bar_id = 1 + g;  // named barrier per column half (128 threads)
     uint32_t tc = 0;
     for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++tc) {
-      const int m0 = (tile / p.tiles_n) * C::BM, n0 = (tile % p.tiles_n) * C::BN;
+      const GemmUnit gu = gemm_unit(p, tile);
+      const int m0 = gu.m0, n0 = gu.n0;
+      const bool active = 128 * g < gu.width;  // half tiles: column group 1 has nothing to store
       const int b = tc & 1;
       mbar_wait(ACC_FULL(b), (tc >> 1) & 1);
       tc_fence_after();
@@ -150,7 +200,7 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
       named_bar_sync(bar_id, 128);
       const uint32_t tacc = tmem + lane_off + 256 * b + 128 * g;
 #pragma unroll 1
-      for (int q = 0; q < 4; ++q) {
+      for (int q = 0; q < (active ? 4 : 0); ++q) {
         uint32_t v[32];
         tmem_ld_32x32b_x32(tacc + 32 * q, v);
         tmem_wait_ld();
@@ -188,7 +238,7 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
       mbar_arrive(ACC_EMPTY(b));
       fence_proxy_async_smem();
       named_bar_sync(bar_id, 128);
-      if (row == 0) {
+      if (row == 0 && active) {
 #pragma unroll
         for (int c = 2 * g; c < 2 * g + 2; ++c)
           if (n0 + c * 64 < p.N) tma_store_3d(&p.tmC, sbase + C::OFF_STG + c * C::C_BOX, n0 + c * 64, m0, 0);
@@ -205,6 +255,191 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
   }
 }
 
+// ------------------------------------------------------------------------------------------------
+// CTA-pair variant (cta_group::2): a cluster of two CTAs on one TPC computes a 256 x 256 output
+// tile.  CTA r loads A rows m0 + 128 r .. (its half of M) and W rows n0 + 128 r .. (its half of N);
+// the leader (r = 0) issues tcgen05.mma.cta_group::2 M=256 N=256 K=16, which reads both CTAs' smem
+// and leaves rows 128 r .. of the accumulator in CTA r's TMEM.  Per SM and 64-deep K block that is
+// 32 KB of operand traffic for 512 MMA cycles, against 48 KB for the single-CTA 128 x 256 tile: the
+// L2 -> SMEM feed, not the tensor core, bounds the single-CTA kernel on the MLP shapes.
+//   FULL[s]      leader only, count 1 (its arrive.expect_tx of both CTAs' bytes); both CTAs' TMA
+//                loads complete_tx on it
+//   EMPTY[s]     both CTAs, count 1: the leader's MMA commit is multicast to both
+//   ACC_FULL[b]  both CTAs, count 1: multicast commit after a tile's last MMA
+//   ACC_EMPTY[b] leader only, count 16: one arrival per epilogue warp of either CTA (remote for r = 1)
+struct Gemm2Cfg {
+  static constexpr int BM = 128, BN = 128, BK = 64;  // per CTA: A 128 x 64, W 128 x 64 per stage
+#ifndef GEMM2_STAGES
+#define GEMM2_STAGES 5
+#endif
+  static constexpr int STAGES = GEMM2_STAGES;
+  static constexpr int A_BYTES = BM * BK * 2;  // 16 KB
+  static constexpr int B_BYTES = BN * BK * 2;  // 16 KB
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int C_BOX = 128 * 64 * 2;
+  static constexpr int OFF_STG = STAGES * STAGE_BYTES;
+  static constexpr int OFF_BAR = OFF_STG + 4 * C_BOX;
+  static constexpr int NUM_BARS = 2 * STAGES + 4;
+  static constexpr int OFF_TMEMPTR = OFF_BAR + NUM_BARS * 8;
+  static constexpr int SMEM_ALLOC = OFF_TMEMPTR + 16;
+  static constexpr int THREADS = 384;
+  static_assert(SMEM_ALLOC <= 232448, "shared memory budget");
+};
+
+template <int ACT>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_act_2sm_kernel(const __grid_constant__ GemmParams p) {
+  using C = Gemm2Cfg;
+  extern __shared__ __align__(1024) uint8_t smem[];
+  const uint32_t sbase = smem_u32(smem);
+  const uint32_t bar = sbase + C::OFF_BAR;
+  auto FULL = [&](int s) { return bar + 8 * s; };
+  auto EMPTY = [&](int s) { return bar + 8 * (C::STAGES + s); };
+  auto ACC_FULL = [&](int b) { return bar + 8 * (2 * C::STAGES + b); };
+  auto ACC_EMPTY = [&](int b) { return bar + 8 * (2 * C::STAGES + 2 + b); };
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(smem + C::OFF_TMEMPTR);
+  const int warp = warp_id(), lane = lane_id();
+  const uint32_t rank = cluster_ctarank();
+  const int nk = (p.K + C::BK - 1) / C::BK;
+  const int num_tiles = p.num_units;                  // 256 x 256 tiles
+  const int cid = blockIdx.x >> 1, ncl = gridDim.x >> 1;
+
+  if (threadIdx.x == 0) {
+    if (sbase & 1023u) __trap();
+    for (int s = 0; s < C::STAGES; ++s) {
+      mbar_init(FULL(s), 1);
+      mbar_init(EMPTY(s), 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(ACC_FULL(b), 1);
+      mbar_init(ACC_EMPTY(b), 16);
+    }
+    fence_mbar_init();
+  }
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&p.tmA);
+    tma_prefetch_desc(&p.tmW2);
+    tma_prefetch_desc(&p.tmC);
+  }
+  if (warp == 1) tmem_alloc_2sm(smem_u32(tmem_holder), 512);
+  tc_fence_before();
+  cluster_sync_all();  // both CTAs' barriers initialised and TMEM allocated before any signal crosses
+  tc_fence_after();
+  const uint32_t tmem = *tmem_holder;
+  if (warp == 1) tmem_relinquish_2sm();
+
+  if (warp == 0) {
+    // ---------------------------------------------------------------- TMA producer (both CTAs)
+    uint32_t it = 0;
+    const uint64_t keep = policy_evict_last();
+    for (int tile = cid; tile < num_tiles; tile += ncl) {
+      const int m0 = (tile / p.tiles_n) * 256, n0 = (tile % p.tiles_n) * 256;
+      for (int kb = 0; kb < nk; ++kb, ++it) {
+        const int s = it % C::STAGES;
+        mbar_wait(EMPTY(s), ((it / C::STAGES) & 1) ^ 1);
+        if (rank == 0) mbar_arrive_expect_tx_elect(FULL(s), 2 * C::STAGE_BYTES);
+        const uint32_t sA = sbase + s * C::STAGE_BYTES;
+        const uint32_t full_leader = mapa_shared(FULL(s), 0);
+        tma_load_3d_2sm_elect(sA, &p.tmA, full_leader, kb * C::BK, m0 + 128 * rank, 0, keep);
+        tma_load_3d_2sm_elect(sA + C::A_BYTES, &p.tmW2, full_leader, kb * C::BK, n0 + 128 * rank, 0, keep);
+      }
+    }
+  } else if (warp == 1) {
+    // ---------------------------------------------------------------- MMA issuer (leader only)
+    if (rank == 0) {
+      constexpr uint32_t IDESC = idesc_f16(false, 256, 256, false, false);
+      const uint64_t desc0 = sdesc_sw128(sbase, 16, 1024);
+      uint32_t it = 0, tc = 0;
+      for (int tile = cid; tile < num_tiles; tile += ncl, ++tc) {
+        const int b = tc & 1;
+        mbar_wait(ACC_EMPTY(b), ((tc >> 1) & 1) ^ 1);  // both CTAs' epilogues drained this accumulator
+        tc_fence_after();
+        const uint32_t tacc = tmem + 256 * b;
+        for (int kb = 0; kb < nk; ++kb, ++it) {
+          const int s = it % C::STAGES;
+          mbar_wait(FULL(s), (it / C::STAGES) & 1);
+          tc_fence_after();
+          const uint32_t aoff = s * C::STAGE_BYTES, boff = aoff + C::A_BYTES;
+#pragma unroll
+          for (int kk = 0; kk < C::BK / 16; ++kk)
+            umma_ss_2sm_elect(tacc, desc0 + ((aoff + kk * 32) >> 4), desc0 + ((boff + kk * 32) >> 4), IDESC,
+                              (kb > 0 || kk > 0));
+          umma_commit_2sm_mc_elect(EMPTY(s));
+        }
+        umma_commit_2sm_mc_elect(ACC_FULL(b));
+      }
+    }
+  } else if (warp >= 4) {
+    // ---------------------------------------------------------------- epilogue (both CTAs)
+    const int g = (warp - 4) >> 2, quad = warp & 3;
+    const int row = quad * 32 + lane;
+    const uint32_t lane_off = static_cast<uint32_t>(quad * 32) << 16;
+    const uint32_t bar_id = 1 + g;
+    uint32_t tc = 0;
+    for (int tile = cid; tile < num_tiles; tile += ncl, ++tc) {
+      const int m0 = (tile / p.tiles_n) * 256 + 128 * static_cast<int>(rank), n0 = (tile % p.tiles_n) * 256;
+      const int b = tc & 1;
+      mbar_wait(ACC_FULL(b), (tc >> 1) & 1);
+      tc_fence_after();
+      if (row == 0) tma_store_wait_read0();
+      named_bar_sync(bar_id, 128);
+      const uint32_t tacc = tmem + lane_off + 256 * b + 128 * g;
+#pragma unroll 1
+      for (int q = 0; q < 4; ++q) {
+        uint32_t v[32];
+        tmem_ld_32x32b_x32(tacc + 32 * q, v);
+        tmem_wait_ld();
+        reg_fence(v);
+        const int col0 = 128 * g + 32 * q;
+        float bv[32];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int n = n0 + col0 + 8 * u;
+          uint4 raw = make_uint4(0u, 0u, 0u, 0u);
+          if (p.bias && n < p.N) raw = __ldg(reinterpret_cast<const uint4*>(p.bias + n));
+          const __half2* h2 = reinterpret_cast<const __half2*>(&raw);
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const float2 f2 = __half22float2(h2[e]);
+            bv[8 * u + 2 * e] = f2.x;
+            bv[8 * u + 2 * e + 1] = f2.y;
+          }
+        }
+        float f[32];
+#pragma unroll
+        for (int k = 0; k < 32; ++k) f[k] = apply_act<ACT>(__uint_as_float(v[k]) + bv[k]);
+        const uint32_t box = sbase + C::OFF_STG + (col0 / 64) * C::C_BOX + row * 128;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int unit = ((col0 % 64) / 8) + u;
+          st_shared_v4(box + ((unit ^ (row & 7)) << 4), pack2<false>(f[8 * u + 0], f[8 * u + 1]),
+                       pack2<false>(f[8 * u + 2], f[8 * u + 3]), pack2<false>(f[8 * u + 4], f[8 * u + 5]),
+                       pack2<false>(f[8 * u + 6], f[8 * u + 7]));
+        }
+      }
+      // this warp's accumulator reads are done: one arrival per warp on the leader's ACC_EMPTY
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive_cluster(mapa_shared(ACC_EMPTY(b), 0));
+      fence_proxy_async_smem();
+      named_bar_sync(bar_id, 128);
+      if (row == 0) {
+#pragma unroll
+        for (int c = 2 * g; c < 2 * g + 2; ++c)
+          if (n0 + c * 64 < p.N && m0 < p.M)
+            tma_store_3d(&p.tmC, sbase + C::OFF_STG + c * C::C_BOX, n0 + c * 64, m0, 0);
+        tma_store_commit();
+      }
+    }
+    if (row == 0) tma_store_wait0();
+  }
+  tc_fence_before();
+  cluster_sync_all();  // the peer's last MMA-side signals and TMEM reads are done before dealloc
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc_2sm(tmem, 512);
+  }
+}
+
 // Host launcher (defined here so the ABI file stays thin).
 int make_map_2d_rows(CUtensorMap* m, const void* base, uint64_t cols, uint64_t rows, uint32_t box_rows,
                      char* err, size_t errlen);
@@ -216,6 +451,7 @@ inline int launch_gemm_bias_act(const void* A, const void* W, const void* bias, 
   int st;
   if ((st = make_map_2d_rows(&prm.tmA, A, K, M, GemmCfg::BM, err, errlen)) != 0) return st;
   if ((st = make_map_2d_rows(&prm.tmW, W, K, N, GemmCfg::BN, err, errlen)) != 0) return st;
+  if ((st = make_map_2d_rows(&prm.tmW2, W, K, N, GemmCfg::BN / 2, err, errlen)) != 0) return st;
   if ((st = make_map_2d_rows(&prm.tmC, Cm, N, M, GemmCfg::BM, err, errlen)) != 0) return st;
   prm.bias = static_cast<const __half*>(bias);
   prm.M = M;
@@ -224,6 +460,40 @@ inline int launch_gemm_bias_act(const void* A, const void* W, const void* bias, 
   prm.act = act;
   prm.tiles_m = (M + GemmCfg::BM - 1) / GemmCfg::BM;
   prm.tiles_n = (N + GemmCfg::BN - 1) / GemmCfg::BN;
+  // CTA-pair kernel for problems with at least one 256 x 256 tile per pair of SMs
+  const long long pair_tiles = static_cast<long long>((M + 255) / 256) * ((N + 255) / 256);
+  bool two_sm = pair_tiles >= sms / 2 && sms >= 2;
+#ifdef GEMM_FORCE_1SM
+  two_sm = false;
+#endif
+  if (two_sm) {
+    prm.tiles_m = (M + 255) / 256;
+    prm.tiles_n = (N + 255) / 256;
+    prm.split_from = prm.num_units = static_cast<int>(pair_tiles);
+    void (*k2)(GemmParams) = act == 1 ? gemm_bias_act_2sm_kernel<1>
+                            : act == 2 ? gemm_bias_act_2sm_kernel<2>
+                            : act == 3 ? gemm_bias_act_2sm_kernel<3>
+                                       : gemm_bias_act_2sm_kernel<0>;
+    static bool attr2[64][4];
+    int dev2 = 0;
+    cudaGetDevice(&dev2);
+    if (dev2 >= 64 || !attr2[dev2][act]) {
+      cudaError_t e = cudaFuncSetAttribute(k2, cudaFuncAttributeMaxDynamicSharedMemorySize, Gemm2Cfg::SMEM_ALLOC);
+      if (e != cudaSuccess) {
+        snprintf(err, errlen, "cudaFuncSetAttribute(gemm2sm): %s", cudaGetErrorString(e));
+        return 4;
+      }
+      if (dev2 < 64) attr2[dev2][act] = true;
+    }
+    const long long clusters = std::min<long long>(pair_tiles, sms / 2);
+    k2<<<static_cast<unsigned>(2 * clusters), Gemm2Cfg::THREADS, Gemm2Cfg::SMEM_ALLOC, stream>>>(prm);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) {
+      snprintf(err, errlen, "gemm_bias_act_2sm_kernel launch: %s", cudaGetErrorString(e));
+      return 4;
+    }
+    return 0;
+  }
   void (*kern)(GemmParams) = act == 1 ? gemm_bias_act_kernel<1>
                             : act == 2 ? gemm_bias_act_kernel<2>
                             : act == 3 ? gemm_bias_act_kernel<3>
@@ -240,6 +510,11 @@ inline int launch_gemm_bias_act(const void* A, const void* W, const void* bias, 
     if (dev < 64) attr_done[dev][act] = true;
   }
   const long long tiles = static_cast<long long>(prm.tiles_m) * prm.tiles_n;
+  const long long r = tiles > sms ? tiles % sms : 0;  // big tiles in the last, partial wave
+  const long long split = (r > 0 && 2 * r <= sms) ? r : 0;
+  if (tiles + split > 2147483647LL) return 2;
+  prm.split_from = static_cast<int>(tiles - split);
+  prm.num_units = static_cast<int>(tiles + split);
   dim3 grid(static_cast<unsigned>(tiles < sms ? tiles : sms), 1, 1);
   kern<<<grid, GemmCfg::THREADS, GemmCfg::SMEM_ALLOC, stream>>>(prm);
   cudaError_t e = cudaGetLastError();

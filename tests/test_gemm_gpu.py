@@ -50,3 +50,13 @@ def test_mlp_config_sampled_rows():
     # layer 2 checked on the GPU's own (rounded) H so the comparison isolates this GEMM
     hrows = h[torch.from_numpy(rows).to(DEV)].cpu()
     check(y[torch.from_numpy(rows).to(DEV)], gemm_bias_act_fp64(hrows, w2, b2, 0), "mlp layer 2")
+
+
+@pytest.mark.parametrize("m,n,k", [(19200, 512, 128), (16384, 1024, 256)])
+def test_gemm_tail_half_tiles(m, n, k):
+    """Shapes whose last wave of 128x256 tiles is at most half full run it as 128x128 half tiles
+    (GemmParams::split_from): (19200, 512) has 300 tiles = 2 waves + 4, (16384, 1024) 512 = 3 + 68."""
+    a, w, b = make_gemm_inputs(m, n, k)
+    c = fm.gemm_bias_act(a.to(DEV), w.to(DEV), b.to(DEV), act="gelu")
+    torch.cuda.synchronize()
+    check(c, gemm_bias_act_fp64(a, w, b, 2), f"{m}x{n}x{k} gelu (tail half tiles)")
