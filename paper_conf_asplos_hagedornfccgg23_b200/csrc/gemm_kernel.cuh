@@ -23,7 +23,8 @@ namespace b200 {
 struct GemmParams {
   CUtensorMap tmA;  // {K, M, 1} box {64, 128, 1}
   CUtensorMap tmW;  // {K, N, 1} box {64, 256, 1}
-  CUtensorMap tmW2;  // {K, N, 1} box {64, 128, 1} (half tiles)
+  CUtensorMap tmW2;  // {K, N, 1} box {64, 128, 1} (half tiles; the CTA-pair kernel's W half)
+  CUtensorMap tmW3;  // {K, N, 1} box {64, 64, 1}  (the CTA-pair kernel's half tiles)
   CUtensorMap tmC;  // {N, M, 1} box {64, 128, 1}
   const __half* bias;
   int M, N, K;
@@ -47,6 +48,21 @@ __device__ __forceinline__ GemmUnit gemm_unit(const GemmParams& p, int u) {
   } else {
     const int h = u - p.split_from, b = p.split_from + (h >> 1);
     g.m0 = (b / p.tiles_n) * 128;
+    g.n0 = (b % p.tiles_n) * 256 + (h & 1) * 128;
+    g.width = 128;
+  }
+  return g;
+}
+// the same for the CTA pair's 256 x 256 tiles (half tiles 256 x 128)
+__device__ __forceinline__ GemmUnit gemm_unit2(const GemmParams& p, int u) {
+  GemmUnit g;
+  if (u < p.split_from) {
+    g.m0 = (u / p.tiles_n) * 256;
+    g.n0 = (u % p.tiles_n) * 256;
+    g.width = 256;
+  } else {
+    const int h = u - p.split_from, b = p.split_from + (h >> 1);
+    g.m0 = (b / p.tiles_n) * 256;
     g.n0 = (b % p.tiles_n) * 256 + (h & 1) * 128;
     g.width = 128;
   }
@@ -332,21 +348,24 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
     uint32_t it = 0;
     const uint64_t keep = policy_evict_last();
     for (int tile = cid; tile < num_tiles; tile += ncl) {
-      const int m0 = (tile / p.tiles_n) * 256, n0 = (tile % p.tiles_n) * 256;
+      const GemmUnit gu = gemm_unit2(p, tile);
+      const bool half = gu.width == 128;  // N = 128 tile: 64 W rows per CTA
       for (int kb = 0; kb < nk; ++kb, ++it) {
         const int s = it % C::STAGES;
         mbar_wait(EMPTY(s), ((it / C::STAGES) & 1) ^ 1);
-        if (rank == 0) mbar_arrive_expect_tx_elect(FULL(s), 2 * C::STAGE_BYTES);
+        if (rank == 0) mbar_arrive_expect_tx_elect(FULL(s), 2 * (half ? C::A_BYTES + C::B_BYTES / 2 : C::STAGE_BYTES));
         const uint32_t sA = sbase + s * C::STAGE_BYTES;
         const uint32_t full_leader = mapa_shared(FULL(s), 0);
-        tma_load_3d_2sm_elect(sA, &p.tmA, full_leader, kb * C::BK, m0 + 128 * rank, 0, keep);
-        tma_load_3d_2sm_elect(sA + C::A_BYTES, &p.tmW2, full_leader, kb * C::BK, n0 + 128 * rank, 0, keep);
+        tma_load_3d_2sm_elect(sA, &p.tmA, full_leader, kb * C::BK, gu.m0 + 128 * rank, 0, keep);
+        tma_load_3d_2sm_elect(sA + C::A_BYTES, half ? &p.tmW3 : &p.tmW2, full_leader, kb * C::BK,
+                              gu.n0 + (half ? 64 : 128) * rank, 0, keep);
       }
     }
   } else if (warp == 1) {
     // ---------------------------------------------------------------- MMA issuer (leader only)
     if (rank == 0) {
       constexpr uint32_t IDESC = idesc_f16(false, 256, 256, false, false);
+      constexpr uint32_t IDESC_HALF = idesc_f16(false, 256, 128, false, false);
       const uint64_t desc0 = sdesc_sw128(sbase, 16, 1024);
       uint32_t it = 0, tc = 0;
       for (int tile = cid; tile < num_tiles; tile += ncl, ++tc) {
@@ -354,6 +373,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
         mbar_wait(ACC_EMPTY(b), ((tc >> 1) & 1) ^ 1);  // both CTAs' epilogues drained this accumulator
         tc_fence_after();
         const uint32_t tacc = tmem + 256 * b;
+        const uint32_t idesc = tile < p.split_from ? IDESC : IDESC_HALF;
         for (int kb = 0; kb < nk; ++kb, ++it) {
           const int s = it % C::STAGES;
           mbar_wait(FULL(s), (it / C::STAGES) & 1);
@@ -361,7 +381,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
           const uint32_t aoff = s * C::STAGE_BYTES, boff = aoff + C::A_BYTES;
 #pragma unroll
           for (int kk = 0; kk < C::BK / 16; ++kk)
-            umma_ss_2sm_elect(tacc, desc0 + ((aoff + kk * 32) >> 4), desc0 + ((boff + kk * 32) >> 4), IDESC,
+            umma_ss_2sm_elect(tacc, desc0 + ((aoff + kk * 32) >> 4), desc0 + ((boff + kk * 32) >> 4), idesc,
                               (kb > 0 || kk > 0));
           umma_commit_2sm_mc_elect(EMPTY(s));
         }
@@ -376,7 +396,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
     const uint32_t bar_id = 1 + g;
     uint32_t tc = 0;
     for (int tile = cid; tile < num_tiles; tile += ncl, ++tc) {
-      const int m0 = (tile / p.tiles_n) * 256 + 128 * static_cast<int>(rank), n0 = (tile % p.tiles_n) * 256;
+      const GemmUnit gu = gemm_unit2(p, tile);
+      const int m0 = gu.m0 + 128 * static_cast<int>(rank), n0 = gu.n0;
+      const bool active = 128 * g < gu.width;  // half tiles: column group 1 has nothing to store
       const int b = tc & 1;
       mbar_wait(ACC_FULL(b), (tc >> 1) & 1);
       tc_fence_after();
@@ -384,7 +406,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
       named_bar_sync(bar_id, 128);
       const uint32_t tacc = tmem + lane_off + 256 * b + 128 * g;
 #pragma unroll 1
-      for (int q = 0; q < 4; ++q) {
+      for (int q = 0; q < (active ? 4 : 0); ++q) {
         uint32_t v[32];
         tmem_ld_32x32b_x32(tacc + 32 * q, v);
         tmem_wait_ld();
@@ -422,7 +444,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
       if (lane == 0) mbar_arrive_cluster(mapa_shared(ACC_EMPTY(b), 0));
       fence_proxy_async_smem();
       named_bar_sync(bar_id, 128);
-      if (row == 0) {
+      if (row == 0 && active) {
 #pragma unroll
         for (int c = 2 * g; c < 2 * g + 2; ++c)
           if (n0 + c * 64 < p.N && m0 < p.M)
@@ -469,7 +491,12 @@ inline int launch_gemm_bias_act(const void* A, const void* W, const void* bias, 
   if (two_sm) {
     prm.tiles_m = (M + 255) / 256;
     prm.tiles_n = (N + 255) / 256;
-    prm.split_from = prm.num_units = static_cast<int>(pair_tiles);
+    const long long ncl = std::min<long long>(pair_tiles, sms / 2);
+    const long long r2 = pair_tiles > ncl ? pair_tiles % ncl : 0;  // tiles in the last, partial wave
+    const long long split2 = (r2 > 0 && 2 * r2 <= ncl) ? r2 : 0;
+    prm.split_from = static_cast<int>(pair_tiles - split2);
+    prm.num_units = static_cast<int>(pair_tiles + split2);
+    if ((st = make_map_2d_rows(&prm.tmW3, W, K, N, 64, err, errlen)) != 0) return st;
     void (*k2)(GemmParams) = act == 1 ? gemm_bias_act_2sm_kernel<1>
                             : act == 2 ? gemm_bias_act_2sm_kernel<2>
                             : act == 3 ? gemm_bias_act_2sm_kernel<3>
