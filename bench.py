@@ -114,6 +114,19 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
+def exp_roofline(pairs: float, ms_step: float, sampler) -> dict:
+    """Second roofline for the FMHA kernel: one exponential per visible (query, key)
+    pair against the MUFU ex2 rate, 16 per clock per SM (B300_MICROARCH / profiles/ubench.txt) x 148
+    SMs x the SM clock sampled during the timed region.  At D = 64 this unit, not the tensor core,
+    bounds the kernel; 2 of every 8 exp2 pairs run as FMA-pipe polynomials, so frac may exceed 1."""
+    mhz = (sampler.summary() or {}).get("sm_mhz") or 1965
+    peak = 148 * 16 * mhz * 1e6
+    achieved = pairs / (ms_step * 1e-3)
+    return {"bound": "alu", "unit": "Gexp/s", "achieved": round(achieved / 1e9, 1), "peak": round(peak / 1e9, 1),
+            "frac": round(achieved / peak, 4),
+            "peak_source": "MUFU.EX2 16/clk/SM x 148 SMs x sampled SM clock (derived, DESIGN.md §6)"}
+
+
 def cpu_oracle_sample(cfg, q, k, v, kv_len, budget_s: float):
     """Times the CPU oracle (as it stands) on whole (b,h) units of this workload until ~budget_s."""
     from oracle import attention_fp64
@@ -294,6 +307,7 @@ def main():
                          "frac": round(achieved / peak_burst, 4), "traffic": traffic,
                          "peak_source": f"{peak_src} bf16 dense burst (fp16 = bf16 rate)",
                          "kernel": "fmha_fwd_kernel"},
+            "roofline_exp": exp_roofline(alg_flops(cfg, kv_len) / (4.0 * cfg.head_dim), ms_step, sampler),
             "cpu_baseline": cpu,
             "check_max_abs_err": check_err,
         }

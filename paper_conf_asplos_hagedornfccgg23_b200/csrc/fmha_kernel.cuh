@@ -185,14 +185,17 @@ struct FmhaCfg {
 #ifndef FMHA_POLY_MOD
 #define FMHA_POLY_MOD 8
 #endif
-  static constexpr int POLY_MOD = FMHA_POLY_MOD, POLY_CNT = (D == 64) ? FMHA_POLY_CNT : 0;
+#ifndef FMHA_POLY_CNT128
+#define FMHA_POLY_CNT128 0
+#endif
+  static constexpr int POLY_MOD = FMHA_POLY_MOD, POLY_CNT = (D == 64) ? FMHA_POLY_CNT : FMHA_POLY_CNT128;
 #ifndef FMHA_POLY_MASK
 #define FMHA_POLY_MASK 0
 #endif
   // optional explicit 8-bit pattern over (pair index % 8); 0 = use POLY_MOD / POLY_CNT
   static constexpr unsigned POLY_MASK = FMHA_POLY_MASK;
   static __host__ __device__ constexpr bool poly_pair(int q) {
-    return D != 64 ? false : (POLY_MASK ? ((POLY_MASK >> (q % 8)) & 1u) != 0 : (q % POLY_MOD) < POLY_CNT);
+    return POLY_MASK && D == 64 ? ((POLY_MASK >> (q % 8)) & 1u) != 0 : (q % POLY_MOD) < POLY_CNT;
   }
   static_assert(8 * 32 * REG_SOFTMAX + 4 * 32 * REG_CORR + 4 * 32 * REG_MISC <= 128 * THREADS, "register pool");
   static_assert(SMEM_ALLOC <= 232448, "shared memory budget");
