@@ -156,7 +156,7 @@ def main():
     ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", default="bert_large_512", choices=sorted(CONFIGS) + sorted(VARLEN_CONFIGS) + sorted(LAYER_CONFIGS) + ["mlp"])
+    ap.add_argument("--workload", default="bert_large_512", choices=sorted(CONFIGS) + sorted(VARLEN_CONFIGS) + sorted(LAYER_CONFIGS) + ["mlp", "lstm_cell"])
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of CPU oracle timing")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -170,6 +170,8 @@ def main():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if args.workload == "mlp":
         return run_mlp(args, world, rank, local)
+    if args.workload == "lstm_cell":
+        return run_lstm(args, world, rank, local)
     if args.workload in VARLEN_CONFIGS:
         return run_varlen(args, world, rank, local)
     if args.workload in LAYER_CONFIGS:
@@ -680,6 +682,53 @@ def run_layer(args, world, rank, local):
         print(json.dumps(line), flush=True)
     if dist:
         dist.destroy_process_group()
+
+
+def run_lstm(args, world, rank, local):
+    """the paper's simplified LSTM cell (Fig. 12) as one
+    dual_gemm_bias_act launch per step: relu(X Wx^T + H Wh^T + b), tokens 16384, input = hidden = 1024,
+    4 gates (N = 4096).  The unfused torch composition (two cuBLAS GEMMs, add, ReLU) is timed beside it."""
+    import torch.nn.functional as F
+    import paper_conf_asplos_hagedornfccgg23_b200 as fm
+    from workloads import make_gemm_inputs
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    m, n, k1, k2 = 16384, 4096, 1024, 1024
+    x, wx, b = (t.to(dev) for t in make_gemm_inputs(m, n, k1, cfg_id=12))
+    h, wh, _ = (t.to(dev) for t in make_gemm_inputs(m, n, k2, cfg_id=13))
+    y = torch.empty((m, n), dtype=torch.float16, device=dev)
+    stream = torch.cuda.current_stream(dev)
+    step = lambda: fm.dual_gemm_bias_act(x, wx, h, wh, b, act="relu", out=y)
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    sampler = ClockSampler(local)
+    with sampler:
+        ms = _time_graph(step, args.steps, stream)
+    unfused = lambda: (F.linear(x, wx) + F.linear(h, wh, b)).relu_()
+    for _ in range(3):
+        unfused()
+    torch.cuda.synchronize()
+    torch_ms = _time_graph(unfused, args.steps, stream)
+    flops = 2.0 * m * n * (k1 + k2)
+    peak_burst, _, _, src = measured_peaks()
+    from oracle import dual_gemm_bias_act_fp64
+    rows = np.array([0, 1, m // 2, m - 1])
+    ref = dual_gemm_bias_act_fp64(x[rows].cpu(), wx.cpu(), h[rows].cpu(), wh.cpu(), b.cpu(), 1)
+    err = float(np.abs(y[torch.from_numpy(rows).to(dev)].double().cpu().numpy() - ref).max())
+    val = flops / (ms * 1e-3) / 1e12
+    if rank == 0:
+        print(json.dumps({
+            "metric": "simplified LSTM cell relu(X Wx^T + H Wh^T + b) TFLOP/s", "value": round(val, 2),
+            "unit": "TFLOP/s", "n_gpus": 1, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 5),
+            "higher_is_better": True, "dtype": "f16", "data": "synthetic",
+            "config": {"workload": "lstm_cell", "tokens": m, "input": k1, "hidden": k2, "gates_n": n},
+            "context_torch_unfused": {"ms_per_step": round(torch_ms, 5), "speedup": round(torch_ms / ms, 3),
+                                      "what": "F.linear + F.linear(+bias) + add + relu_ (cuBLAS + elementwise)"},
+            "clocks": sampler.summary(), "gpu_launches": args.steps,
+            "roofline": {"bound": "tensor", "achieved": round(val, 2), "peak": peak_burst, "unit": "TFLOP/s",
+                         "frac": round(val / peak_burst, 4), "peak_source": f"{src} bf16 dense burst"},
+            "check_max_abs_err": err}), flush=True)
 
 
 def run_reference(args, cfg, world, rank):

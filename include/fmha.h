@@ -115,10 +115,20 @@ FMHA_API int fmha_fwd_from_host(int dtype, const void* hQ, const void* hK, const
  * A [M,K], W [N,K] (nn.Linear layout), bias [N] (or NULL), C [M,N]: fp16, row-major, DEVICE,
  * 16-byte aligned; fp32 accumulation, bias and activation in fp32, one RNE rounding to fp16.
  * Requires K % 8 == 0 and N % 8 == 0 (16-byte row pitch for TMA).
- * act: 0 none, 1 ReLU, 2 GELU (erf), 3 GELU (tanh). */
-typedef enum { ACT_NONE = 0, ACT_RELU = 1, ACT_GELU_ERF = 2, ACT_GELU_TANH = 3 } fmha_act_t;
+ * act: 0 none, 1 ReLU, 2 GELU (erf), 3 GELU (tanh), 4 tanh. */
+typedef enum { ACT_NONE = 0, ACT_RELU = 1, ACT_GELU_ERF = 2, ACT_GELU_TANH = 3, ACT_TANH = 4 } fmha_act_t;
 FMHA_API int gemm_bias_act(const void* A, const void* W, const void* bias, void* C, int M, int N, int K, int act,
                   fmha_stream_t stream);
+
+/* Dual GEMM + bias + activation in one kernel: the paper's simplified LSTM cell (PAPER.md L471-L475,
+ * Fig. 12: "two independent GEMMs followed by an addition and two more pointwise operations"):
+ *     C[m,n] = act( sum_k A1[m,k] W1[n,k] + sum_k A2[m,k] W2[n,k] + bias[n] )
+ * A1 [M,K1], W1 [N,K1], A2 [M,K2], W2 [N,K2], bias [N] or NULL, C [M,N]; fp16, row-major, DEVICE,
+ * 16-byte aligned; both products accumulate into ONE fp32 accumulator (no intermediate tensor),
+ * then bias, activation (act as gemm_bias_act, plus 4 = tanh, the LSTM cell's usual activation)
+ * and one RNE rounding.  Requires K1, K2, N multiples of 8.  Errors as gemm_bias_act. */
+FMHA_API int dual_gemm_bias_act(const void* A1, const void* W1, const void* A2, const void* W2, const void* bias,
+                                void* C, int M, int N, int K1, int K2, int act, fmha_stream_t stream);
 
 /* End-to-end synthetic Transformer layer (the paper's end-to-end use of its
  * fused kernels), fp16, tokens packed as in fmha_fwd_varlen:

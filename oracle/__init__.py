@@ -20,7 +20,7 @@ Modules
 fmha   numpy fp64, unfused GEMM -> softmax -> GEMM per (batch, head);
        the same per (sequence, head) of a packed variable-length batch   [pinned]
 brute  pure-Python scalar loops with math.fsum, tiny shapes only        [pinned]
-gemm   numpy fp64 act(A @ W^T + b)                                      [pinned]
+gemm   numpy fp64 act(A @ W^T + b); act(A1 W1^T + A2 W2^T + b) (LSTM cell) [pinned]
 layer  QKV GEMM -> varlen FMHA -> out GEMM -> MLP, fp16 storage between  [pinned]
 
 Every function is pinned by ``tests/test_oracle.py`` against closed forms,
@@ -31,7 +31,7 @@ unpinned" function in this package.
 
 from .fmha import attention_fp64, attention_rows_fp64, attention_varlen_fp64, softmax_probs_fp64, fmha_flops
 from .brute import attention_brute
-from .gemm import gemm_bias_act_fp64, gelu_erf, gelu_tanh, relu
+from .gemm import dual_gemm_bias_act_fp64, gemm_bias_act_fp64, gelu_erf, gelu_tanh, relu
 from .layer import round_fp16, transformer_layer_fp64
 
 __all__ = [
@@ -42,6 +42,7 @@ __all__ = [
     "fmha_flops",
     "attention_brute",
     "gemm_bias_act_fp64",
+    "dual_gemm_bias_act_fp64",
     "gelu_erf",
     "gelu_tanh",
     "relu",

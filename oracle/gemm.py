@@ -19,7 +19,7 @@ import numpy as np
 
 from .fmha import _as_f64
 
-ACT_NONE, ACT_RELU, ACT_GELU_ERF, ACT_GELU_TANH = 0, 1, 2, 3
+ACT_NONE, ACT_RELU, ACT_GELU_ERF, ACT_GELU_TANH, ACT_TANH = 0, 1, 2, 3, 4
 
 
 def relu(x: np.ndarray) -> np.ndarray:
@@ -54,4 +54,32 @@ def gemm_bias_act_fp64(a, w, bias=None, act: int = ACT_NONE) -> np.ndarray:
         return gelu_erf(c)
     if act == ACT_GELU_TANH:
         return gelu_tanh(c)
+    if act == ACT_TANH:
+        return np.tanh(c)
+    raise ValueError(f"unknown act {act}")
+
+
+def dual_gemm_bias_act_fp64(a1, w1, a2, w2, bias=None, act: int = ACT_RELU) -> np.ndarray:
+    """The paper's simplified LSTM cell (Fig. 12): two independent GEMMs, their
+    addition, the bias addition and the activation -- act(A1 @ W1^T + A2 @ W2^T + b) -- in float64,
+    in the order the paper lists the nodes."""
+    g1 = _as_f64(a1) @ _as_f64(w1).T             # GEMM 1
+    g2 = _as_f64(a2) @ _as_f64(w2).T             # GEMM 2 (independent)
+    c = g1 + g2                                  # addition
+    if bias is not None:
+        c = c + _as_f64(bias)[None, :]           # pointwise bias
+    return _act(c, act)                          # activation
+
+
+def _act(c: np.ndarray, act: int) -> np.ndarray:
+    if act == ACT_NONE:
+        return c
+    if act == ACT_RELU:
+        return relu(c)
+    if act == ACT_GELU_ERF:
+        return gelu_erf(c)
+    if act == ACT_GELU_TANH:
+        return gelu_tanh(c)
+    if act == ACT_TANH:
+        return np.tanh(c)
     raise ValueError(f"unknown act {act}")

@@ -9,6 +9,7 @@ sm_100 device these functions raise.
     fmha_fwd_varlen(qkv, cu_seqlens, max_seqlen, causal=False, scale=None, out=None) -> O
     fmha_fwd_from_host(q, k, v, ..., workspace) -> O  (host tensors; copies inside the call)
     gemm_bias_act(a, w, bias=None, act="none", out=None) -> C
+    dual_gemm_bias_act(a1, w1, a2, w2, bias=None, act="relu", out=None) -> C  (simplified LSTM cell)
     transformer_layer(x, weights, cu_seqlens, max_seqlen, heads, ...) -> Y  (5 launches, one call)
 """
 
@@ -22,11 +23,11 @@ import torch
 from . import _lib
 from ._lib import FmhaError, FmhaMask
 
-__all__ = ["fmha_fwd", "fmha_fwd_varlen", "fmha_fwd_from_host", "gemm_bias_act", "transformer_layer", "layer_workspace_bytes", "workspace_bytes", "FmhaError",
+__all__ = ["fmha_fwd", "fmha_fwd_varlen", "fmha_fwd_from_host", "gemm_bias_act", "dual_gemm_bias_act", "transformer_layer", "layer_workspace_bytes", "workspace_bytes", "FmhaError",
            "MASK_NONE", "MASK_KEY_PADDING", "MASK_CAUSAL", "ACTS", "version"]
 
 MASK_NONE, MASK_KEY_PADDING, MASK_CAUSAL = 0, 1, 2
-ACTS = {"none": 0, "relu": 1, "gelu": 2, "gelu_erf": 2, "gelu_tanh": 3}
+ACTS = {"none": 0, "relu": 1, "gelu": 2, "gelu_erf": 2, "gelu_tanh": 3, "tanh": 4}
 
 
 def version() -> str:
@@ -189,4 +190,27 @@ def transformer_layer(x: torch.Tensor, wqkv: torch.Tensor, bqkv, wo: torch.Tenso
                                    int(bool(causal)), workspace.data_ptr(),
                                    workspace.numel() * workspace.element_size(), _stream_ptr(x.device))
     _lib.check(st, "transformer_layer_fwd")
+    return out
+
+
+def dual_gemm_bias_act(a1: torch.Tensor, w1: torch.Tensor, a2: torch.Tensor, w2: torch.Tensor,
+                       bias: torch.Tensor | None = None, act: str = "relu",
+                       out: torch.Tensor | None = None) -> torch.Tensor:
+    """C = act(A1 W1^T + A2 W2^T + bias) in one kernel (the paper's simplified LSTM cell, Fig. 12):
+    a1 [M,K1], w1 [N,K1], a2 [M,K2], w2 [N,K2], bias [N]; fp16 CUDA tensors -> [M,N] fp16."""
+    lib = _lib.load()
+    ts = [a1, w1, a2, w2] + ([] if bias is None else [bias])
+    if any(t.dtype != torch.float16 or not t.is_cuda for t in ts):
+        raise TypeError("dual_gemm_bias_act takes fp16 CUDA tensors (no CPU fallback)")
+    a1, w1, a2, w2 = (t.contiguous() for t in (a1, w1, a2, w2))
+    m_, k1 = a1.shape
+    n_, k2 = w1.shape[0], a2.shape[1]
+    if w1.shape[1] != k1 or a2.shape[0] != m_ or w2.shape != (n_, k2):
+        raise ValueError("shape mismatch")
+    if out is None:
+        out = torch.empty((m_, n_), dtype=torch.float16, device=a1.device)
+    st = lib.dual_gemm_bias_act(a1.data_ptr(), w1.data_ptr(), a2.data_ptr(), w2.data_ptr(),
+                                None if bias is None else bias.contiguous().data_ptr(), out.data_ptr(),
+                                m_, n_, k1, k2, ACTS[act], _stream_ptr(a1.device))
+    _lib.check(st, "dual_gemm_bias_act")
     return out

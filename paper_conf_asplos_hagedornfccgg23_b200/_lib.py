@@ -31,6 +31,7 @@ EXPORTED_SYMBOLS = (
     "fmha_workspace_bytes",
     "fmha_fwd_from_host",
     "gemm_bias_act",
+    "dual_gemm_bias_act",
     "transformer_layer_workspace_bytes",
     "transformer_layer_fwd",
     "fmha_status_string",
@@ -78,6 +79,9 @@ def load() -> ctypes.CDLL:
     lib.fmha_fwd_from_host.restype = i32
     lib.gemm_bias_act.argtypes = [vp, vp, vp, vp, i32, i32, i32, i32, vp]
     lib.gemm_bias_act.restype = i32
+    if hasattr(lib, "dual_gemm_bias_act"):
+        lib.dual_gemm_bias_act.argtypes = [vp, vp, vp, vp, vp, vp, i32, i32, i32, i32, i32, vp]
+        lib.dual_gemm_bias_act.restype = i32
     if hasattr(lib, "transformer_layer_fwd"):  # absent only in old tuning builds
         lib.transformer_layer_workspace_bytes.argtypes = [i32, i32, i32]
         lib.transformer_layer_workspace_bytes.restype = sz

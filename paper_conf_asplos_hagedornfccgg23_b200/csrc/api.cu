@@ -379,7 +379,7 @@ int gemm_bias_act(const void* A, const void* W, const void* bias, void* Cm, int 
                   fmha_stream_t stream) {
   g_last_cuda_error[0] = 0;
   if (M < 0 || N < 0 || K < 0) return FMHA_ERR_INVALID_ARG;
-  if (act < ACT_NONE || act > ACT_GELU_TANH) return FMHA_ERR_UNSUPPORTED;
+  if (act < ACT_NONE || act > ACT_TANH) return FMHA_ERR_UNSUPPORTED;
   if (M == 0 || N == 0) return FMHA_OK;
   if (!A || !W || !Cm || K == 0) return FMHA_ERR_INVALID_ARG;
   if ((K % 8) != 0 || (N % 8) != 0) return FMHA_ERR_UNSUPPORTED;
@@ -387,8 +387,28 @@ int gemm_bias_act(const void* A, const void* W, const void* bias, void* Cm, int 
   int sms = 0;
   int st = check_device(&sms);
   if (st != FMHA_OK) return st;
-  return b200::launch_gemm_bias_act(A, W, bias, Cm, M, N, K, act, sms, reinterpret_cast<cudaStream_t>(stream),
-                                    g_last_cuda_error, sizeof(g_last_cuda_error));
+  return b200::launch_gemm_bias_act(A, W, nullptr, nullptr, bias, Cm, M, N, K, 0, act, sms,
+                                    reinterpret_cast<cudaStream_t>(stream), g_last_cuda_error,
+                                    sizeof(g_last_cuda_error));
+}
+
+int dual_gemm_bias_act(const void* A1, const void* W1, const void* A2, const void* W2, const void* bias, void* Cm,
+                       int M, int N, int K1, int K2, int act, fmha_stream_t stream) {
+  g_last_cuda_error[0] = 0;
+  if (M < 0 || N < 0 || K1 < 0 || K2 < 0) return FMHA_ERR_INVALID_ARG;
+  if (act < ACT_NONE || act > ACT_TANH) return FMHA_ERR_UNSUPPORTED;
+  if (M == 0 || N == 0) return FMHA_OK;
+  if (!A1 || !W1 || !A2 || !W2 || !Cm || K1 == 0 || K2 == 0) return FMHA_ERR_INVALID_ARG;
+  if ((K1 % 8) != 0 || (K2 % 8) != 0 || (N % 8) != 0) return FMHA_ERR_UNSUPPORTED;
+  if (!aligned16(A1) || !aligned16(W1) || !aligned16(A2) || !aligned16(W2) || !aligned16(Cm) ||
+      (bias && !aligned16(bias)))
+    return FMHA_ERR_MISALIGNED;
+  int sms = 0;
+  int st = check_device(&sms);
+  if (st != FMHA_OK) return st;
+  return b200::launch_gemm_bias_act(A1, W1, A2, W2, bias, Cm, M, N, K1, K2, act, sms,
+                                    reinterpret_cast<cudaStream_t>(stream), g_last_cuda_error,
+                                    sizeof(g_last_cuda_error));
 }
 
 const char* fmha_status_string(int status) {

@@ -21,13 +21,13 @@
 namespace b200 {
 
 struct GemmParams {
-  CUtensorMap tmA;  // {K, M, 1} box {64, 128, 1}
-  CUtensorMap tmW;  // {K, N, 1} box {64, 256, 1}
-  CUtensorMap tmW2;  // {K, N, 1} box {64, 128, 1} (half tiles; the CTA-pair kernel's W half)
-  CUtensorMap tmW3;  // {K, N, 1} box {64, 64, 1}  (the CTA-pair kernel's half tiles)
+  // Operand pair q (q = 1 only for the dual GEMM, K2 > 0): C = act(A_0 W_0^T + A_1 W_1^T + bias).
+  CUtensorMap tmA[2];     // A_q {K_q, M, 1} box {64, 128, 1}
+  CUtensorMap tmW[2][3];  // W_q {K_q, N, 1} boxes of {64, 256 | 128 | 64, 1} rows: single-CTA tile,
+                          // single-CTA half tile / CTA-pair W half, CTA-pair half tile
   CUtensorMap tmC;  // {N, M, 1} box {64, 128, 1}
   const __half* bias;
-  int M, N, K;
+  int M, N, K, K2;  // K2 = 0: a single GEMM
   int act;
   int tiles_m, tiles_n;
   // Work units: big tiles u < split_from are 128 x 256 (u / tiles_n, u % tiles_n); the last
@@ -112,6 +112,7 @@ __device__ __forceinline__ float apply_act(float x) {
   if (ACT == 1) return fmaxf(x, 0.f);
   if (ACT == 2) return gelu_erf_fast(x);
   if (ACT == 3) return 0.5f * x * (1.f + tanhf(0.7978845608028654f * (x + 0.044715f * x * x * x)));
+  if (ACT == 4) return tanhf(x);
   return x;
 }
 
@@ -127,7 +128,8 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
   auto ACC_EMPTY = [&](int b) { return bar + 8 * (2 * C::STAGES + 2 + b); };
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(smem + C::OFF_TMEMPTR);
   const int warp = warp_id(), lane = lane_id();
-  const int nk = (p.K + C::BK - 1) / C::BK;
+  const int nk1 = (p.K + C::BK - 1) / C::BK;
+  const int nk = nk1 + (p.K2 + C::BK - 1) / C::BK;
   const int num_tiles = p.num_units;
 
   if (threadIdx.x == 0) {
@@ -143,9 +145,9 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
     fence_mbar_init();
   }
   if (warp == 0 && lane == 0) {
-    tma_prefetch_desc(&p.tmA);
-    tma_prefetch_desc(&p.tmW);
-    tma_prefetch_desc(&p.tmW2);
+    tma_prefetch_desc(&p.tmA[0]);
+    tma_prefetch_desc(&p.tmW[0][0]);
+    tma_prefetch_desc(&p.tmW[0][1]);
     tma_prefetch_desc(&p.tmC);
   }
   if (warp == 1) {
@@ -169,8 +171,9 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
         mbar_wait(EMPTY(s), ((it / C::STAGES) & 1) ^ 1);
         mbar_arrive_expect_tx_elect(FULL(s), half ? C::A_BYTES + C::B_BYTES / 2 : C::STAGE_BYTES);
         const uint32_t sA = sbase + s * C::STAGE_BYTES;
-        tma_load_3d_hint_elect(sA, &p.tmA, FULL(s), kb * C::BK, g.m0, 0, keep);
-        tma_load_3d_hint_elect(sA + C::A_BYTES, half ? &p.tmW2 : &p.tmW, FULL(s), kb * C::BK, g.n0, 0, keep);
+        const int q = kb >= nk1, kq = (kb - (q ? nk1 : 0)) * C::BK;  // operand pair, its K offset
+        tma_load_3d_hint_elect(sA, &p.tmA[q], FULL(s), kq, g.m0, 0, keep);
+        tma_load_3d_hint_elect(sA + C::A_BYTES, &p.tmW[q][half ? 1 : 0], FULL(s), kq, g.n0, 0, keep);
       }
     }
   } else if (warp == 1) {
@@ -315,7 +318,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(smem + C::OFF_TMEMPTR);
   const int warp = warp_id(), lane = lane_id();
   const uint32_t rank = cluster_ctarank();
-  const int nk = (p.K + C::BK - 1) / C::BK;
+  const int nk1 = (p.K + C::BK - 1) / C::BK;
+  const int nk = nk1 + (p.K2 + C::BK - 1) / C::BK;
   const int num_tiles = p.num_units;                  // 256 x 256 tiles
   const int cid = blockIdx.x >> 1, ncl = gridDim.x >> 1;
 
@@ -332,8 +336,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
     fence_mbar_init();
   }
   if (warp == 0 && lane == 0) {
-    tma_prefetch_desc(&p.tmA);
-    tma_prefetch_desc(&p.tmW2);
+    tma_prefetch_desc(&p.tmA[0]);
+    tma_prefetch_desc(&p.tmW[0][1]);
     tma_prefetch_desc(&p.tmC);
   }
   if (warp == 1) tmem_alloc_2sm(smem_u32(tmem_holder), 512);
@@ -356,8 +360,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
         if (rank == 0) mbar_arrive_expect_tx_elect(FULL(s), 2 * (half ? C::A_BYTES + C::B_BYTES / 2 : C::STAGE_BYTES));
         const uint32_t sA = sbase + s * C::STAGE_BYTES;
         const uint32_t full_leader = mapa_shared(FULL(s), 0);
-        tma_load_3d_2sm_elect(sA, &p.tmA, full_leader, kb * C::BK, gu.m0 + 128 * rank, 0, keep);
-        tma_load_3d_2sm_elect(sA + C::A_BYTES, half ? &p.tmW3 : &p.tmW2, full_leader, kb * C::BK,
+        const int q = kb >= nk1, kq = (kb - (q ? nk1 : 0)) * C::BK;  // operand pair, its K offset
+        tma_load_3d_2sm_elect(sA, &p.tmA[q], full_leader, kq, gu.m0 + 128 * rank, 0, keep);
+        tma_load_3d_2sm_elect(sA + C::A_BYTES, &p.tmW[q][half ? 2 : 1], full_leader, kq,
                               gu.n0 + (half ? 64 : 128) * rank, 0, keep);
       }
     }
@@ -466,19 +471,27 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
 int make_map_2d_rows(CUtensorMap* m, const void* base, uint64_t cols, uint64_t rows, uint32_t box_rows,
                      char* err, size_t errlen);
 
-inline int launch_gemm_bias_act(const void* A, const void* W, const void* bias, void* Cm, int M, int N, int K,
-                                int act, int sms, cudaStream_t stream, char* err, size_t errlen) {
+// C = act(A W^T [+ A2 W2^T] + bias); A2 / W2 are used when K2 > 0 (the dual GEMM).
+inline int launch_gemm_bias_act(const void* A, const void* W, const void* A2, const void* W2, const void* bias,
+                                void* Cm, int M, int N, int K, int K2, int act, int sms, cudaStream_t stream,
+                                char* err, size_t errlen) {
   GemmParams prm;
   memset(&prm, 0, sizeof(prm));
   int st;
-  if ((st = make_map_2d_rows(&prm.tmA, A, K, M, GemmCfg::BM, err, errlen)) != 0) return st;
-  if ((st = make_map_2d_rows(&prm.tmW, W, K, N, GemmCfg::BN, err, errlen)) != 0) return st;
-  if ((st = make_map_2d_rows(&prm.tmW2, W, K, N, GemmCfg::BN / 2, err, errlen)) != 0) return st;
+  for (int q = 0; q < (K2 > 0 ? 2 : 1); ++q) {
+    const void* a = q ? A2 : A;
+    const void* w = q ? W2 : W;
+    const int kq = q ? K2 : K;
+    if ((st = make_map_2d_rows(&prm.tmA[q], a, kq, M, GemmCfg::BM, err, errlen)) != 0) return st;
+    for (int v = 0; v < 3; ++v)
+      if ((st = make_map_2d_rows(&prm.tmW[q][v], w, kq, N, 256 >> v, err, errlen)) != 0) return st;
+  }
   if ((st = make_map_2d_rows(&prm.tmC, Cm, N, M, GemmCfg::BM, err, errlen)) != 0) return st;
   prm.bias = static_cast<const __half*>(bias);
   prm.M = M;
   prm.N = N;
   prm.K = K;
+  prm.K2 = K2 > 0 ? K2 : 0;
   prm.act = act;
   prm.tiles_m = (M + GemmCfg::BM - 1) / GemmCfg::BM;
   prm.tiles_n = (N + GemmCfg::BN - 1) / GemmCfg::BN;
@@ -496,12 +509,12 @@ inline int launch_gemm_bias_act(const void* A, const void* W, const void* bias, 
     const long long split2 = (r2 > 0 && 2 * r2 <= ncl) ? r2 : 0;
     prm.split_from = static_cast<int>(pair_tiles - split2);
     prm.num_units = static_cast<int>(pair_tiles + split2);
-    if ((st = make_map_2d_rows(&prm.tmW3, W, K, N, 64, err, errlen)) != 0) return st;
     void (*k2)(GemmParams) = act == 1 ? gemm_bias_act_2sm_kernel<1>
                             : act == 2 ? gemm_bias_act_2sm_kernel<2>
                             : act == 3 ? gemm_bias_act_2sm_kernel<3>
+                            : act == 4 ? gemm_bias_act_2sm_kernel<4>
                                        : gemm_bias_act_2sm_kernel<0>;
-    static bool attr2[64][4];
+    static bool attr2[64][5];
     int dev2 = 0;
     cudaGetDevice(&dev2);
     if (dev2 >= 64 || !attr2[dev2][act]) {
@@ -524,8 +537,9 @@ inline int launch_gemm_bias_act(const void* A, const void* W, const void* bias, 
   void (*kern)(GemmParams) = act == 1 ? gemm_bias_act_kernel<1>
                             : act == 2 ? gemm_bias_act_kernel<2>
                             : act == 3 ? gemm_bias_act_kernel<3>
+                            : act == 4 ? gemm_bias_act_kernel<4>
                                        : gemm_bias_act_kernel<0>;
-  static bool attr_done[64][4];
+  static bool attr_done[64][5];
   int dev = 0;
   cudaGetDevice(&dev);
   if (dev >= 64 || !attr_done[dev][act]) {

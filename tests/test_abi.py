@@ -70,6 +70,12 @@ def test_validation_codes(lib):
     assert lib.gemm_bias_act(16, 16, None, 16, 4, 8, 12, 0, None) == 2  # K % 8
     assert lib.gemm_bias_act(16, 16, None, 16, 4, 8, 16, 9, None) == 2  # act
     assert lib.gemm_bias_act(16, 16, None, 16, 0, 8, 16, 0, None) == 0
+    dg = lib.dual_gemm_bias_act
+    assert dg(16, 16, 16, 16, None, 16, 4, 8, 16, 12, 1, None) == 2    # K2 % 8
+    assert dg(16, 16, 16, 16, None, 16, 4, 8, 16, 16, 5, None) == 2    # act
+    assert dg(16, 16, None, 16, None, 16, 4, 8, 16, 16, 1, None) == 1  # null A2
+    assert dg(16, 16, 24, 16, None, 16, 4, 8, 16, 16, 1, None) == 3    # misaligned
+    assert dg(16, 16, 16, 16, None, 16, 0, 8, 16, 16, 1, None) == 0    # M = 0
     # varlen: validation before any device access
     vl = lib.fmha_fwd_varlen
     assert vl(16, 16, 16, 2, 8, 16, 2, 96, 0.1, 0, 0, None) == 2       # head_dim

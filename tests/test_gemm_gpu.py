@@ -60,3 +60,16 @@ def test_gemm_tail_half_tiles(m, n, k):
     c = fm.gemm_bias_act(a.to(DEV), w.to(DEV), b.to(DEV), act="gelu")
     torch.cuda.synchronize()
     check(c, gemm_bias_act_fp64(a, w, b, 2), f"{m}x{n}x{k} gelu (tail half tiles)")
+
+
+@pytest.mark.parametrize("m,n,k1,k2", [(200, 136, 64, 96), (1000, 264, 1024, 72), (4096, 1024, 512, 256)])
+@pytest.mark.parametrize("act", ["relu", "tanh", "none"])
+def test_dual_gemm_parity(m, n, k1, k2, act):
+    """The simplified LSTM cell: both products in one accumulator (single-CTA and CTA-pair kernels)."""
+    from oracle import dual_gemm_bias_act_fp64
+    a1, w1, b = make_gemm_inputs(m, n, k1)
+    a2, w2, _ = make_gemm_inputs(m, n, k2, seed=11)
+    c = fm.dual_gemm_bias_act(a1.to(DEV), w1.to(DEV), a2.to(DEV), w2.to(DEV), b.to(DEV), act=act)
+    torch.cuda.synchronize()
+    check(c, dual_gemm_bias_act_fp64(a1, w1, a2, w2, b, {"none": 0, "relu": 1, "tanh": 4}[act]),
+          f"dual {m}x{n}x({k1}+{k2}) {act}")

@@ -335,3 +335,28 @@ def test_layer_matches_torch_fp64_composition():
     # ulp of an intermediate, propagated (tiny next to the GPU tolerance)
     np.testing.assert_allclose(y, yt.numpy(), atol=2e-3, rtol=0)
     assert np.abs(y - yt.numpy()).mean() < 1e-6
+
+
+# ---------------------------------------------------------------- simplified LSTM cell (f4)
+def test_dual_gemm_pins():
+    """act(A1 W1^T + A2 W2^T + b): equals one GEMM over the K-concatenated operands (a block-matrix
+    identity), torch fp64 linear + linear, and ReLU / tanh closed forms on hand values."""
+    from oracle import dual_gemm_bias_act_fp64
+    from oracle.gemm import ACT_NONE, ACT_RELU, ACT_TANH
+    r = np.random.default_rng(5)
+    a1, w1 = r.standard_normal((7, 5)), r.standard_normal((4, 5))
+    a2, w2 = r.standard_normal((7, 3)), r.standard_normal((4, 3))
+    b = r.standard_normal(4)
+    cat = gemm_bias_act_fp64(np.hstack([a1, a2]), np.hstack([w1, w2]), b, ACT_NONE)
+    np.testing.assert_allclose(dual_gemm_bias_act_fp64(a1, w1, a2, w2, b, ACT_NONE), cat, atol=1e-13, rtol=0)
+    lin = (torch.nn.functional.linear(torch.from_numpy(a1), torch.from_numpy(w1))
+           + torch.nn.functional.linear(torch.from_numpy(a2), torch.from_numpy(w2), torch.from_numpy(b)))
+    np.testing.assert_allclose(dual_gemm_bias_act_fp64(a1, w1, a2, w2, b, ACT_RELU), lin.clamp_min(0).numpy(),
+                               atol=1e-13, rtol=0)
+    np.testing.assert_allclose(dual_gemm_bias_act_fp64(a1, w1, a2, w2, b, ACT_TANH), torch.tanh(lin).numpy(),
+                               atol=1e-13, rtol=0)
+    # by hand: 1x1 operands
+    one = np.ones((1, 1))
+    assert dual_gemm_bias_act_fp64(2 * one, 3 * one, -4 * one, 2 * one, np.array([1.0]), ACT_RELU)[0, 0] == 0.0
+    assert dual_gemm_bias_act_fp64(2 * one, 3 * one, 1 * one, 2 * one, np.array([-1.0]), ACT_RELU)[0, 0] == 7.0
+    assert dual_gemm_bias_act_fp64(one, one, one, -one, None, ACT_TANH)[0, 0] == 0.0
