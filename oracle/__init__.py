@@ -22,6 +22,7 @@ fmha   numpy fp64, unfused GEMM -> softmax -> GEMM per (batch, head);
 brute  pure-Python scalar loops with math.fsum, tiny shapes only        [pinned]
 gemm   numpy fp64 act(A @ W^T + b); act(A1 W1^T + A2 W2^T + b) (LSTM cell) [pinned]
 layer  QKV GEMM -> varlen FMHA -> out GEMM -> MLP, fp16 storage between  [pinned]
+mlp    L chained (GEMM + bias + act) layers, N = K, fp16 between layers  [pinned]
 
 Every function is pinned by ``tests/test_oracle.py`` against closed forms,
 invariants, a hand-derived golden fixture (``tests/golden/``), brute force and
@@ -33,6 +34,7 @@ from .fmha import attention_fp64, attention_rows_fp64, attention_varlen_fp64, so
 from .brute import attention_brute
 from .gemm import dual_gemm_bias_act_fp64, gemm_bias_act_fp64, gelu_erf, gelu_tanh, relu
 from .layer import round_fp16, transformer_layer_fp64
+from .mlp import mlp_fused_flops, mlp_fused_fp64, mlp_fused_rows_fp64
 
 __all__ = [
     "attention_fp64",
@@ -48,4 +50,7 @@ __all__ = [
     "relu",
     "round_fp16",
     "transformer_layer_fp64",
+    "mlp_fused_fp64",
+    "mlp_fused_rows_fp64",
+    "mlp_fused_flops",
 ]

@@ -360,3 +360,117 @@ def test_dual_gemm_pins():
     assert dual_gemm_bias_act_fp64(2 * one, 3 * one, -4 * one, 2 * one, np.array([1.0]), ACT_RELU)[0, 0] == 0.0
     assert dual_gemm_bias_act_fp64(2 * one, 3 * one, 1 * one, 2 * one, np.array([-1.0]), ACT_RELU)[0, 0] == 7.0
     assert dual_gemm_bias_act_fp64(one, one, one, -one, None, ACT_TANH)[0, 0] == 0.0
+
+
+# ---------------------------------------------------------------------------------------------
+# Fused multi-layer MLP (Fig. 11): pins for oracle.mlp_fused_fp64
+
+
+def _fp16_round_scalar(x: float) -> float:
+    import struct
+    return struct.unpack("<e", struct.pack("<e", x))[0]  # IEEE half, round-to-nearest-even
+
+
+def _mlp_brute(x, w, b, act_relu=True):
+    """Pure-Python scalar loops (math.fsum), fp16 rounding between layers: an implementation that
+    shares nothing with numpy's GEMM."""
+    h = [list(map(float, r)) for r in x]
+    L = len(w)
+    for l in range(L):
+        out = []
+        for r in h:
+            row = []
+            for n in range(len(w[l])):
+                z = math.fsum([r[k] * float(w[l][n][k]) for k in range(len(r))] + [float(b[l][n])])
+                z = max(z, 0.0) if act_relu else z
+                row.append(z if l + 1 == L else _fp16_round_scalar(z))
+            out.append(row)
+        h = out
+    return np.array(h)
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_mlp_brute_force_tiny(seed):
+    from oracle import mlp_fused_fp64
+    rng = np.random.default_rng(seed)
+    m, n, L = 3, 5, 4
+    x = rng.uniform(-1, 1, (m, n)).astype(np.float16)
+    w = (rng.standard_normal((L, n, n)) * 0.6).astype(np.float16)
+    b = rng.uniform(-0.3, 0.3, (L, n)).astype(np.float16)
+    got = mlp_fused_fp64(x, w, b, ACT_RELU)
+    want = _mlp_brute(x.tolist(), w.tolist(), b.tolist())
+    np.testing.assert_allclose(got, want, rtol=0, atol=1e-12)
+    got_lin = mlp_fused_fp64(x, w, b, ACT_NONE)
+    np.testing.assert_allclose(got_lin, _mlp_brute(x.tolist(), w.tolist(), b.tolist(), act_relu=False),
+                               rtol=0, atol=1e-12)
+
+
+def test_mlp_identity_weights_closed_form():
+    """W_l = I, b_l = c >= 0, X >= 0 (ReLU): every layer adds c exactly, so Y = X + L c."""
+    from oracle import mlp_fused_fp64
+    n, L = 16, 20
+    x = (np.arange(4 * n).reshape(4, n) % 7).astype(np.float16)
+    w = np.stack([np.eye(n)] * L).astype(np.float16)
+    c = np.float16(0.5)
+    b = np.full((L, n), c, dtype=np.float16)
+    np.testing.assert_array_equal(mlp_fused_fp64(x, w, b), x.astype(np.float64) + L * 0.5)
+
+
+def test_mlp_zero_weights_leave_last_bias():
+    from oracle import mlp_fused_fp64
+    rng = np.random.default_rng(5)
+    n, L = 8, 3
+    x = rng.uniform(-1, 1, (6, n)).astype(np.float16)
+    b = rng.uniform(-1, 1, (L, n)).astype(np.float16)
+    y = mlp_fused_fp64(x, np.zeros((L, n, n), np.float16), b)
+    np.testing.assert_array_equal(y, np.broadcast_to(np.maximum(b[-1].astype(np.float64), 0), y.shape))
+
+
+def test_mlp_hidden_permutation_invariance():
+    """Relabelling the hidden units between two layers (W_l -> P W_l, b_l -> P b_l,
+    W_{l+1} -> W_{l+1} P^T) leaves Y unchanged bit for bit: ReLU and the fp16 rounding are
+    elementwise.  A transposed operand or a mixed-up row/column index breaks it."""
+    from oracle import mlp_fused_fp64
+    rng = np.random.default_rng(11)
+    n, L = 12, 3
+    x = rng.uniform(-1, 1, (7, n)).astype(np.float16)
+    w = (rng.standard_normal((L, n, n)) / np.sqrt(n) * np.sqrt(2)).astype(np.float16)
+    b = rng.uniform(-0.2, 0.2, (L, n)).astype(np.float16)
+    perm = rng.permutation(n)
+    w2, b2 = w.copy(), b.copy()
+    w2[0] = w[0][perm]
+    b2[0] = b[0][perm]
+    w2[1] = w[1][:, perm]
+    np.testing.assert_array_equal(mlp_fused_fp64(x, w, b), mlp_fused_fp64(x, w2, b2))
+    w3 = w.copy()
+    w3[0] = w[0].T.copy()  # the transposed-operand mistake is visible
+    assert not np.array_equal(mlp_fused_fp64(x, w, b), mlp_fused_fp64(x, w3, b))
+
+
+def test_mlp_matches_torch_fp64_sequential():
+    """Library special case: torch.nn.functional.linear + relu in float64, rounded to fp16 between
+    layers by numpy's direct float64 -> float16 cast (torch's double -> half goes through float32,
+    a double rounding that flips rare near-tie elements)."""
+    from oracle import mlp_fused_fp64
+    rng = np.random.default_rng(3)
+    m, n, L = 33, 64, 6
+    x = rng.uniform(-1, 1, (m, n)).astype(np.float16)
+    w = (rng.standard_normal((L, n, n)) * np.sqrt(2.0 / n)).astype(np.float16)
+    b = rng.uniform(-0.1, 0.1, (L, n)).astype(np.float16)
+    h = torch.from_numpy(x).double()
+    for l in range(L):
+        h = torch.relu(torch.nn.functional.linear(h, torch.from_numpy(w[l]).double(), torch.from_numpy(b[l]).double()))
+        if l + 1 < L:
+            h = torch.from_numpy(h.numpy().astype(np.float16).astype(np.float64))
+    np.testing.assert_allclose(mlp_fused_fp64(x, w, b), h.numpy(), rtol=0, atol=1e-12)
+
+
+def test_mlp_positive_homogeneity():
+    """b = 0 and ReLU: Y(2 X) = 2 Y(X) exactly (scaling by 2 commutes with fp16 rounding)."""
+    from oracle import mlp_fused_fp64
+    rng = np.random.default_rng(8)
+    n, L = 16, 5
+    x = rng.uniform(-1, 1, (9, n)).astype(np.float16)
+    w = (rng.standard_normal((L, n, n)) * np.sqrt(2.0 / n)).astype(np.float16)
+    b = np.zeros((L, n), np.float16)
+    np.testing.assert_array_equal(mlp_fused_fp64(2 * x, w, b), 2 * mlp_fused_fp64(x, w, b))

@@ -274,3 +274,30 @@ def make_layer_inputs(cfg: LayerConfig, lengths=None, seed: int = SEED):
     arrs = [r(0).uniform(-1, 1, (t, d)).astype(np.float32), w(1, 3 * d, d), b(2, 3 * d), w(3, d, d), b(4, d),
             w(5, f, d), b(6, f), w(7, d, f), b(8, d)]
     return tuple(_round(a, torch.float16) for a in arrs), cu
+
+@dataclass(frozen=True)
+class FusedMlpConfig:
+    """The paper's fused multi-layer MLP (Fig. 11): `layers` chained GEMM + bias + ReLU
+    layers of width N = K <= 128 over M rows.  The paper gives no M; 65536 rows is an assumption
+    (DESIGN.md §4)."""
+    name: str
+    cfg_id: int
+    m: int
+    width: int
+    layers: int
+
+
+FUSED_MLP_CONFIGS = {
+    "mlp_fused": FusedMlpConfig("mlp_fused", 12, 65536, 128, 20),
+    "mlp_fused_w64": FusedMlpConfig("mlp_fused_w64", 13, 65536, 64, 20),
+}
+
+
+def make_fused_mlp_inputs(m: int, width: int, layers: int, seed: int = SEED, cfg_id: int = 12):
+    """x ~ U(-1, 1) [M, N]; W_l ~ N(0, 2/N) [L, N, N] (He scaling, so activations keep their size
+    through ReLU layers); b_l ~ U(-0.1, 0.1) [L, N].  fp16 CPU tensors (RNE from fp32)."""
+    r = lambda tid: _rng(cfg_id, tid, m, width * 1000 + layers, seed)
+    x = r(0).uniform(-1, 1, (m, width)).astype(np.float32)
+    w = (r(1).standard_normal((layers, width, width), dtype=np.float32) * np.sqrt(2.0 / width)).astype(np.float32)
+    b = r(2).uniform(-0.1, 0.1, (layers, width)).astype(np.float32)
+    return tuple(_round(a, torch.float16) for a in (x, w, b))
