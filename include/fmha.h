@@ -130,6 +130,21 @@ FMHA_API int gemm_bias_act(const void* A, const void* W, const void* bias, void*
 FMHA_API int dual_gemm_bias_act(const void* A1, const void* W1, const void* A2, const void* W2, const void* bias,
                                 void* C, int M, int N, int K1, int K2, int act, fmha_stream_t stream);
 
+/* Fused multi-layer MLP in ONE kernel: the paper's Fig. 11 ("Fusing
+ * multiple MLP-Layers (GEMM + bias-add + ReLU activation) into a single kernel", possible "for
+ * N=K<=128 with arbitrary M", up to 20 layers), SURVEY.md §8(f) f4:
+ *     h_0 = X;   h_l[m,n] = act( sum_k h_{l-1}[m,k] * W[l-1][n][k] + bias[l-1][n] ),  l = 1..layers;
+ *     Y = h_layers
+ * X, Y [M, width]; W [layers, width, width] (each layer nn.Linear [out, in]); bias [layers, width] or
+ * NULL: fp16, row-major, DEVICE, 16-byte aligned.  Every layer accumulates in fp32 and rounds once
+ * (RNE) to fp16; the intermediates h_1..h_{layers-1} are fp16 tiles that never leave shared memory
+ * (R19).  width must be 64 or 128 (FMHA_ERR_UNSUPPORTED otherwise), 1 <= layers <= 65535,
+ * any M >= 0 (M = 0: no launch).  act as gemm_bias_act (the paper's is 1 = ReLU).  Y must not
+ * overlap W or bias; Y == X (in place) is allowed (each 128-row tile is read before it is written,
+ * by the same CTA).  Errors: as gemm_bias_act. */
+FMHA_API int mlp_fused_fwd(const void* X, const void* W, const void* bias, void* Y, int M, int width, int layers,
+                           int act, fmha_stream_t stream);
+
 /* End-to-end synthetic Transformer layer (the paper's end-to-end use of its
  * fused kernels), fp16, tokens packed as in fmha_fwd_varlen:
  *     QKV = X Wqkv^T + bqkv        X [T, d_model], Wqkv [3 d_model, d_model] (rows: Q heads, K heads,

@@ -23,7 +23,7 @@ import torch
 from . import _lib
 from ._lib import FmhaError, FmhaMask
 
-__all__ = ["fmha_fwd", "fmha_fwd_varlen", "fmha_fwd_from_host", "gemm_bias_act", "dual_gemm_bias_act", "transformer_layer", "layer_workspace_bytes", "workspace_bytes", "FmhaError",
+__all__ = ["fmha_fwd", "fmha_fwd_varlen", "fmha_fwd_from_host", "gemm_bias_act", "dual_gemm_bias_act", "mlp_fused", "transformer_layer", "layer_workspace_bytes", "workspace_bytes", "FmhaError",
            "MASK_NONE", "MASK_KEY_PADDING", "MASK_CAUSAL", "ACTS", "version"]
 
 MASK_NONE, MASK_KEY_PADDING, MASK_CAUSAL = 0, 1, 2
@@ -213,4 +213,25 @@ def dual_gemm_bias_act(a1: torch.Tensor, w1: torch.Tensor, a2: torch.Tensor, w2:
                                 None if bias is None else bias.contiguous().data_ptr(), out.data_ptr(),
                                 m_, n_, k1, k2, ACTS[act], _stream_ptr(a1.device))
     _lib.check(st, "dual_gemm_bias_act")
+    return out
+
+
+def mlp_fused(x: torch.Tensor, w: torch.Tensor, bias: torch.Tensor | None = None, act: str = "relu",
+              out: torch.Tensor | None = None) -> torch.Tensor:
+    """Y = h_L of h_l = act(h_{l-1} W_l^T + b_l) in ONE kernel (the paper's fused multi-layer MLP,
+    Fig. 11): x [M,N], w [L,N,N], bias [L,N]; N in {64, 128}; fp16 CUDA tensors -> [M,N] fp16."""
+    lib = _lib.load()
+    ts = [x, w] + ([] if bias is None else [bias])
+    if any(t.dtype != torch.float16 or not t.is_cuda for t in ts):
+        raise TypeError("mlp_fused takes fp16 CUDA tensors (no CPU fallback)")
+    x, w = x.contiguous(), w.contiguous()
+    m_, n_ = x.shape
+    layers = w.shape[0]
+    if w.shape != (layers, n_, n_) or (bias is not None and bias.shape != (layers, n_)):
+        raise ValueError("shape mismatch")
+    if out is None:
+        out = torch.empty((m_, n_), dtype=torch.float16, device=x.device)
+    st = lib.mlp_fused_fwd(x.data_ptr(), w.data_ptr(), None if bias is None else bias.contiguous().data_ptr(),
+                           out.data_ptr(), m_, n_, layers, ACTS[act], _stream_ptr(x.device))
+    _lib.check(st, "mlp_fused_fwd")
     return out

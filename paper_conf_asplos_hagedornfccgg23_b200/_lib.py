@@ -32,6 +32,7 @@ EXPORTED_SYMBOLS = (
     "fmha_fwd_from_host",
     "gemm_bias_act",
     "dual_gemm_bias_act",
+    "mlp_fused_fwd",
     "transformer_layer_workspace_bytes",
     "transformer_layer_fwd",
     "fmha_status_string",
@@ -79,6 +80,9 @@ def load() -> ctypes.CDLL:
     lib.fmha_fwd_from_host.restype = i32
     lib.gemm_bias_act.argtypes = [vp, vp, vp, vp, i32, i32, i32, i32, vp]
     lib.gemm_bias_act.restype = i32
+    if hasattr(lib, "mlp_fused_fwd"):
+        lib.mlp_fused_fwd.argtypes = [vp, vp, vp, vp, i32, i32, i32, i32, vp]
+        lib.mlp_fused_fwd.restype = i32
     if hasattr(lib, "dual_gemm_bias_act"):
         lib.dual_gemm_bias_act.argtypes = [vp, vp, vp, vp, vp, vp, i32, i32, i32, i32, i32, vp]
         lib.dual_gemm_bias_act.restype = i32

@@ -12,6 +12,7 @@
 #include "../../include/fmha.h"
 #include "fmha_kernel.cuh"
 #include "gemm_kernel.cuh"
+#include "mlp_kernel.cuh"
 
 namespace {
 
@@ -267,6 +268,12 @@ int make_map_2d_rows(CUtensorMap* m, const void* base, uint64_t cols, uint64_t r
   if (st != FMHA_OK && err && errlen) snprintf(err, errlen, "%s", g_last_cuda_error);
   return st;
 }
+int make_map_3d_rows(CUtensorMap* m, const void* base, uint64_t cols, uint64_t rows, uint64_t units,
+                     uint32_t box_rows, char* err, size_t errlen) {
+  int st = make_map_3d(m, base, false, cols, rows, units, box_rows);
+  if (st != FMHA_OK && err && errlen) snprintf(err, errlen, "%s", g_last_cuda_error);
+  return st;
+}
 }  // namespace b200
 
 extern "C" {
@@ -409,6 +416,23 @@ int dual_gemm_bias_act(const void* A1, const void* W1, const void* A2, const voi
   return b200::launch_gemm_bias_act(A1, W1, A2, W2, bias, Cm, M, N, K1, K2, act, sms,
                                     reinterpret_cast<cudaStream_t>(stream), g_last_cuda_error,
                                     sizeof(g_last_cuda_error));
+}
+
+int mlp_fused_fwd(const void* X, const void* W, const void* bias, void* Y, int M, int width, int layers, int act,
+                  fmha_stream_t stream) {
+  g_last_cuda_error[0] = 0;
+  if (M < 0 || width < 0 || layers < 0) return FMHA_ERR_INVALID_ARG;
+  if (act < ACT_NONE || act > ACT_TANH) return FMHA_ERR_UNSUPPORTED;
+  if (width != 64 && width != 128) return FMHA_ERR_UNSUPPORTED;
+  if (layers < 1 || layers > 65535) return FMHA_ERR_UNSUPPORTED;
+  if (M == 0) return FMHA_OK;
+  if (!X || !W || !Y) return FMHA_ERR_INVALID_ARG;
+  if (!aligned16(X) || !aligned16(W) || !aligned16(Y) || (bias && !aligned16(bias))) return FMHA_ERR_MISALIGNED;
+  int sms = 0;
+  int st = check_device(&sms);
+  if (st != FMHA_OK) return st;
+  return b200::launch_mlp_fused(X, W, bias, Y, M, width, layers, act, sms, reinterpret_cast<cudaStream_t>(stream),
+                                g_last_cuda_error, sizeof(g_last_cuda_error));
 }
 
 const char* fmha_status_string(int status) {

@@ -1,0 +1,343 @@
+// mlp_kernel.cuh — the paper's fused multi-layer MLP on sm_100a (Fig. 11):
+// L layers h_l = act(h_{l-1} W_l^T + b_l) of width N = K <= 128 in ONE kernel, every intermediate
+// h_l kept on chip ("all intermediate tensors fit into the GPU's shared memory allowing to avoid
+// communication via the slower global memory", L453).  SURVEY §8(f) f4.
+//
+// Persistent, one CTA per SM.  A CTA owns S <= R row tiles of 128 rows at a time (a "group"; S is
+// a launch parameter, R the template's maximum: 4 at N = 128, 8 at N = 64) and walks them through
+// all L layers in lockstep, so every W_l tile loaded into shared memory feeds S MMAs, and while one
+// tile's epilogue runs the tensor core works on the others (a layer of one tile is a serial chain
+// MMA -> epilogue -> next MMA; S tiles in flight hide it):
+//   warp 0        TMA producer: the group's X tiles into ACT[r], then W_1 .. W_L (WS-stage ring)
+//   warp 1        MMA issuer: for each layer l and slot r, ACC_r = ACT[r] W_l^T (tcgen05.mma M=128
+//                 N=NW K=16, fp32 in TMEM columns [r NW, (r + 1) NW)); commit to ACC_FULL[r]
+//   warps 4..19   four epilogue warpgroups.  Warpgroup w owns columns 64 h.. (h = w % H, H = N / 64)
+//                 of slots r = w / H, w / H + 4 / H, ... (thread = accumulator row): TMEM -> + b_l ->
+//                 act -> one RNE rounding -> swizzled st.shared back into ACT[r], which IS the next
+//                 layer's A operand (K-major SW128, the layout TMA produces); after layer L the same
+//                 buffer is TMA-stored to Y
+//
+//   smem  ACT[R] | W ring[WS]   (N = 128: 4 x 32 KB + 3 x 32 KB;  N = 64: 8 x 16 KB + 4 x 8 KB)
+//   TMEM  ACC_r = columns [r NW, (r + 1) NW)   (R NW = 512)
+//
+// Barriers (every producer -> consumer edge has its consumer -> producer partner):
+//   X_FULL[r] / ACT_EMPTY[r]   TMA (X into ACT[r]) -> MMA;  the Y store out of ACT[r] has been read
+//                              (bulk read-completion, signalled by the storing thread) -> TMA
+//   W_FULL[s] / W_EMPTY[s]     TMA -> MMA -> TMA (commit after the last slot's MMA of the layer)
+//   ACC_FULL[r]                MMA commit -> epilogue of slot r
+//   ACT_FULL[r] (count 128 H)  epilogue -> MMA: ACC_r drained AND ACT[r] holds h_l (the generic-proxy
+//                              stores are fenced into the async proxy first)
+// ACT[r] is overwritten by layer l's epilogue only after ACC_FULL: layer l's MMA, the last reader
+// of ACT[r] = h_{l-1}, has completed.
+#pragma once
+#include "gemm_kernel.cuh"  // apply_act, make_map_2d_rows
+#include "sm100.cuh"
+
+namespace b200 {
+
+struct MlpParams {
+  CUtensorMap tmX;  // {NW, M, 1} box {64, 128, 1}, SWIZZLE_128B
+  CUtensorMap tmW;  // {NW, NW, L} box {64, NW, 1}
+  CUtensorMap tmY;  // as tmX
+  const __half* bias;  // [L, NW] or nullptr
+  int M, layers;
+  int slots;       // S: row tiles per group (1 .. R)
+  int num_groups;  // ceil(num_tiles / S)
+  int num_tiles;   // ceil(M / 128)
+};
+
+template <int NW>
+struct MlpCfg {
+  static constexpr int R = 512 / NW;                  // slots: all of TMEM holds accumulators
+  static constexpr int CHUNK = 128 * 128;             // one SW128 box of 128 rows x 64 16-bit elements
+  static constexpr int ATILE = 128 * NW * 2;          // 128 rows x NW
+  static constexpr int WCHUNK = NW * 128;             // NW rows x 64 elements
+  static constexpr int WTILE = NW * NW * 2;
+  static constexpr int WS = (NW == 128) ? 3 : 4;      // W ring stages
+  static constexpr int OFF_ACT = 0;
+  static constexpr int OFF_W = OFF_ACT + R * ATILE;
+  static constexpr int OFF_BAR = OFF_W + WS * WTILE;
+  // barriers: X_FULL[R], ACT_EMPTY[R], ACC_FULL[R], ACT_FULL[R], W_FULL[WS], W_EMPTY[WS]
+  static constexpr int NUM_BARS = 4 * R + 2 * WS;
+  static constexpr int OFF_TMEMPTR = OFF_BAR + NUM_BARS * 8;
+  static constexpr int SMEM_ALLOC = OFF_TMEMPTR + 16;
+  static constexpr int H = NW / 64;                   // column halves (64 columns = one SW128 chunk)
+  static constexpr int EPI_WG = 4;                    // epilogue warpgroups
+  static constexpr int SG = EPI_WG / H;               // slot groups: slot r -> warpgroups (r % SG) H + h
+  static constexpr int SPW = R / SG;                  // slots per epilogue warpgroup
+  static constexpr int THREADS = 128 + 128 * EPI_WG;
+  static constexpr int REG_LAUNCH = (65536 / THREADS) / 8 * 8;
+  static constexpr int REG_CTRL = 56;
+  static constexpr int REG_EPI = (REG_LAUNCH + (REG_LAUNCH - REG_CTRL) / EPI_WG) / 8 * 8;
+  static_assert(128 * REG_CTRL + 128 * EPI_WG * REG_EPI <= THREADS * REG_LAUNCH, "register pool");
+  static_assert(NW == 64 || NW == 128, "width");
+  static_assert(SMEM_ALLOC <= 232448, "shared memory budget");
+};
+
+template <int NW, int ACT>
+__global__ void __launch_bounds__(MlpCfg<NW>::THREADS, 1) mlp_fused_kernel(const __grid_constant__ MlpParams p) {
+  using C = MlpCfg<NW>;
+  constexpr int R = C::R;
+  extern __shared__ __align__(1024) uint8_t smem[];
+  const uint32_t sbase = smem_u32(smem);
+  const uint32_t bar = sbase + C::OFF_BAR;
+  auto X_FULL = [&](int r) { return bar + 8 * r; };
+  auto ACT_EMPTY = [&](int r) { return bar + 8 * (R + r); };
+  auto ACC_FULL = [&](int r) { return bar + 8 * (2 * R + r); };
+  auto ACT_FULL = [&](int r) { return bar + 8 * (3 * R + r); };
+  auto W_FULL = [&](int s) { return bar + 8 * (4 * R + s); };
+  auto W_EMPTY = [&](int s) { return bar + 8 * (4 * R + C::WS + s); };
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(smem + C::OFF_TMEMPTR);
+  const int warp = warp_id(), lane = lane_id();
+  const int S = p.slots, L = p.layers;
+
+  if (threadIdx.x == 0) {
+    if (sbase & 1023u) __trap();
+    for (int r = 0; r < R; ++r) {
+      mbar_init(X_FULL(r), 1);
+      mbar_init(ACT_EMPTY(r), 1);
+      mbar_init(ACC_FULL(r), 1);
+      mbar_init(ACT_FULL(r), 128 * C::H);
+    }
+    for (int s = 0; s < C::WS; ++s) {
+      mbar_init(W_FULL(s), 1);
+      mbar_init(W_EMPTY(s), 1);
+    }
+    fence_mbar_init();
+  }
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&p.tmX);
+    tma_prefetch_desc(&p.tmW);
+    tma_prefetch_desc(&p.tmY);
+  }
+  if (warp == 1) {
+    tmem_alloc(smem_u32(tmem_holder), 512);
+    tmem_relinquish();
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_holder;
+  // tiles of group g: g * S + r for r < ntiles(g)
+  auto ntiles = [&](int g) { return min(S, p.num_tiles - g * S); };
+
+  // registers: the launch gives every thread 65536 / THREADS (96 at 640 threads); warpgroup 0 (TMA,
+  // MMA, two idle warps) gives some back to the epilogue warps (setmaxnreg inside each role's
+  // branch, so ptxas allocates each region with its own budget)
+  if (warp < 4) {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(C::REG_CTRL));
+    if (warp == 0) {
+      // -------------------------------------------------------------- TMA producer
+      const uint64_t keep = policy_evict_last();   // W: re-read by every group of every CTA
+      const uint64_t once = policy_evict_first();  // X rows: read once
+      uint32_t wl = 0, xbits = 0;  // bit r: parity of the X loads into ACT[r] so far
+      for (int g = blockIdx.x; g < p.num_groups; g += gridDim.x) {
+        const int nt = ntiles(g);
+#pragma unroll 1
+        for (int r = 0; r < nt; ++r) {
+          mbar_wait(ACT_EMPTY(r), ((xbits >> r) & 1) ^ 1);  // the previous group's Y store has read ACT[r]
+          xbits ^= 1u << r;
+          mbar_arrive_expect_tx_elect(X_FULL(r), C::ATILE);
+#pragma unroll
+          for (int c = 0; c < NW / 64; ++c)
+            tma_load_3d_hint_elect(sbase + C::OFF_ACT + r * C::ATILE + c * C::CHUNK, &p.tmX, X_FULL(r), 64 * c,
+                                   (g * S + r) * 128, 0, once);
+        }
+        for (int l = 0; l < L; ++l, ++wl) {
+          const int s = wl % C::WS;
+          mbar_wait(W_EMPTY(s), ((wl / C::WS) & 1) ^ 1);
+          mbar_arrive_expect_tx_elect(W_FULL(s), C::WTILE);
+#pragma unroll
+          for (int c = 0; c < NW / 64; ++c)
+            tma_load_3d_hint_elect(sbase + C::OFF_W + s * C::WTILE + c * C::WCHUNK, &p.tmW, W_FULL(s), 64 * c, 0,
+                                   l, keep);
+        }
+      }
+    } else if (warp == 1) {
+      // -------------------------------------------------------------- MMA issuer
+      constexpr uint32_t IDESC = idesc_f16(false, 128, NW, false, false);  // A, W: K-major
+      const uint64_t desc0 = sdesc_sw128(sbase, 16, 1024);
+      // parity bits per slot (bit r): MMAs issued into ACC_r, X tiles consumed from ACT[r]
+      uint32_t wl = 0, ubits = 0, xbits = 0;
+      for (int g = blockIdx.x; g < p.num_groups; g += gridDim.x) {
+        const int nt = ntiles(g);
+        for (int l = 0; l < L; ++l, ++wl) {
+          const int s = wl % C::WS;
+          mbar_wait(W_FULL(s), (wl / C::WS) & 1);
+          const uint32_t woff = C::OFF_W + s * C::WTILE;
+#pragma unroll 1
+          for (int r = 0; r < nt; ++r) {
+            if (l == 0) {
+              mbar_wait(X_FULL(r), (xbits >> r) & 1);  // (the previous group's last epilogue of slot r
+              xbits ^= 1u << r;                        //  drained ACC_r before its Y store: implied)
+            } else {
+              mbar_wait(ACT_FULL(r), ((ubits >> r) & 1) ^ 1);  // ACC_r drained, ACT[r] = h_{l-1}
+            }
+            tc_fence_after();
+            const uint32_t aoff = C::OFF_ACT + r * C::ATILE;
+#pragma unroll
+            for (int kk = 0; kk < NW / 16; ++kk)
+              umma_ss_elect(tmem + r * NW, desc0 + ((aoff + (kk / 4) * C::CHUNK + (kk % 4) * 32) >> 4),
+                            desc0 + ((woff + (kk / 4) * C::WCHUNK + (kk % 4) * 32) >> 4), IDESC, kk > 0);
+            umma_commit_elect(ACC_FULL(r));
+            ubits ^= 1u << r;
+          }
+          umma_commit_elect(W_EMPTY(s));
+        }
+      }
+    }
+  } else {
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(C::REG_EPI));
+    // ---------------------------------------------------------------- epilogue
+    // warp 4 + 4 w + quad: accumulator rows 32 quad.., columns 64 h .. 64 h + 63 (= SW128 chunk h of
+    // the next layer's A operand) of slots sg, sg + SG, ...
+    const int w = (warp - 4) >> 2, h = w % C::H, sg = w / C::H, quad = warp & 3;
+    const int row = quad * 32 + lane;
+    const uint32_t lane_off = static_cast<uint32_t>(quad * 32) << 16;
+    constexpr uint32_t EPI_THREADS = 128 * C::H;  // threads writing one slot's ACT tile
+    uint32_t use[C::SPW];
+#pragma unroll
+    for (int j = 0; j < C::SPW; ++j) use[j] = 0;
+    for (int g = blockIdx.x; g < p.num_groups; g += gridDim.x) {
+      const int nt = ntiles(g);
+      for (int l = 0; l < L; ++l) {
+        const uint4* bl =
+            p.bias ? reinterpret_cast<const uint4*>(p.bias + static_cast<size_t>(l) * NW + 64 * h) : nullptr;
+        // this thread's 64 bias values are one 128-byte line: pull the next layer's into L1 now (an
+        // L2 round trip per layer would otherwise sit on every tile's MMA -> epilogue -> MMA chain)
+        if (bl) {
+          const __half* nxt = p.bias + static_cast<size_t>(l + 1 < L ? l + 1 : 0) * NW + 64 * h;
+          if (l == 0) asm volatile("prefetch.global.L1 [%0];" ::"l"(bl));
+          asm volatile("prefetch.global.L1 [%0];" ::"l"(nxt));
+        }
+#pragma unroll
+        for (int j = 0; j < C::SPW; ++j) {  // this warpgroup's slots, in the MMA warp's issue order
+          const int r = sg + j * C::SG;
+          if (r >= nt) continue;
+          mbar_wait(ACC_FULL(r), use[j] & 1);
+          ++use[j];
+          tc_fence_after();
+          uint32_t v[64];
+          const uint32_t tacc = tmem + lane_off + r * NW + 64 * h;
+          tmem_ld_32x32b_x32(tacc, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+          tmem_ld_32x32b_x32(tacc + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
+          tmem_wait_ld();
+          reg_fence(v);
+          const uint32_t act_box = sbase + C::OFF_ACT + r * C::ATILE + h * C::CHUNK + row * 128;
+#pragma unroll
+          for (int q = 0; q < 2; ++q) {  // 32 columns at a time: their bias (4 x 16 B, L1-resident)
+            uint4 braw[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) braw[u] = bl ? __ldg(bl + 4 * q + u) : make_uint4(0u, 0u, 0u, 0u);
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+              const __half2* b2 = reinterpret_cast<const __half2*>(&braw[u]);
+              const uint32_t* vv = &v[32 * q + 8 * u];
+              uint32_t pk[4];
+#pragma unroll
+              for (int e = 0; e < 4; ++e) {
+                const float2 bf = __half22float2(b2[e]);
+                pk[e] = pack2<false>(apply_act<ACT>(__uint_as_float(vv[2 * e]) + bf.x),
+                                     apply_act<ACT>(__uint_as_float(vv[2 * e + 1]) + bf.y));
+              }
+              const int unit = 4 * q + u;  // 16-byte unit of the 128-byte row, XOR-swizzled (SW128)
+              st_shared_v4(act_box + ((unit ^ (row & 7)) << 4), pk[0], pk[1], pk[2], pk[3]);
+            }
+          }
+          fence_proxy_async_smem();  // h_l visible to the async proxy (tensor core operand reads, TMA store)
+          tc_fence_before();
+          mbar_arrive(ACT_FULL(r));
+          if (l == L - 1) {  // Y rows of tile r (rows >= M clipped by the tensor map)
+            named_bar_sync(1 + sg, EPI_THREADS);
+            if (row == 0 && h == 0) {
+#pragma unroll
+              for (int c = 0; c < NW / 64; ++c)
+                tma_store_3d(&p.tmY, sbase + C::OFF_ACT + r * C::ATILE + c * C::CHUNK, 64 * c, (g * S + r) * 128, 0);
+              tma_store_commit();
+              tma_store_wait_read0();  // ACT[r] read out: the next group's X may land in it
+              mbar_arrive(ACT_EMPTY(r));
+            }
+          }
+        }
+      }
+    }
+    if (row == 0 && h == 0) tma_store_wait0();
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc(tmem, 512);
+  }
+}
+
+int make_map_3d_rows(CUtensorMap* m, const void* base, uint64_t cols, uint64_t rows, uint64_t units,
+                     uint32_t box_rows, char* err, size_t errlen);
+
+template <int NW>
+inline int launch_mlp_fused_w(MlpParams& prm, int act, int sms, cudaStream_t stream, char* err, size_t errlen) {
+  using C = MlpCfg<NW>;
+  constexpr int R = C::R;
+  void (*kern)(MlpParams) = act == 1 ? mlp_fused_kernel<NW, 1>
+                            : act == 2 ? mlp_fused_kernel<NW, 2>
+                            : act == 3 ? mlp_fused_kernel<NW, 3>
+                            : act == 4 ? mlp_fused_kernel<NW, 4>
+                                       : mlp_fused_kernel<NW, 0>;
+  static bool attr_done[64][5];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 64 || !attr_done[dev][act]) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_ALLOC);
+    if (e != cudaSuccess) {
+      snprintf(err, errlen, "cudaFuncSetAttribute(mlp_fused): %s", cudaGetErrorString(e));
+      return 4;
+    }
+    if (dev < 64) attr_done[dev][act] = true;
+  }
+  // Slots per group S.  One tile's layer is a serial chain: MMA (t) -> epilogue (E ~ e t, e ~ 3) ->
+  // next MMA.  With S tiles in flight a group's layer takes about max(S t, t + E ceil(S / SG)) (an
+  // epilogue warpgroup serves ceil(S / SG) slots in turn), and a CTA runs ceil(groups / SMs) rounds;
+  // pick the S with the least rounds x that, the larger S on ties (more reuse of each W_l tile).
+  {
+    const double e = 3.0;
+    double best = 1e300;
+    for (int s = 1; s <= R; ++s) {
+      const long long groups = (prm.num_tiles + s - 1) / s;
+      const long long rounds = (groups + sms - 1) / std::max(sms, 1);
+      const double per = std::max(static_cast<double>(s), 1.0 + e * ((s + C::SG - 1) / C::SG));
+      const double cost = static_cast<double>(rounds) * per;
+      if (cost <= best) {
+        best = cost;
+        prm.slots = s;
+      }
+    }
+  }
+  prm.num_groups = (prm.num_tiles + prm.slots - 1) / prm.slots;
+  const int grid = std::min(prm.num_groups, sms);
+  kern<<<grid, C::THREADS, C::SMEM_ALLOC, stream>>>(prm);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) {
+    snprintf(err, errlen, "mlp_fused_kernel launch: %s", cudaGetErrorString(e));
+    return 4;
+  }
+  return 0;
+}
+
+// Y = h_L of the chain (see the file comment); W [L, NW, NW], bias [L, NW] or nullptr.
+inline int launch_mlp_fused(const void* X, const void* W, const void* bias, void* Y, int M, int NW, int L, int act,
+                            int sms, cudaStream_t stream, char* err, size_t errlen) {
+  MlpParams prm;
+  memset(&prm, 0, sizeof(prm));
+  int st;
+  if ((st = make_map_2d_rows(&prm.tmX, X, NW, M, 128, err, errlen)) != 0) return st;
+  if ((st = make_map_2d_rows(&prm.tmY, Y, NW, M, 128, err, errlen)) != 0) return st;
+  if ((st = make_map_3d_rows(&prm.tmW, W, NW, NW, L, NW, err, errlen)) != 0) return st;
+  prm.bias = static_cast<const __half*>(bias);
+  prm.M = M;
+  prm.layers = L;
+  prm.num_tiles = (M + 127) / 128;
+  return NW == 128 ? launch_mlp_fused_w<128>(prm, act, sms, stream, err, errlen)
+                   : launch_mlp_fused_w<64>(prm, act, sms, stream, err, errlen);
+}
+
+}  // namespace b200

@@ -76,6 +76,14 @@ def test_validation_codes(lib):
     assert dg(16, 16, None, 16, None, 16, 4, 8, 16, 16, 1, None) == 1  # null A2
     assert dg(16, 16, 24, 16, None, 16, 4, 8, 16, 16, 1, None) == 3    # misaligned
     assert dg(16, 16, 16, 16, None, 16, 0, 8, 16, 16, 1, None) == 0    # M = 0
+    mf = lib.mlp_fused_fwd
+    assert mf(16, 16, None, 16, 4, 96, 3, 1, None) == 2                # width not 64 / 128
+    assert mf(16, 16, None, 16, 4, 128, 0, 1, None) == 2               # no layers
+    assert mf(16, 16, None, 16, 4, 128, 3, 9, None) == 2               # act
+    assert mf(16, 16, None, 16, -1, 128, 3, 1, None) == 1              # negative M
+    assert mf(None, 16, None, 16, 4, 128, 3, 1, None) == 1             # null X
+    assert mf(16, 24, None, 16, 4, 128, 3, 1, None) == 3               # misaligned W
+    assert mf(None, None, None, None, 0, 128, 3, 1, None) == 0         # M = 0
     # varlen: validation before any device access
     vl = lib.fmha_fwd_varlen
     assert vl(16, 16, 16, 2, 8, 16, 2, 96, 0.1, 0, 0, None) == 2       # head_dim
@@ -95,3 +103,4 @@ def test_no_device_is_loud(lib):
         pytest.skip("GPU present")
     # a valid compute call on a machine without an sm_100 device must fail, never fall back
     assert call_fmha(lib) == 5
+    assert lib.mlp_fused_fwd(16, 16, None, 16, 4, 128, 3, 1, None) == 5

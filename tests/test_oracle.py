@@ -474,3 +474,21 @@ def test_mlp_positive_homogeneity():
     w = (rng.standard_normal((L, n, n)) * np.sqrt(2.0 / n)).astype(np.float16)
     b = np.zeros((L, n), np.float16)
     np.testing.assert_array_equal(mlp_fused_fp64(2 * x, w, b), 2 * mlp_fused_fp64(x, w, b))
+
+
+def test_mlp_tolerance_covers_fp32_kernel_model():
+    """The fused-MLP GPU tolerance (tests/test_mlp_fused_gpu.py) against a numpy model of the
+    kernel's arithmetic: fp32 accumulation, fp32 bias add and ReLU, fp16 (RNE) store per layer.
+    At 20 layers the model must pass the depth-scaled bound and fail the depth-independent one
+    (so the scaling is needed, not slack)."""
+    from oracle import mlp_fused_fp64
+    from workloads import make_fused_mlp_inputs
+    x, w, b = (t.numpy() for t in make_fused_mlp_inputs(500, 128, 20))
+    ref = mlp_fused_fp64(x, w, b)
+    h = x.astype(np.float32)
+    for l in range(20):
+        h = np.maximum(h @ w[l].astype(np.float32).T + b[l].astype(np.float32), 0).astype(np.float16).astype(np.float32)
+    d = np.abs(h.astype(np.float64) - ref)
+    assert not (d > 1e-3 * (1 + np.sqrt(20)) + 2 ** -8 * np.abs(ref)).any()
+    assert np.linalg.norm(d) / np.linalg.norm(ref) <= 1e-3
+    assert (d > 2e-3 + 2 ** -9 * np.abs(ref)).any()
