@@ -9,21 +9,22 @@
 // tile's epilogue runs the tensor core works on the others (a layer of one tile is a serial chain
 // MMA -> epilogue -> next MMA; S tiles in flight hide it):
 //   warp 0        TMA producer: the group's X tiles into ACT[r], then W_1 .. W_L (WS-stage ring)
-//   warp 1        MMA issuer: for each layer l and slot r, ACC_r = ACT[r] W_l^T (tcgen05.mma M=128
+//   warp 1 + r    MMA issuer of slot r: for each layer l, ACC_r = ACT[r] W_l^T (tcgen05.mma M=128
 //                 N=NW K=16, fp32 in TMEM columns [r NW, (r + 1) NW)); commit to ACC_FULL[r]
-//   warps 4..19   four epilogue warpgroups.  Warpgroup w owns columns 64 h.. (h = w % H, H = N / 64)
+//   last 16 warps four epilogue warpgroups.  Warpgroup w owns columns 64 h.. (h = w % H, H = N / 64)
 //                 of slots r = w / H, w / H + 4 / H, ... (thread = accumulator row): TMEM -> + b_l ->
 //                 act -> one RNE rounding -> swizzled st.shared back into ACT[r], which IS the next
 //                 layer's A operand (K-major SW128, the layout TMA produces); after layer L the same
 //                 buffer is TMA-stored to Y
 //
-//   smem  ACT[R] | W ring[WS]   (N = 128: 4 x 32 KB + 3 x 32 KB;  N = 64: 8 x 16 KB + 4 x 8 KB)
+//   smem  ACT[R] | W ring[WS] | fp32 bias ring   (N = 128: 4 x 32 KB + 3 x 32 KB + 2 KB;
+//                                                  N = 64: 8 x 16 KB + 4 x 8 KB + 2 KB)
 //   TMEM  ACC_r = columns [r NW, (r + 1) NW)   (R NW = 512)
 //
 // Barriers (every producer -> consumer edge has its consumer -> producer partner):
 //   X_FULL[r] / ACT_EMPTY[r]   TMA (X into ACT[r]) -> MMA;  the Y store out of ACT[r] has been read
 //                              (bulk read-completion, signalled by the storing thread) -> TMA
-//   W_FULL[s] / W_EMPTY[s]     TMA -> MMA -> TMA (commit after the last slot's MMA of the layer)
+//   W_FULL[s] / W_EMPTY[s]     TMA -> MMA warps -> TMA (count R: every slot warp commits once per layer)
 //   ACC_FULL[r]                MMA commit -> epilogue of slot r
 //   ACT_FULL[r] (count 128 H)  epilogue -> MMA: ACC_r drained AND ACT[r] holds h_l (the generic-proxy
 //                              stores are fenced into the async proxy first)
@@ -56,7 +57,8 @@ struct MlpCfg {
   static constexpr int WS = (NW == 128) ? 3 : 4;      // W ring stages
   static constexpr int OFF_ACT = 0;
   static constexpr int OFF_W = OFF_ACT + R * ATILE;
-  static constexpr int OFF_BAR = OFF_W + WS * WTILE;
+  static constexpr int OFF_BIAS = OFF_W + WS * WTILE;  // fp32 b_l ring: [slot group][2][NW]
+  static constexpr int OFF_BAR = OFF_BIAS + (4 / (NW / 64)) * 2 * NW * 4;
   // barriers: X_FULL[R], ACT_EMPTY[R], ACC_FULL[R], ACT_FULL[R], W_FULL[WS], W_EMPTY[WS]
   static constexpr int NUM_BARS = 4 * R + 2 * WS;
   static constexpr int OFF_TMEMPTR = OFF_BAR + NUM_BARS * 8;
@@ -65,11 +67,16 @@ struct MlpCfg {
   static constexpr int EPI_WG = 4;                    // epilogue warpgroups
   static constexpr int SG = EPI_WG / H;               // slot groups: slot r -> warpgroups (r % SG) H + h
   static constexpr int SPW = R / SG;                  // slots per epilogue warpgroup
-  static constexpr int THREADS = 128 + 128 * EPI_WG;
+  // control warpgroups: warp 0 the TMA producer, warps 1..R one MMA issuer per slot (an mbarrier
+  // wait of an issuing warp queues behind that warp's in-flight MMAs, so one warp walking all slots
+  // left the tensor core idle between slots: measured ~420 cycles per slot)
+  static constexpr int CW = (1 + R + 3) / 4;
+  static constexpr int W_EPI = 4 * CW;                // first epilogue warp
+  static constexpr int THREADS = 128 * CW + 128 * EPI_WG;
   static constexpr int REG_LAUNCH = (65536 / THREADS) / 8 * 8;
-  static constexpr int REG_CTRL = 56;
-  static constexpr int REG_EPI = (REG_LAUNCH + (REG_LAUNCH - REG_CTRL) / EPI_WG) / 8 * 8;
-  static_assert(128 * REG_CTRL + 128 * EPI_WG * REG_EPI <= THREADS * REG_LAUNCH, "register pool");
+  static constexpr int REG_CTRL = 40;
+  static constexpr int REG_EPI = (REG_LAUNCH + (REG_LAUNCH - REG_CTRL) * CW / EPI_WG) / 8 * 8;
+  static_assert(128 * CW * REG_CTRL + 128 * EPI_WG * REG_EPI <= THREADS * REG_LAUNCH, "register pool");
   static_assert(NW == 64 || NW == 128, "width");
   static_assert(SMEM_ALLOC <= 232448, "shared memory budget");
 };
@@ -90,6 +97,7 @@ __global__ void __launch_bounds__(MlpCfg<NW>::THREADS, 1) mlp_fused_kernel(const
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(smem + C::OFF_TMEMPTR);
   const int warp = warp_id(), lane = lane_id();
   const int S = p.slots, L = p.layers;
+  TRACE_DECL  // debug timeline build only (FMHA_TRACE, tools/trace_mlp.py)
 
   if (threadIdx.x == 0) {
     if (sbase & 1023u) __trap();
@@ -101,7 +109,7 @@ __global__ void __launch_bounds__(MlpCfg<NW>::THREADS, 1) mlp_fused_kernel(const
     }
     for (int s = 0; s < C::WS; ++s) {
       mbar_init(W_FULL(s), 1);
-      mbar_init(W_EMPTY(s), 1);
+      mbar_init(W_EMPTY(s), R);  // one commit per slot MMA warp (idle slots commit at once)
     }
     fence_mbar_init();
   }
@@ -121,10 +129,10 @@ __global__ void __launch_bounds__(MlpCfg<NW>::THREADS, 1) mlp_fused_kernel(const
   // tiles of group g: g * S + r for r < ntiles(g)
   auto ntiles = [&](int g) { return min(S, p.num_tiles - g * S); };
 
-  // registers: the launch gives every thread 65536 / THREADS (96 at 640 threads); warpgroup 0 (TMA,
-  // MMA, two idle warps) gives some back to the epilogue warps (setmaxnreg inside each role's
-  // branch, so ptxas allocates each region with its own budget)
-  if (warp < 4) {
+  // registers: the launch gives every thread 65536 / THREADS; the control warpgroups (TMA, MMA,
+  // idle warps) give some back to the epilogue warps (setmaxnreg inside each role's branch, so
+  // ptxas allocates each region with its own budget)
+  if (warp < C::W_EPI) {
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(C::REG_CTRL));
     if (warp == 0) {
       // -------------------------------------------------------------- TMA producer
@@ -153,68 +161,77 @@ __global__ void __launch_bounds__(MlpCfg<NW>::THREADS, 1) mlp_fused_kernel(const
                                    l, keep);
         }
       }
-    } else if (warp == 1) {
-      // -------------------------------------------------------------- MMA issuer
+    } else if (warp <= R) {
+      // -------------------------------------------------------------- MMA issuer of slot r
+      const int r = warp - 1;
       constexpr uint32_t IDESC = idesc_f16(false, 128, NW, false, false);  // A, W: K-major
       const uint64_t desc0 = sdesc_sw128(sbase, 16, 1024);
-      // parity bits per slot (bit r): MMAs issued into ACC_r, X tiles consumed from ACT[r]
-      uint32_t wl = 0, ubits = 0, xbits = 0;
+      const uint32_t aoff = C::OFF_ACT + r * C::ATILE;
+      uint32_t wl = 0, use = 0, xc = 0;
       for (int g = blockIdx.x; g < p.num_groups; g += gridDim.x) {
-        const int nt = ntiles(g);
+        const bool active = r < ntiles(g);
         for (int l = 0; l < L; ++l, ++wl) {
           const int s = wl % C::WS;
-          mbar_wait(W_FULL(s), (wl / C::WS) & 1);
-          const uint32_t woff = C::OFF_W + s * C::WTILE;
-#pragma unroll 1
-          for (int r = 0; r < nt; ++r) {
+          mbar_wait(W_FULL(s), (wl / C::WS) & 1);  // (also keeps an idle slot's W_EMPTY arrival in phase)
+          if (active) {
             if (l == 0) {
-              mbar_wait(X_FULL(r), (xbits >> r) & 1);  // (the previous group's last epilogue of slot r
-              xbits ^= 1u << r;                        //  drained ACC_r before its Y store: implied)
+              mbar_wait(X_FULL(r), xc & 1);  // (the previous group's last epilogue of slot r drained ACC_r
+              ++xc;                          //  before its Y store: implied)
             } else {
-              mbar_wait(ACT_FULL(r), ((ubits >> r) & 1) ^ 1);  // ACC_r drained, ACT[r] = h_{l-1}
+              mbar_wait(ACT_FULL(r), (use - 1) & 1);  // ACC_r drained, ACT[r] = h_{l-1}
             }
             tc_fence_after();
-            const uint32_t aoff = C::OFF_ACT + r * C::ATILE;
+            TRACE_EV(5, r * 64 + l);
+            const uint32_t woff = C::OFF_W + s * C::WTILE;
 #pragma unroll
             for (int kk = 0; kk < NW / 16; ++kk)
               umma_ss_elect(tmem + r * NW, desc0 + ((aoff + (kk / 4) * C::CHUNK + (kk % 4) * 32) >> 4),
                             desc0 + ((woff + (kk / 4) * C::WCHUNK + (kk % 4) * 32) >> 4), IDESC, kk > 0);
             umma_commit_elect(ACC_FULL(r));
-            ubits ^= 1u << r;
+            TRACE_EV(6, r * 64 + l);
+            ++use;
           }
-          umma_commit_elect(W_EMPTY(s));
+          umma_commit_elect(W_EMPTY(s));  // this slot's reads of W_l are done
         }
       }
     }
   } else {
     asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(C::REG_EPI));
     // ---------------------------------------------------------------- epilogue
-    // warp 4 + 4 w + quad: accumulator rows 32 quad.., columns 64 h .. 64 h + 63 (= SW128 chunk h of
+    // warp W_EPI + 4 w + quad: accumulator rows 32 quad.., columns 64 h .. 64 h + 63 (= SW128 chunk h of
     // the next layer's A operand) of slots sg, sg + SG, ...
-    const int w = (warp - 4) >> 2, h = w % C::H, sg = w / C::H, quad = warp & 3;
+    const int w = (warp - C::W_EPI) >> 2, h = w % C::H, sg = w / C::H, quad = warp & 3;
     const int row = quad * 32 + lane;
     const uint32_t lane_off = static_cast<uint32_t>(quad * 32) << 16;
     constexpr uint32_t EPI_THREADS = 128 * C::H;  // threads writing one slot's ACT tile
     uint32_t use[C::SPW];
 #pragma unroll
     for (int j = 0; j < C::SPW; ++j) use[j] = 0;
+    auto bias_at = [&](int l) {
+      return p.bias ? __half2float(p.bias[static_cast<size_t>(l) * NW + 64 * h + (row & 63)]) : 0.f;
+    };
+    float bnext = 0.f;
+    bool first = true;
     for (int g = blockIdx.x; g < p.num_groups; g += gridDim.x) {
       const int nt = ntiles(g);
       for (int l = 0; l < L; ++l) {
-        const uint4* bl =
-            p.bias ? reinterpret_cast<const uint4*>(p.bias + static_cast<size_t>(l) * NW + 64 * h) : nullptr;
-        // this thread's 64 bias values are one 128-byte line: pull the next layer's into L1 now (an
-        // L2 round trip per layer would otherwise sit on every tile's MMA -> epilogue -> MMA chain)
-        if (bl) {
-          const __half* nxt = p.bias + static_cast<size_t>(l + 1 < L ? l + 1 : 0) * NW + 64 * h;
-          if (l == 0) asm volatile("prefetch.global.L1 [%0];" ::"l"(bl));
-          asm volatile("prefetch.global.L1 [%0];" ::"l"(nxt));
+        // b_l in fp32 for this slot group: thread (row < 64, h) converts column 64 h + row into the
+        // ring entry l % 2 (its previous readers, layer l - 2, are past the last layer's barrier)
+        const uint32_t bring = sbase + C::OFF_BIAS + (sg * 2 + (l & 1)) * NW * 4;
+        // (its global load was issued one layer ahead, so the L2 latency is off the chain)
+        if (row < 64) {
+          const float bv = first ? bias_at(l) : bnext;
+          bnext = bias_at(l + 1 < L ? l + 1 : 0);
+          first = false;
+          asm volatile("st.shared.f32 [%0], %1;" ::"r"(bring + (64 * h + row) * 4), "f"(bv) : "memory");
         }
+        named_bar_sync(1 + sg, EPI_THREADS);
 #pragma unroll
         for (int j = 0; j < C::SPW; ++j) {  // this warpgroup's slots, in the MMA warp's issue order
           const int r = sg + j * C::SG;
           if (r >= nt) continue;
           mbar_wait(ACC_FULL(r), use[j] & 1);
+          TRACE_EV(1, r * 64 + l);
           ++use[j];
           tc_fence_after();
           uint32_t v[64];
@@ -223,30 +240,38 @@ __global__ void __launch_bounds__(MlpCfg<NW>::THREADS, 1) mlp_fused_kernel(const
           tmem_ld_32x32b_x32(tacc + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
           tmem_wait_ld();
           reg_fence(v);
+          TRACE_EV(2, r * 64 + l);
           const uint32_t act_box = sbase + C::OFF_ACT + r * C::ATILE + h * C::CHUNK + row * 128;
+          const float4* bias4 = reinterpret_cast<const float4*>(smem + (bring - sbase)) + 16 * h;
 #pragma unroll
-          for (int q = 0; q < 2; ++q) {  // 32 columns at a time: their bias (4 x 16 B, L1-resident)
-            uint4 braw[4];
+          for (int u = 0; u < 8; ++u) {  // 8 columns -> one 16-byte unit of the 128-byte row
+            // broadcast reads (every thread the same address), plain loads so the compiler can
+            // hoist them ahead of the previous unit's stores
+            const float4 b0 = bias4[2 * u], b1 = bias4[2 * u + 1];
+            const float bb[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+            uint32_t pk[4];
 #pragma unroll
-            for (int u = 0; u < 4; ++u) braw[u] = bl ? __ldg(bl + 4 * q + u) : make_uint4(0u, 0u, 0u, 0u);
-#pragma unroll
-            for (int u = 0; u < 4; ++u) {
-              const __half2* b2 = reinterpret_cast<const __half2*>(&braw[u]);
-              const uint32_t* vv = &v[32 * q + 8 * u];
-              uint32_t pk[4];
-#pragma unroll
-              for (int e = 0; e < 4; ++e) {
-                const float2 bf = __half22float2(b2[e]);
-                pk[e] = pack2<false>(apply_act<ACT>(__uint_as_float(vv[2 * e]) + bf.x),
-                                     apply_act<ACT>(__uint_as_float(vv[2 * e + 1]) + bf.y));
+            for (int e = 0; e < 4; ++e) {
+              const float2 x = fadd2(make_float2(__uint_as_float(v[8 * u + 2 * e]), __uint_as_float(v[8 * u + 2 * e + 1])),
+                                     make_float2(bb[2 * e], bb[2 * e + 1]));
+              if constexpr (ACT == 1) {
+                // ReLU inside the conversion: cvt.rn.relu clamps the rounded pair at 0 (rounding is
+                // monotonic and keeps 0, so this equals rounding max(x, 0))
+                asm("cvt.rn.relu.f16x2.f32 %0, %1, %2;" : "=r"(pk[e]) : "f"(x.y), "f"(x.x));
+              } else if constexpr (ACT == 0) {
+                pk[e] = pack2<false>(x.x, x.y);
+              } else {
+                pk[e] = pack2<false>(apply_act<ACT>(x.x), apply_act<ACT>(x.y));
               }
-              const int unit = 4 * q + u;  // 16-byte unit of the 128-byte row, XOR-swizzled (SW128)
-              st_shared_v4(act_box + ((unit ^ (row & 7)) << 4), pk[0], pk[1], pk[2], pk[3]);
             }
+            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(act_box + ((u ^ (row & 7)) << 4)),
+                         "r"(pk[0]), "r"(pk[1]), "r"(pk[2]), "r"(pk[3]));
           }
+          TRACE_EV(3, r * 64 + l);
           fence_proxy_async_smem();  // h_l visible to the async proxy (tensor core operand reads, TMA store)
           tc_fence_before();
           mbar_arrive(ACT_FULL(r));
+          TRACE_EV(4, r * 64 + l);
           if (l == L - 1) {  // Y rows of tile r (rows >= M clipped by the tensor map)
             named_bar_sync(1 + sg, EPI_THREADS);
             if (row == 0 && h == 0) {
@@ -311,6 +336,10 @@ inline int launch_mlp_fused_w(MlpParams& prm, int act, int sms, cudaStream_t str
         prm.slots = s;
       }
     }
+  }
+  if (const char* ov = getenv("B200_MLP_SLOTS")) {  // tuning experiments only (tools/mlp_sweep.py)
+    const int v = atoi(ov);
+    if (v >= 1 && v <= R) prm.slots = v;
   }
   prm.num_groups = (prm.num_tiles + prm.slots - 1) / prm.slots;
   const int grid = std::min(prm.num_groups, sms);
