@@ -27,7 +27,7 @@ sys.path.insert(0, ROOT)
 import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
-from workloads import (CONFIGS, FUSED_MLP_CONFIGS, LAYER_CONFIGS, MASK_CAUSAL, MASK_KEY_PADDING, VARLEN_CONFIGS,  # noqa: E402
+from workloads import (CONFIGS, FUSED_MLP_CONFIGS, SPLITKV_CONFIGS, LAYER_CONFIGS, MASK_CAUSAL, MASK_KEY_PADDING, VARLEN_CONFIGS,  # noqa: E402
                        make_fmha_inputs, make_layer_inputs, make_varlen_inputs, shard)
 
 METRIC = "FMHA fwd TFLOP/s & % of B200 fp16 tensor peak at BERT-large shapes, 1/2/4/8 GPU"
@@ -156,7 +156,7 @@ def main():
     ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", default="bert_large_512", choices=sorted(CONFIGS) + sorted(VARLEN_CONFIGS) + sorted(LAYER_CONFIGS) + ["mlp", "lstm_cell"] + sorted(FUSED_MLP_CONFIGS))
+    ap.add_argument("--workload", default="bert_large_512", choices=sorted(CONFIGS) + sorted(VARLEN_CONFIGS) + sorted(LAYER_CONFIGS) + ["mlp", "lstm_cell"] + sorted(FUSED_MLP_CONFIGS) + sorted(SPLITKV_CONFIGS))
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of CPU oracle timing")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -174,6 +174,8 @@ def main():
         return run_lstm(args, world, rank, local)
     if args.workload in FUSED_MLP_CONFIGS:
         return run_mlp_fused(args, world, rank, local)
+    if args.workload in SPLITKV_CONFIGS:
+        return run_splitkv(args, world, rank, local)
     if args.workload in VARLEN_CONFIGS:
         return run_varlen(args, world, rank, local)
     if args.workload in LAYER_CONFIGS:
@@ -798,6 +800,76 @@ def run_mlp_fused(args, world, rank, local):
             "roofline": {"bound": "tensor", "achieved": round(val, 2), "peak": peak_burst, "unit": "TFLOP/s",
                          "frac": round(val / peak_burst, 4), "peak_source": f"{src} bf16 dense burst",
                          "kernel": "mlp_fused_kernel"},
+            "check_max_abs_err": err}), flush=True)
+
+
+def run_splitkv(args, world, rank, local):
+    """split-KV FMHA on a decode-like shape (few (b, h) units, a 16-row query block,
+    16k keys): one fmha_fwd_splitkv call per step (split kernel + merge kernel, default split
+    count).  The dense fmha_fwd kernel on the same inputs (one work item per (b, h): 32 of 148 SMs
+    busy) is timed beside it.  HBM-bound: the roofline is the algorithmic bytes (Q + K + V + O) per
+    step over the measured HBM bandwidth."""
+    import paper_conf_asplos_hagedornfccgg23_b200 as fm
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    cfg = SPLITKV_CONFIGS[args.workload]
+    q, k, v, _ = make_fmha_inputs(cfg)
+    set_bytes = alg_bytes(cfg)
+    n_sets = max(1, int(np.ceil(3 * L2_BYTES / set_bytes)))
+    qd, kd, vd = q.to(dev), k.to(dev), v.to(dev)
+    sets = [(qd, kd, vd, torch.empty_like(qd))] + [
+        (qd.clone(), kd.clone(), vd.clone(), torch.empty_like(qd)) for _ in range(n_sets - 1)]
+    lib = fm._lib.load()
+    splits = lib.fmha_splitkv_default_splits(cfg.batch, cfg.heads, cfg.seq_q, cfg.seq_kv)
+    ws = torch.empty(max(16, lib.fmha_splitkv_workspace_bytes(cfg.batch, cfg.heads, cfg.seq_q, cfg.head_dim, splits)),
+                     dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream(dev)
+    it = [0]
+
+    def step():
+        a, b_, c, o = sets[it[0] % n_sets]
+        it[0] += 1
+        fm.fmha_fwd_splitkv(a, b_, c, scale=cfg.scale, num_splits=splits, out=o, workspace=ws)
+
+    def dense():
+        a, b_, c, o = sets[it[0] % n_sets]
+        it[0] += 1
+        fm.fmha_fwd(a, b_, c, scale=cfg.scale, out=o)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    sampler = ClockSampler(local)
+    with sampler:
+        ms = _time_graph(step, args.steps, stream)
+    for _ in range(3):
+        dense()
+    torch.cuda.synchronize()
+    dense_ms = _time_graph(dense, args.steps, stream)
+    _, _, hbm, src = measured_peaks()
+    gbs = set_bytes / (ms * 1e-3) / 1e9
+    from oracle import attention_rows_fp64
+    o = sets[0][3]
+    step_ok = fm.fmha_fwd_splitkv(qd, kd, vd, scale=cfg.scale, num_splits=splits, out=o, workspace=ws)
+    torch.cuda.synchronize()
+    units = [(0, 0, 0), (cfg.batch - 1, cfg.heads - 1, cfg.seq_q - 1)]
+    ref = attention_rows_fp64(q, k, v, cfg.scale, units)
+    err = float(np.abs(torch.stack([step_ok[b, h, i] for b, h, i in units]).double().cpu().numpy() - ref).max())
+    if rank == 0:
+        print(json.dumps({
+            "metric": "split-KV FMHA fwd achieved HBM GB/s (decode-like shape)", "value": round(gbs, 1),
+            "unit": "GB/s", "n_gpus": 1, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 5),
+            "higher_is_better": True, "dtype": "bf16" if cfg.dtype == "bf16" else "f16", "data": "synthetic",
+            "config": {"workload": cfg.name, "batch": cfg.batch, "heads": cfg.heads, "seq_q": cfg.seq_q,
+                       "seq_kv": cfg.seq_kv, "head_dim": cfg.head_dim, "num_splits": splits,
+                       "l2": f"rotating {n_sets} input/output sets ({n_sets * set_bytes / 1e6:.0f} MB > 3x L2)"},
+            "tflops": round(alg_flops(cfg, None) / (ms * 1e-3) / 1e12, 2),
+            "context_dense_fmha_fwd": {"ms_per_step": round(dense_ms, 5), "speedup": round(dense_ms / ms, 3),
+                                       "what": "fmha_fwd (one work item per (b, h, q-tile pair)) on the same inputs"},
+            "clocks": sampler.summary(), "gpu_launches": 2 * args.steps,
+            "roofline": {"bound": "hbm", "achieved": round(gbs, 1), "peak": hbm, "unit": "GB/s",
+                         "frac": round(gbs / hbm, 4), "peak_source": f"{src} HBM copy bandwidth",
+                         "kernel": "fmha_fwd_kernel (split) + fmha_splitkv_combine_kernel"},
             "check_max_abs_err": err}), flush=True)
 
 

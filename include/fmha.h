@@ -110,6 +110,26 @@ FMHA_API int fmha_fwd_from_host(int dtype, const void* hQ, const void* hK, const
                        const fmha_mask_t* mask, void* workspace, size_t workspace_bytes, int batch, int heads,
                        int seq_q, int seq_kv, int head_dim, float scale, fmha_stream_t stream);
 
+/* Split-KV FMHA: the same operation as fmha_fwd / fmha_fwd_bf16 (dtype 0 = fp16,
+ * 1 = bf16; same layouts, mask and scale rules), for shapes where (batch x heads x query-tile pairs)
+ * would leave SMs idle -- few heads, short query blocks (seq_q <= 128: decode-like) and long keys.
+ * Each row's keys are cut into `num_splits` contiguous ranges of whole 128-key tiles; one kernel
+ * computes every (b, h, q-tile pair, split) as its own work item and writes the split's online-softmax
+ * state (unnormalised O in fp32, the exp2 reference scale*log2(e)*m and the row sum l, PAPER.md L487's
+ * softmax restricted to the range) into `workspace`; a second kernel merges the splits
+ * (O = sum_s 2^(m_s - M) O_s / sum_s 2^(m_s - M) l_s) and rounds O once.  num_splits = 0 picks
+ * fmha_splitkv_default_splits(); the count is clamped so every split holds at least one key tile, and
+ * a count of 1 runs the fmha_fwd kernel (no workspace needed).  `workspace`: DEVICE, 16-byte aligned,
+ * >= fmha_splitkv_workspace_bytes(batch, heads, seq_q, head_dim, splits) bytes (else
+ * FMHA_ERR_INVALID_ARG), owned by the caller, used until both kernels complete (stream order).
+ * Two launches on `stream`; errors as fmha_fwd. */
+FMHA_API int fmha_splitkv_default_splits(int batch, int heads, int seq_q, int seq_kv);
+FMHA_API size_t fmha_splitkv_workspace_bytes(int batch, int heads, int seq_q, int head_dim, int num_splits);
+FMHA_API int fmha_fwd_splitkv(int dtype, const void* Q, const void* K, const void* V, void* O,
+                              const fmha_mask_t* mask, int batch, int heads, int seq_q, int seq_kv, int head_dim,
+                              float scale, int num_splits, void* workspace, size_t workspace_bytes,
+                              fmha_stream_t stream);
+
 /* GEMM + bias + activation, the MLP building block:
  *     C[m,n] = act( sum_k A[m,k] * W[n,k] + bias[n] )
  * A [M,K], W [N,K] (nn.Linear layout), bias [N] (or NULL), C [M,N]: fp16, row-major, DEVICE,

@@ -23,7 +23,7 @@ import torch
 from . import _lib
 from ._lib import FmhaError, FmhaMask
 
-__all__ = ["fmha_fwd", "fmha_fwd_varlen", "fmha_fwd_from_host", "gemm_bias_act", "dual_gemm_bias_act", "mlp_fused", "transformer_layer", "layer_workspace_bytes", "workspace_bytes", "FmhaError",
+__all__ = ["fmha_fwd", "fmha_fwd_splitkv", "fmha_fwd_varlen", "fmha_fwd_from_host", "gemm_bias_act", "dual_gemm_bias_act", "mlp_fused", "transformer_layer", "layer_workspace_bytes", "workspace_bytes", "FmhaError",
            "MASK_NONE", "MASK_KEY_PADDING", "MASK_CAUSAL", "ACTS", "version"]
 
 MASK_NONE, MASK_KEY_PADDING, MASK_CAUSAL = 0, 1, 2
@@ -76,6 +76,42 @@ def fmha_fwd(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, kv_len: torch.Te
     st = fn(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), ctypes.byref(m), b, h, sq, skv, d,
             scale, _stream_ptr(q.device))
     _lib.check(st, "fmha_fwd")
+    return out
+
+
+def fmha_fwd_splitkv(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, kv_len: torch.Tensor | None = None,
+                     causal: bool = False, scale: float | None = None, num_splits: int = 0,
+                     out: torch.Tensor | None = None, workspace: torch.Tensor | None = None) -> torch.Tensor:
+    """The same operation as fmha_fwd with each row's keys split over `num_splits` work items and
+    merged by a second kernel (0 = the library's default for this shape).  `workspace` (a CUDA byte
+    tensor) is allocated here when not given.  Calls ``fmha_fwd_splitkv`` of the C ABI."""
+    lib = _lib.load()
+    if q.dtype not in (torch.float16, torch.bfloat16) or k.dtype != q.dtype or v.dtype != q.dtype:
+        raise TypeError("q, k, v must share dtype fp16 or bf16")
+    if not (q.is_cuda and k.is_cuda and v.is_cuda):
+        raise TypeError("q, k, v must be CUDA tensors (no CPU fallback)")
+    if not (q.is_contiguous() and k.is_contiguous() and v.is_contiguous()):
+        raise ValueError("q, k, v must be contiguous [B,H,S,D]")
+    b, h, sq, d = q.shape
+    skv = k.shape[2]
+    if k.shape != (b, h, skv, d) or v.shape != k.shape:
+        raise ValueError(f"shape mismatch q{tuple(q.shape)} k{tuple(k.shape)} v{tuple(v.shape)}")
+    if kv_len is not None:
+        if kv_len.dtype != torch.int32 or not kv_len.is_cuda or kv_len.numel() != b:
+            raise ValueError("kv_len must be a CUDA int32 tensor of length batch")
+        kv_len = kv_len.contiguous()
+    if out is None:
+        out = torch.empty_like(q)
+    splits = num_splits if num_splits > 0 else lib.fmha_splitkv_default_splits(b, h, sq, skv)
+    need = lib.fmha_splitkv_workspace_bytes(b, h, sq, d, splits)
+    if workspace is None or workspace.numel() < need:
+        workspace = torch.empty(max(need, 16), dtype=torch.uint8, device=q.device)
+    scale = 1.0 / math.sqrt(d) if scale is None else float(scale)
+    m = _mask(kv_len, causal)
+    st = lib.fmha_fwd_splitkv(0 if q.dtype == torch.float16 else 1, q.data_ptr(), k.data_ptr(), v.data_ptr(),
+                              out.data_ptr(), ctypes.byref(m), b, h, sq, skv, d, scale, splits,
+                              workspace.data_ptr(), workspace.numel(), _stream_ptr(q.device))
+    _lib.check(st, "fmha_fwd_splitkv")
     return out
 
 

@@ -30,6 +30,9 @@ EXPORTED_SYMBOLS = (
     "fmha_fwd_varlen",
     "fmha_workspace_bytes",
     "fmha_fwd_from_host",
+    "fmha_splitkv_default_splits",
+    "fmha_splitkv_workspace_bytes",
+    "fmha_fwd_splitkv",
     "gemm_bias_act",
     "dual_gemm_bias_act",
     "mlp_fused_fwd",
@@ -80,6 +83,13 @@ def load() -> ctypes.CDLL:
     lib.fmha_fwd_from_host.restype = i32
     lib.gemm_bias_act.argtypes = [vp, vp, vp, vp, i32, i32, i32, i32, vp]
     lib.gemm_bias_act.restype = i32
+    if hasattr(lib, "fmha_fwd_splitkv"):
+        lib.fmha_splitkv_default_splits.argtypes = [i32] * 4
+        lib.fmha_splitkv_default_splits.restype = i32
+        lib.fmha_splitkv_workspace_bytes.argtypes = [i32] * 5
+        lib.fmha_splitkv_workspace_bytes.restype = sz
+        lib.fmha_fwd_splitkv.argtypes = [i32, vp, vp, vp, vp, mp, i32, i32, i32, i32, i32, f32, i32, vp, sz, vp]
+        lib.fmha_fwd_splitkv.restype = i32
     if hasattr(lib, "mlp_fused_fwd"):
         lib.mlp_fused_fwd.argtypes = [vp, vp, vp, vp, i32, i32, i32, i32, vp]
         lib.mlp_fused_fwd.restype = i32

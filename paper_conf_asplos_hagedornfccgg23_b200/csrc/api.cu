@@ -13,6 +13,7 @@
 #include "fmha_kernel.cuh"
 #include "gemm_kernel.cuh"
 #include "mlp_kernel.cuh"
+#include "splitkv_kernel.cuh"
 
 namespace {
 
@@ -125,13 +126,15 @@ bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) ==
 template <int D, bool BF16>
 int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) {
   using C = b200::FmhaCfg<D>;
-  const int mode = prm.cu_seqlens ? (prm.sched ? b200::MODE_VARLEN_SCHED : b200::MODE_VARLEN)
-                                  : (prm.pair_mode ? b200::MODE_PAIRX : b200::MODE_DENSE);
+  const int mode = prm.num_splits > 1 ? b200::MODE_SPLIT
+                   : prm.cu_seqlens ? (prm.sched ? b200::MODE_VARLEN_SCHED : b200::MODE_VARLEN)
+                                    : (prm.pair_mode ? b200::MODE_PAIRX : b200::MODE_DENSE);
   void (*kern)(b200::FmhaParams) = mode == b200::MODE_DENSE    ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_DENSE>
                                    : mode == b200::MODE_PAIRX  ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_PAIRX>
                                    : mode == b200::MODE_VARLEN ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_VARLEN>
+                                   : mode == b200::MODE_SPLIT  ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_SPLIT>
                                                                : b200::fmha_fwd_sm100<D, BF16, b200::MODE_VARLEN_SCHED>;
-  static bool attr_done[64][4];
+  static bool attr_done[64][5];
   int dev = 0;
   cudaGetDevice(&dev);
   if (dev >= 64 || !attr_done[dev][mode]) {
@@ -144,11 +147,48 @@ int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) 
   kern<<<grid, C::THREADS, C::SMEM_ALLOC, stream>>>(prm);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "fmha_fwd_kernel launch");
+  if (mode == b200::MODE_SPLIT) {  // merge the splits into O (same stream, so after the kernel)
+    const long long rows = static_cast<long long>(prm.num_units) * prm.seq_q;
+    const long long blocks = (rows * 32 + 255) / 256;
+    b200::fmha_splitkv_combine_kernel<D, BF16><<<static_cast<unsigned>(blocks), 256, 0, stream>>>(
+        prm.ws_o, prm.ws_m, prm.ws_l, prm.o_ptr, prm.num_splits, rows);
+    e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "fmha_splitkv_combine_kernel launch");
+  }
   return FMHA_OK;
 }
 
+// Split-KV (fmha_fwd_splitkv): workspace floats for `splits` splits.
+size_t splitkv_ws_bytes(long long units, int seq_q, int head_dim, int splits) {
+  return static_cast<size_t>(splits) * units * seq_q * (head_dim + 2) * sizeof(float);
+}
+
+// Default split count.  A CTA runs ceil(items * s / SMs) rounds of items of ceil(nkv / s) KV tiles
+// plus a fixed per-item cost (Q load, pipeline fill, the fp32 partial-O store; ~2 tiles); pick the
+// s with the least rounds x (tiles + 2), at least one KV tile per split.  1 when the dense schedule
+// already fills the SMs.
+int splitkv_default(long long units, int seq_q, int seq_kv, int sms) {
+  const long long items = units * ((seq_q + 127) / 128 + 1) / 2;
+  const int nkv = (seq_kv + 127) / 128;
+  if (items <= 0 || items >= sms || nkv <= 1) return 1;
+  int best_s = 1;
+  long long best = -1;
+  for (int s = 1; s <= std::min(nkv, 64); ++s) {
+    const int per = (nkv + s - 1) / s;
+    if ((nkv + per - 1) / per != s) continue;  // s not reachable with whole tiles per split
+    const long long rounds = (items * s + sms - 1) / sms;
+    const long long cost = rounds * (per + 2);
+    if (best < 0 || cost < best) {
+      best = cost;
+      best_s = s;
+    }
+  }
+  return best_s;
+}
+
 int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask,
-                int batch, int heads, int seq_q, int seq_kv, int head_dim, float scale, cudaStream_t stream) {
+                int batch, int heads, int seq_q, int seq_kv, int head_dim, float scale, cudaStream_t stream,
+                int splits = 1, void* workspace = nullptr, size_t workspace_bytes = 0) {
   g_last_cuda_error[0] = 0;
   if (batch < 0 || heads < 0 || seq_q < 0 || seq_kv < 0) return FMHA_ERR_INVALID_ARG;
   if (!std::isfinite(scale)) return FMHA_ERR_INVALID_ARG;
@@ -198,6 +238,30 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   prm.div_pairs.init(static_cast<uint32_t>(std::max((prm.num_q_tiles + 1) / 2, 1)));
   prm.div_qtiles.init(static_cast<uint32_t>(std::max(prm.num_q_tiles, 1)));
   prm.div_heads.init(static_cast<uint32_t>(std::max(heads, 1)));
+  if (splits == 0) splits = splitkv_default(units, seq_q, seq_kv, sm_count);
+  if (splits > 1) {
+    const int nkv = (seq_kv + 127) / 128;
+    const int per = (nkv + splits - 1) / splits;
+    splits = (nkv + per - 1) / per;  // every split gets at least one KV tile
+  }
+  if (splits > 1) {
+    if (!workspace || workspace_bytes < splitkv_ws_bytes(units, seq_q, head_dim, splits)) return FMHA_ERR_INVALID_ARG;
+    if (reinterpret_cast<uintptr_t>(workspace) % 16 != 0) return FMHA_ERR_MISALIGNED;
+    const int nkv = (seq_kv + 127) / 128;
+    prm.num_splits = splits;
+    prm.split_tiles = (nkv + splits - 1) / splits;
+    prm.pair_mode = 0;  // (pairs of one unit's q-tiles; the split index is the fastest item digit)
+    const long long items = units * ((prm.num_q_tiles + 1) / 2) * splits;
+    if (items > 2147483647LL) return FMHA_ERR_UNSUPPORTED;
+    prm.num_items = static_cast<int>(items);
+    prm.div_splits.init(static_cast<uint32_t>(splits));
+    float* ws = static_cast<float*>(workspace);
+    const size_t rows = static_cast<size_t>(units) * seq_q;
+    prm.ws_o = ws;
+    prm.ws_m = ws + static_cast<size_t>(splits) * rows * head_dim;
+    prm.ws_l = prm.ws_m + static_cast<size_t>(splits) * rows;
+    prm.o_ptr = static_cast<uint8_t*>(O);
+  }
 
   if (head_dim == 64)
     return bf16 ? launch_fmha<64, true>(prm, sm_count, stream) : launch_fmha<64, false>(prm, sm_count, stream);
@@ -416,6 +480,26 @@ int dual_gemm_bias_act(const void* A1, const void* W1, const void* A2, const voi
   return b200::launch_gemm_bias_act(A1, W1, A2, W2, bias, Cm, M, N, K1, K2, act, sms,
                                     reinterpret_cast<cudaStream_t>(stream), g_last_cuda_error,
                                     sizeof(g_last_cuda_error));
+}
+
+size_t fmha_splitkv_workspace_bytes(int batch, int heads, int seq_q, int head_dim, int num_splits) {
+  if (batch <= 0 || heads <= 0 || seq_q <= 0 || head_dim <= 0 || num_splits <= 1) return 0;
+  return splitkv_ws_bytes(static_cast<long long>(batch) * heads, seq_q, head_dim, num_splits);
+}
+
+int fmha_splitkv_default_splits(int batch, int heads, int seq_q, int seq_kv) {
+  int sms = 0;
+  if (batch <= 0 || heads <= 0 || seq_q <= 0 || seq_kv <= 0 || check_device(&sms) != FMHA_OK) return 1;
+  return splitkv_default(static_cast<long long>(batch) * heads, seq_q, seq_kv, sms);
+}
+
+int fmha_fwd_splitkv(int dtype, const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask,
+                     int batch, int heads, int seq_q, int seq_kv, int head_dim, float scale, int num_splits,
+                     void* workspace, size_t workspace_bytes, fmha_stream_t stream) {
+  if (dtype != 0 && dtype != 1) return FMHA_ERR_UNSUPPORTED;
+  if (num_splits < 0 || num_splits > 1024) return FMHA_ERR_UNSUPPORTED;
+  return fmha_common(dtype == 1, Q, K, V, O, mask, batch, heads, seq_q, seq_kv, head_dim, scale,
+                     reinterpret_cast<cudaStream_t>(stream), num_splits, workspace, workspace_bytes);
 }
 
 int mlp_fused_fwd(const void* X, const void* W, const void* bias, void* Y, int M, int width, int layers, int act,

@@ -123,6 +123,15 @@ struct FmhaParams {
   int mask_kind;
   float scale_log2;  // scale * log2(e)
   FastDiv div_units, div_pairs, div_qtiles, div_heads;  // num_units, ceil(num_q_tiles/2), num_q_tiles, heads
+  // Split-KV mode (MODE_SPLIT, fmha_fwd_splitkv): item idx = (unit, q-tile pair) *
+  // num_splits + split; split s visits KV tiles [s * split_tiles, (s + 1) * split_tiles) and writes
+  // its unnormalised partial O (fp32), its exp2 reference mc = scale*log2e*m and its row sum l to
+  // the workspace; fmha_splitkv_combine_kernel merges the splits.
+  int num_splits, split_tiles;
+  FastDiv div_splits;
+  float* ws_o;   // [num_splits][num_units][seq_q][D]
+  float* ws_m;   // [num_splits][num_units][seq_q]
+  float* ws_l;   // [num_splits][num_units][seq_q]
 };
 
 template <int D>
@@ -214,6 +223,8 @@ struct WorkItem {
   int tok0, tok1;  // varlen: first token of the sequence of tile 0 / 1; len = its length
   int len0, len1;
   int head;        // varlen: h of unit bh0
+  int jb;          // split-KV: first KV tile of this item's range (0 otherwise)
+  int split;       // split-KV: split index
   // TMA coordinates (c1, c2) of the 128-row block starting at row r of tile t (c0 = d)
   __device__ __forceinline__ int c1(bool varlen, int t, int r) const { return varlen ? head : r; }
   __device__ __forceinline__ int c2(bool varlen, int t, int r) const { return varlen ? tok(t) + r : bh(t); }
@@ -232,10 +243,17 @@ struct WorkItem {
   }
 };
 
-template <bool PAIRX, bool VL>
+template <bool PAIRX, bool VL, bool SPLIT = false>
 __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
   WorkItem w;
   int qt0;
+  w.jb = 0;
+  w.split = 0;
+  if constexpr (SPLIT) {
+    const int rest = p.div_splits.div(idx);
+    w.split = idx - rest * p.num_splits;
+    idx = rest;
+  }
   if (!PAIRX) {
     const int pairs = (p.num_q_tiles + 1) >> 1;
     int pr;
@@ -291,6 +309,11 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
   }
   w.n0 = w.has0 ? (kv_end0 + 127) / 128 : 0;
   w.n1 = w.has1 ? (kv_end1 + 127) / 128 : 0;
+  if constexpr (SPLIT) {  // this split's KV tiles [jb, jb + split_tiles) of each tile's range
+    w.jb = w.split * p.split_tiles;
+    w.n0 = min(max(w.n0 - w.jb, 0), p.split_tiles);
+    w.n1 = min(max(w.n1 - w.jb, 0), p.split_tiles);
+  }
   return w;
 }
 
@@ -379,12 +402,13 @@ __device__ __forceinline__ int item_at(const FmhaParams& p, const SchedTable* tb
 // Kernel instances (MODE): dense [B,H,S,D]; dense with cross-unit tile pairing (pair_mode 1, see
 // FmhaParams::pair_mode); varlen packed; varlen packed with the cost-sorted schedule.  Separate
 // instances keep the varlen and scheduling code out of the dense kernels entirely.
-enum : int { MODE_DENSE = 0, MODE_PAIRX = 1, MODE_VARLEN = 2, MODE_VARLEN_SCHED = 3 };
+enum : int { MODE_DENSE = 0, MODE_PAIRX = 1, MODE_VARLEN = 2, MODE_VARLEN_SCHED = 3, MODE_SPLIT = 4 };
 
 template <int D, bool BF16, int MODE>
 __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
   using C = FmhaCfg<D>;
-  constexpr bool PAIRX = MODE == MODE_PAIRX, VL = MODE >= MODE_VARLEN, SCHED = MODE == MODE_VARLEN_SCHED;
+  constexpr bool PAIRX = MODE == MODE_PAIRX, VL = MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
+                 SCHED = MODE == MODE_VARLEN_SCHED, SPLIT = MODE == MODE_SPLIT;
   // Dynamic shared memory starts at the (1024-byte aligned) base of the CTA's shared window; the
   // SWIZZLE_128B tiles need that alignment.  Using the base directly keeps smem addresses uniform.
   extern __shared__ __align__(1024) uint8_t smem[];
@@ -461,11 +485,11 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
 #pragma unroll
           for (int c = 0; c < D / 64; ++c)
             tma_load_3d_hint_elect(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64,
-                                   w.c1(vl, t, j * 128), w.c2(vl, t, j * 128), keep);
+                                   w.c1(vl, t, (w.jb + j) * 128), w.c2(vl, t, (w.jb + j) * 128), keep);
         }
       };
       for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
-        const WorkItem w = decode_item<PAIRX, VL>(p, idx);
+        const WorkItem w = decode_item<PAIRX, VL, SPLIT>(p, idx);
         const int N = max(w.n0, w.n1);
 #pragma unroll
         for (int t = 0; t < 2; ++t) {
@@ -533,7 +557,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       auto seek = [&](Cursor& cu, int k, uint32_t base) {
         cu.valid = false;
         for (int idx; (idx = item_at<SCHED>(p, sched, k)) >= 0; ++k) {
-          const WorkItem w = decode_item<PAIRX, VL>(p, idx);
+          const WorkItem w = decode_item<PAIRX, VL, SPLIT>(p, idx);
           const int N = max(w.n0, w.n1);
           if (N == 0) continue;
           cu.w.n0 = w.n0;
@@ -672,7 +696,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     // g = real steps this thread has done so far: the phase count of S_FULL and PV_DONE
     uint32_t g = 0, lc = 0;
     for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
-      const WorkItem w = decode_item<PAIRX, VL>(p, idx);
+      const WorkItem w = decode_item<PAIRX, VL, SPLIT>(p, idx);
       const int n = w.n(t);
       const int N = C::TURNS ? max(w.n0, w.n1) : n;
       TRACE_EV(EV_ITEM, 1);
@@ -703,9 +727,9 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           tc_fence_before();
           mbar_arrive(S_FREE);
         }
-        const int rem = lim - j * 128;
+        const int rem = lim - (w.jb + j) * 128;
         // 32-key chunks no row of this warp can see are skipped: their P is stored as zeros
-        const int rem_w = lim_w - j * 128;
+        const int rem_w = lim_w - (w.jb + j) * 128;
         if (rem < 128) {  // boundary tile for this row (a5)
 #pragma unroll
           for (int k = 0; k < 128; ++k)
@@ -831,6 +855,13 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       TRACE_EV(EV_ITEM, 3);
       ++lc;
       s_lsum[t * 128 + row] = l;
+      if constexpr (SPLIT) {  // this split's row statistics (rows inside the sequence only)
+        if (qi < p.seq_q) {
+          const size_t o = (static_cast<size_t>(w.split) * p.num_units + w.bh(t)) * p.seq_q + qi;
+          p.ws_m[o] = (m_ref == -INFINITY) ? -INFINITY : m_ref * c;
+          p.ws_l[o] = l;
+        }
+      }
       mbar_arrive(L_FULL);
     }
     if (C::TURNS && t == 0) named_bar_sync(2 + 2 * quad, 64);  // consume tile 1's last hand-over
@@ -842,7 +873,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     const uint32_t lane_off = static_cast<uint32_t>(quad * 32) << 16;
     uint32_t ofc[2] = {0, 0}, lc[2] = {0, 0};
     for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
-      const WorkItem w = decode_item<PAIRX, VL>(p, idx);
+      const WorkItem w = decode_item<PAIRX, VL, SPLIT>(p, idx);
       // ------------------------------------------------------------ epilogue per tile (a9)
 #pragma unroll 1
       for (int t = 0; t < 2; ++t) {
@@ -879,6 +910,16 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             for (int k = 0; k < 32; ++k) o[k] = 0u;
           }
           const int col0 = 32 * q;
+          if constexpr (SPLIT) {  // unnormalised fp32 partial O of this split, rows inside the sequence
+            const int qi = w.row0(t) + row;
+            if (qi < p.seq_q) {
+              float* dst = p.ws_o + ((static_cast<size_t>(w.split) * p.num_units + w.bh(t)) * p.seq_q + qi) * D + col0;
+#pragma unroll
+              for (int u = 0; u < 8; ++u)
+                st_global_v4(dst + 4 * u, o[4 * u], o[4 * u + 1], o[4 * u + 2], o[4 * u + 3]);
+            }
+            continue;
+          }
           const uint32_t box = stg + (col0 / 64) * C::CHUNK + row * 128;
 #pragma unroll
           for (int u = 0; u < 4; ++u) {
@@ -899,7 +940,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           tc_fence_before();
           mbar_arrive(BAR(C::B_O_EMPTY + t));
         }
-        if (!rowwise) {
+        if (!rowwise && !SPLIT) {
           fence_proxy_async_smem();
           named_bar_sync(1, 128);
           if (row == 0) {

@@ -76,6 +76,13 @@ def test_validation_codes(lib):
     assert dg(16, 16, None, 16, None, 16, 4, 8, 16, 16, 1, None) == 1  # null A2
     assert dg(16, 16, 24, 16, None, 16, 4, 8, 16, 16, 1, None) == 3    # misaligned
     assert dg(16, 16, 16, 16, None, 16, 0, 8, 16, 16, 1, None) == 0    # M = 0
+    sk = lib.fmha_fwd_splitkv
+    assert sk(2, 16, 16, 16, 16, None, 1, 1, 8, 8, 64, 0.1, 2, 16, 1 << 20, None) == 2   # dtype
+    assert sk(0, 16, 16, 16, 16, None, 1, 1, 8, 8, 64, 0.1, -1, 16, 1 << 20, None) == 2  # splits
+    assert sk(0, 16, 16, 16, 16, None, 1, 1, 8, 8, 96, 0.1, 2, 16, 1 << 20, None) == 2   # head_dim
+    assert sk(0, 16, 16, 16, 16, None, 0, 1, 8, 8, 64, 0.1, 2, None, 0, None) == 0       # no work
+    assert lib.fmha_splitkv_workspace_bytes(2, 3, 5, 64, 4) == 4 * 2 * 3 * 5 * 66 * 4
+    assert lib.fmha_splitkv_workspace_bytes(2, 3, 5, 64, 1) == 0
     mf = lib.mlp_fused_fwd
     assert mf(16, 16, None, 16, 4, 96, 3, 1, None) == 2                # width not 64 / 128
     assert mf(16, 16, None, 16, 4, 128, 0, 1, None) == 2               # no layers

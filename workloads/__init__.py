@@ -73,6 +73,13 @@ CONFIGS = {
 }
 
 
+# split-KV: few (b, h) units, a short query block, long keys -- the shape where one
+# work item per (b, h, q-tile pair) leaves most SMs idle (decode / speculative-decode blocks)
+SPLITKV_CONFIGS = {
+    "decode_splitkv": FmhaConfig("decode_splitkv", 14, 4, 8, 16, 16384, 128, "bf16"),
+}
+
+
 @dataclass(frozen=True)
 class MlpConfig:
     name: str
