@@ -4,22 +4,25 @@
 // communication via the slower global memory", L453).  SURVEY §8(f) f4.
 //
 // Persistent, one CTA per SM.  A CTA owns S <= R row tiles of 128 rows at a time (a "group"; S is
-// a launch parameter, R the template's maximum: 4 at N = 128, 8 at N = 64) and walks them through
+// a launch parameter, R the template's maximum: 2 at N = 128, 4 at N = 64) and walks them through
 // all L layers in lockstep, so every W_l tile loaded into shared memory feeds S MMAs, and while one
 // tile's epilogue runs the tensor core works on the others (a layer of one tile is a serial chain
 // MMA -> epilogue -> next MMA; S tiles in flight hide it):
 //   warp 0        TMA producer: the group's X tiles into ACT[r], then W_1 .. W_L (WS-stage ring)
-//   warp 1 + r    MMA issuer of slot r: for each layer l, ACC_r = ACT[r] W_l^T (tcgen05.mma M=128
-//                 N=NW K=16, fp32 in TMEM columns [r NW, (r + 1) NW)); commit to ACC_FULL[r]
-//   last 16 warps four epilogue warpgroups.  Warpgroup w owns columns 64 h.. (h = w % H, H = N / 64)
-//                 of slots r = w / H, w / H + 4 / H, ... (thread = accumulator row): TMEM -> + b_l ->
-//                 act -> one RNE rounding -> swizzled st.shared back into ACT[r], which IS the next
-//                 layer's A operand (K-major SW128, the layout TMA produces); after layer L the same
-//                 buffer is TMA-stored to Y
+//   warp 1 + r    MMA issuer of slot r: for each layer l, ACC_r = h_{l-1} W_l^T (tcgen05.mma M=128
+//                 N=NW K=16, fp32 in TMEM columns [r NW, (r + 1) NW); layer 1 reads X from ACT[r] in
+//                 shared memory (SS form), later layers h_{l-1} from TMEM (TS form)); commit to ACC_FULL[r]
+//   last 16 warps four epilogue warpgroups.  Warpgroup w owns 64-column chunks h, h + H, ... of
+//                 slots r = w / H, w / H + 4 / H, ... (thread = accumulator row): TMEM -> + b_l ->
+//                 act -> one RNE rounding -> h_l, stored as the next layer's A operand:
+//                 TA (default): fp16 pairs into TMEM columns A_r (K-major, the TS-form MMA's A, as the
+//                   FMHA's P), so the MMA reads only W from shared memory;
+//                 else: swizzled st.shared back into ACT[r] (K-major SW128, the layout TMA produces).
+//                 After layer L, h_L goes to ACT[r] in shared memory and is TMA-stored to Y
 //
-//   smem  ACT[R] | W ring[WS] | fp32 bias ring   (N = 128: 4 x 32 KB + 3 x 32 KB + 2 KB;
-//                                                  N = 64: 8 x 16 KB + 4 x 8 KB + 2 KB)
-//   TMEM  ACC_r = columns [r NW, (r + 1) NW)   (R NW = 512)
+//   smem  ACT[R] (X in, Y out) | W ring[WS] | fp32 bias ring
+//   TMEM  ACC_r = columns [r NW, (r + 1) NW); TA: A_r = [R NW + r NW / 2, ...) (R = 2 at N = 128:
+//         384 of 512 columns; the shared-memory variant uses R = 512 / N accumulators)
 //
 // Barriers (every producer -> consumer edge has its consumer -> producer partner):
 //   X_FULL[r] / ACT_EMPTY[r]   TMA (X into ACT[r]) -> MMA;  the Y store out of ACT[r] has been read
@@ -47,26 +50,32 @@ struct MlpParams {
   int num_tiles;   // ceil(M / 128)
 };
 
-template <int NW>
+template <int NW, bool TA>
 struct MlpCfg {
-  static constexpr int R = 512 / NW;                  // slots: all of TMEM holds accumulators
+  // TA: the intermediates h_1..h_{L-1} live in TMEM as the A operand of a TS-form MMA (fp16 pairs,
+  // NW / 2 columns per slot) instead of shared memory; slots then need 1.5 NW columns each.
+  static constexpr int R = TA ? (NW == 128 ? 2 : 4) : 512 / NW;  // slots in flight per CTA
+  static constexpr int TMEM_A = R * NW;               // TA: A_r = columns [TMEM_A + r NW / 2, ...)
+  // epilogue warpgroups per slot (H = 1: one warpgroup drains all NW columns of a slot, 64 at a time;
+  // H = 2: two warpgroups, 64 columns each) -- one warpgroup per slot when there are 4 slots, so
+  // the four slots' epilogues run side by side
+  static constexpr int H = (TA && NW == 128) ? 2 : 1;
+  static constexpr int EPI_WG = 4;                    // epilogue warpgroups
+  static constexpr int SG = EPI_WG / H;               // slot groups: slot r -> warpgroups (r % SG) H + h
+  static constexpr int SPW = (R + SG - 1) / SG;       // slots per epilogue warpgroup
   static constexpr int CHUNK = 128 * 128;             // one SW128 box of 128 rows x 64 16-bit elements
   static constexpr int ATILE = 128 * NW * 2;          // 128 rows x NW
   static constexpr int WCHUNK = NW * 128;             // NW rows x 64 elements
   static constexpr int WTILE = NW * NW * 2;
-  static constexpr int WS = (NW == 128) ? 3 : 4;      // W ring stages
+  static constexpr int WS = (NW == 128) ? (TA ? 3 : 2) : 4;  // W ring stages (smem budget at N = 128)
   static constexpr int OFF_ACT = 0;
   static constexpr int OFF_W = OFF_ACT + R * ATILE;
   static constexpr int OFF_BIAS = OFF_W + WS * WTILE;  // fp32 b_l ring: [slot group][2][NW]
-  static constexpr int OFF_BAR = OFF_BIAS + (4 / (NW / 64)) * 2 * NW * 4;
+  static constexpr int OFF_BAR = OFF_BIAS + SG * 2 * NW * 4;
   // barriers: X_FULL[R], ACT_EMPTY[R], ACC_FULL[R], ACT_FULL[R], W_FULL[WS], W_EMPTY[WS]
   static constexpr int NUM_BARS = 4 * R + 2 * WS;
   static constexpr int OFF_TMEMPTR = OFF_BAR + NUM_BARS * 8;
   static constexpr int SMEM_ALLOC = OFF_TMEMPTR + 16;
-  static constexpr int H = NW / 64;                   // column halves (64 columns = one SW128 chunk)
-  static constexpr int EPI_WG = 4;                    // epilogue warpgroups
-  static constexpr int SG = EPI_WG / H;               // slot groups: slot r -> warpgroups (r % SG) H + h
-  static constexpr int SPW = R / SG;                  // slots per epilogue warpgroup
   // control warpgroups: warp 0 the TMA producer, warps 1..R one MMA issuer per slot (an mbarrier
   // wait of an issuing warp queues behind that warp's in-flight MMAs, so one warp walking all slots
   // left the tensor core idle between slots: measured ~420 cycles per slot)
@@ -81,9 +90,9 @@ struct MlpCfg {
   static_assert(SMEM_ALLOC <= 232448, "shared memory budget");
 };
 
-template <int NW, int ACT>
-__global__ void __launch_bounds__(MlpCfg<NW>::THREADS, 1) mlp_fused_kernel(const __grid_constant__ MlpParams p) {
-  using C = MlpCfg<NW>;
+template <int NW, int ACT, bool TA>
+__global__ void __launch_bounds__(MlpCfg<NW, TA>::THREADS, 1) mlp_fused_kernel(const __grid_constant__ MlpParams p) {
+  using C = MlpCfg<NW, TA>;
   constexpr int R = C::R;
   extern __shared__ __align__(1024) uint8_t smem[];
   const uint32_t sbase = smem_u32(smem);
@@ -183,10 +192,17 @@ __global__ void __launch_bounds__(MlpCfg<NW>::THREADS, 1) mlp_fused_kernel(const
             tc_fence_after();
             TRACE_EV(5, r * 64 + l);
             const uint32_t woff = C::OFF_W + s * C::WTILE;
+            if (TA && l > 0) {  // A = h_{l-1} in TMEM (K-major, fp16 pairs), W_l from shared memory
 #pragma unroll
-            for (int kk = 0; kk < NW / 16; ++kk)
-              umma_ss_elect(tmem + r * NW, desc0 + ((aoff + (kk / 4) * C::CHUNK + (kk % 4) * 32) >> 4),
-                            desc0 + ((woff + (kk / 4) * C::WCHUNK + (kk % 4) * 32) >> 4), IDESC, kk > 0);
+              for (int kk = 0; kk < NW / 16; ++kk)
+                umma_ts_elect(tmem + r * NW, tmem + C::TMEM_A + r * (NW / 2) + kk * 8,
+                              desc0 + ((woff + (kk / 4) * C::WCHUNK + (kk % 4) * 32) >> 4), IDESC, kk > 0);
+            } else {
+#pragma unroll
+              for (int kk = 0; kk < NW / 16; ++kk)
+                umma_ss_elect(tmem + r * NW, desc0 + ((aoff + (kk / 4) * C::CHUNK + (kk % 4) * 32) >> 4),
+                              desc0 + ((woff + (kk / 4) * C::WCHUNK + (kk % 4) * 32) >> 4), IDESC, kk > 0);
+            }
             umma_commit_elect(ACC_FULL(r));
             TRACE_EV(6, r * 64 + l);
             ++use;
@@ -204,26 +220,26 @@ __global__ void __launch_bounds__(MlpCfg<NW>::THREADS, 1) mlp_fused_kernel(const
     const int row = quad * 32 + lane;
     const uint32_t lane_off = static_cast<uint32_t>(quad * 32) << 16;
     constexpr uint32_t EPI_THREADS = 128 * C::H;  // threads writing one slot's ACT tile
+    constexpr int CPG = NW / C::H;                 // columns per warpgroup: chunks c = h, h + H, ...
     uint32_t use[C::SPW];
 #pragma unroll
     for (int j = 0; j < C::SPW; ++j) use[j] = 0;
-    auto bias_at = [&](int l) {
-      return p.bias ? __half2float(p.bias[static_cast<size_t>(l) * NW + 64 * h + (row & 63)]) : 0.f;
-    };
+    const int bcol = CPG * h + row;  // the bias column this thread converts (row < CPG)
+    auto bias_at = [&](int l) { return p.bias ? __half2float(p.bias[static_cast<size_t>(l) * NW + bcol]) : 0.f; };
     float bnext = 0.f;
     bool first = true;
     for (int g = blockIdx.x; g < p.num_groups; g += gridDim.x) {
       const int nt = ntiles(g);
       for (int l = 0; l < L; ++l) {
-        // b_l in fp32 for this slot group: thread (row < 64, h) converts column 64 h + row into the
+        // b_l in fp32 for this slot group: thread (row < CPG, h) converts column CPG h + row into the
         // ring entry l % 2 (its previous readers, layer l - 2, are past the last layer's barrier)
         const uint32_t bring = sbase + C::OFF_BIAS + (sg * 2 + (l & 1)) * NW * 4;
         // (its global load was issued one layer ahead, so the L2 latency is off the chain)
-        if (row < 64) {
+        if (row < CPG) {
           const float bv = first ? bias_at(l) : bnext;
           bnext = bias_at(l + 1 < L ? l + 1 : 0);
           first = false;
-          asm volatile("st.shared.f32 [%0], %1;" ::"r"(bring + (64 * h + row) * 4), "f"(bv) : "memory");
+          asm volatile("st.shared.f32 [%0], %1;" ::"r"(bring + bcol * 4), "f"(bv) : "memory");
         }
         named_bar_sync(1 + sg, EPI_THREADS);
 #pragma unroll
@@ -234,41 +250,58 @@ __global__ void __launch_bounds__(MlpCfg<NW>::THREADS, 1) mlp_fused_kernel(const
           TRACE_EV(1, r * 64 + l);
           ++use[j];
           tc_fence_after();
-          uint32_t v[64];
-          const uint32_t tacc = tmem + lane_off + r * NW + 64 * h;
-          tmem_ld_32x32b_x32(tacc, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
-          tmem_ld_32x32b_x32(tacc + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
-          tmem_wait_ld();
-          reg_fence(v);
-          TRACE_EV(2, r * 64 + l);
-          const uint32_t act_box = sbase + C::OFF_ACT + r * C::ATILE + h * C::CHUNK + row * 128;
-          const float4* bias4 = reinterpret_cast<const float4*>(smem + (bring - sbase)) + 16 * h;
+          const bool to_tmem = TA && l + 1 < L;  // h_l -> TMEM A_r (next layer's TS operand)
 #pragma unroll
-          for (int u = 0; u < 8; ++u) {  // 8 columns -> one 16-byte unit of the 128-byte row
-            // broadcast reads (every thread the same address), plain loads so the compiler can
-            // hoist them ahead of the previous unit's stores
-            const float4 b0 = bias4[2 * u], b1 = bias4[2 * u + 1];
-            const float bb[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
-            uint32_t pk[4];
+          for (int ci = 0; ci < NW / 64 / C::H; ++ci) {  // 64-column chunk c = SW128 chunk c of h_l
+            const int c = h + ci * C::H;
+            uint32_t v[64];
+            const uint32_t tacc = tmem + lane_off + r * NW + 64 * c;
+            tmem_ld_32x32b_x32(tacc, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+            tmem_ld_32x32b_x32(tacc + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
+            tmem_wait_ld();
+            reg_fence(v);
+            TRACE_EV(2, r * 64 + l);
+            const uint32_t act_box = sbase + C::OFF_ACT + r * C::ATILE + c * C::CHUNK + row * 128;
+            const float4* bias4 = reinterpret_cast<const float4*>(smem + (bring - sbase)) + 16 * c;
+            uint32_t pk[32];  // this chunk of h_l as fp16 pairs
+            // bias: broadcast reads (every thread the same address), software-pipelined one 8-column
+            // unit ahead so the shared-memory latency is off each unit's add -> convert -> store chain
+            float4 nb0 = bias4[0], nb1 = bias4[1];
 #pragma unroll
-            for (int e = 0; e < 4; ++e) {
-              const float2 x = fadd2(make_float2(__uint_as_float(v[8 * u + 2 * e]), __uint_as_float(v[8 * u + 2 * e + 1])),
-                                     make_float2(bb[2 * e], bb[2 * e + 1]));
-              if constexpr (ACT == 1) {
-                // ReLU inside the conversion: cvt.rn.relu clamps the rounded pair at 0 (rounding is
-                // monotonic and keeps 0, so this equals rounding max(x, 0))
-                asm("cvt.rn.relu.f16x2.f32 %0, %1, %2;" : "=r"(pk[e]) : "f"(x.y), "f"(x.x));
-              } else if constexpr (ACT == 0) {
-                pk[e] = pack2<false>(x.x, x.y);
-              } else {
-                pk[e] = pack2<false>(apply_act<ACT>(x.x), apply_act<ACT>(x.y));
+            for (int u = 0; u < 8; ++u) {  // 8 columns -> one 16-byte unit of the 128-byte row
+              const float4 b0 = nb0, b1 = nb1;
+              if (u + 1 < 8) {
+                nb0 = bias4[2 * u + 2];
+                nb1 = bias4[2 * u + 3];
               }
+              const float bb[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+              for (int e = 0; e < 4; ++e) {
+                const float2 x = fadd2(make_float2(__uint_as_float(v[8 * u + 2 * e]), __uint_as_float(v[8 * u + 2 * e + 1])),
+                                       make_float2(bb[2 * e], bb[2 * e + 1]));
+                uint32_t& d = pk[4 * u + e];
+                if constexpr (ACT == 1) {
+                  // ReLU inside the conversion: cvt.rn.relu clamps the rounded pair at 0 (rounding is
+                  // monotonic and keeps 0, so this equals rounding max(x, 0))
+                  asm("cvt.rn.relu.f16x2.f32 %0, %1, %2;" : "=r"(d) : "f"(x.y), "f"(x.x));
+                } else if constexpr (ACT == 0) {
+                  d = pack2<false>(x.x, x.y);
+                } else {
+                  d = pack2<false>(apply_act<ACT>(x.x), apply_act<ACT>(x.y));
+                }
+              }
+              if (!to_tmem)
+                asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(act_box + ((u ^ (row & 7)) << 4)),
+                             "r"(pk[4 * u]), "r"(pk[4 * u + 1]), "r"(pk[4 * u + 2]), "r"(pk[4 * u + 3]));
             }
-            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(act_box + ((u ^ (row & 7)) << 4)),
-                         "r"(pk[0]), "r"(pk[1]), "r"(pk[2]), "r"(pk[3]));
+            TRACE_EV(7, r * 64 + l);
+            if (to_tmem) {  // row `row`, K columns 64 c .. 64 c + 63 = TMEM columns A_r + 32 c ..
+              tmem_st_32x32b_x32(tmem + lane_off + C::TMEM_A + r * (NW / 2) + 32 * c, pk);
+              tmem_wait_st();
+            }
           }
           TRACE_EV(3, r * 64 + l);
-          fence_proxy_async_smem();  // h_l visible to the async proxy (tensor core operand reads, TMA store)
+          if (!TA || l + 1 == L) fence_proxy_async_smem();  // smem h_l visible to the async proxy
           tc_fence_before();
           mbar_arrive(ACT_FULL(r));
           TRACE_EV(4, r * 64 + l);
@@ -299,15 +332,15 @@ __global__ void __launch_bounds__(MlpCfg<NW>::THREADS, 1) mlp_fused_kernel(const
 int make_map_3d_rows(CUtensorMap* m, const void* base, uint64_t cols, uint64_t rows, uint64_t units,
                      uint32_t box_rows, char* err, size_t errlen);
 
-template <int NW>
+template <int NW, bool TA>
 inline int launch_mlp_fused_w(MlpParams& prm, int act, int sms, cudaStream_t stream, char* err, size_t errlen) {
-  using C = MlpCfg<NW>;
+  using C = MlpCfg<NW, TA>;
   constexpr int R = C::R;
-  void (*kern)(MlpParams) = act == 1 ? mlp_fused_kernel<NW, 1>
-                            : act == 2 ? mlp_fused_kernel<NW, 2>
-                            : act == 3 ? mlp_fused_kernel<NW, 3>
-                            : act == 4 ? mlp_fused_kernel<NW, 4>
-                                       : mlp_fused_kernel<NW, 0>;
+  void (*kern)(MlpParams) = act == 1 ? mlp_fused_kernel<NW, 1, TA>
+                            : act == 2 ? mlp_fused_kernel<NW, 2, TA>
+                            : act == 3 ? mlp_fused_kernel<NW, 3, TA>
+                            : act == 4 ? mlp_fused_kernel<NW, 4, TA>
+                                       : mlp_fused_kernel<NW, 0, TA>;
   static bool attr_done[64][5];
   int dev = 0;
   cudaGetDevice(&dev);
@@ -365,8 +398,16 @@ inline int launch_mlp_fused(const void* X, const void* W, const void* bias, void
   prm.M = M;
   prm.layers = L;
   prm.num_tiles = (M + 127) / 128;
-  return NW == 128 ? launch_mlp_fused_w<128>(prm, act, sms, stream, err, errlen)
-                   : launch_mlp_fused_w<64>(prm, act, sms, stream, err, errlen);
+  // h_l in TMEM (TS-form MMAs; 2 slots at N = 128, 4 at N = 64).  The shared-memory variant (4 / 8
+  // slots) measured 824 vs 887 TF/s at N = 128 (its SS MMAs and the epilogue's h_l stores compete
+  // for the SM's 128 B/clk of shared-memory bandwidth) and 406 vs 439 at N = 64;
+  // B200_MLP_VARIANT=1 selects it (A/B experiments only).
+  static const bool smem_a = getenv("B200_MLP_VARIANT") != nullptr;
+  if (NW == 128)
+    return smem_a ? launch_mlp_fused_w<128, false>(prm, act, sms, stream, err, errlen)
+                  : launch_mlp_fused_w<128, true>(prm, act, sms, stream, err, errlen);
+  return smem_a ? launch_mlp_fused_w<64, false>(prm, act, sms, stream, err, errlen)
+                : launch_mlp_fused_w<64, true>(prm, act, sms, stream, err, errlen);
 }
 
 }  // namespace b200

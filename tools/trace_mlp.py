@@ -15,7 +15,7 @@ import paper_conf_asplos_hagedornfccgg23_b200 as fm  # noqa: E402
 
 lib = _lib.load()
 lib.fmha_trace_set.argtypes = [ctypes.c_void_p]
-EV = {1: "EPI_ACC", 2: "EPI_LDTM", 3: "EPI_STS", 4: "EPI_ARRIVE", 5: "MMA_GO", 6: "MMA_COMMIT"}
+EV = {1: "EPI_ACC", 2: "EPI_LDTM", 3: "EPI_STS", 4: "EPI_ARRIVE", 5: "MMA_GO", 6: "MMA_COMMIT", 7: "EPI_MATH"}
 n, m = int(sys.argv[1]), int(sys.argv[2])
 L = 20
 x = torch.randn(m, n, device="cuda", dtype=torch.float16)
