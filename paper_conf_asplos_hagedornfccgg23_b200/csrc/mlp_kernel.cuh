@@ -83,7 +83,7 @@ struct MlpCfg {
   static constexpr int W_EPI = 4 * CW;                // first epilogue warp
   static constexpr int THREADS = 128 * CW + 128 * EPI_WG;
   static constexpr int REG_LAUNCH = (65536 / THREADS) / 8 * 8;
-  static constexpr int REG_CTRL = 40;
+  static constexpr int REG_CTRL = 48;
   static constexpr int REG_EPI = (REG_LAUNCH + (REG_LAUNCH - REG_CTRL) * CW / EPI_WG) / 8 * 8;
   static_assert(128 * CW * REG_CTRL + 128 * EPI_WG * REG_EPI <= THREADS * REG_LAUNCH, "register pool");
   static_assert(NW == 64 || NW == 128, "width");

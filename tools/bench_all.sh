@@ -3,7 +3,7 @@
 cd "$(dirname "$0")/.."
 mkdir -p gpurun_out
 : > gpurun_out/bench_all.jsonl
-for w in bert_large_512 bert_large_384 bert_base_pad gpt_causal tiny mlp; do
+for w in bert_large_512 bert_large_384 bert_base_pad gpt_causal tiny mlp bert_large_varlen bert_layer lstm_cell mlp_fused mlp_fused_w64 decode_splitkv; do
   timeout 300 python bench.py --workload $w --steps ${STEPS:-50} --warmup 5 --no-cpu-baseline --no-e2e \
     >> gpurun_out/bench_all.jsonl 2> gpurun_out/bench_all_$w.err || echo "{\"workload\": \"$w\", \"error\": true}" >> gpurun_out/bench_all.jsonl
 done

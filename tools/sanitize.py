@@ -1,0 +1,35 @@
+"""Small invocations of every kernel for compute-sanitizer (run via gpurun):
+    compute-sanitizer --tool {memcheck,racecheck,synccheck} python tools/sanitize.py"""
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_asplos_hagedornfccgg23_b200 as fm  # noqa: E402
+
+dev = torch.device("cuda:0")
+g = torch.Generator(device="cpu").manual_seed(0)
+r = lambda *s, dt=torch.float16: torch.randn(*s, generator=g).to(dt).to(dev)
+for d in (64, 128):
+    for dt in (torch.float16, torch.bfloat16):
+        q, k, v = r(1, 2, 200, d, dt=dt), r(1, 2, 300, d, dt=dt), r(1, 2, 300, d, dt=dt)
+        fm.fmha_fwd(q, k, v)
+        fm.fmha_fwd(q, k, v, causal=True)
+        fm.fmha_fwd(q, k, v, kv_len=torch.tensor([150], dtype=torch.int32, device=dev))
+        q3 = r(2, 2, 384, d, dt=dt)
+        fm.fmha_fwd(q3, q3, q3)  # pair_mode 1 (odd q-tile count)
+        fm.fmha_fwd_splitkv(q[:, :, :16].contiguous(), k, v, num_splits=3)
+qkv = r(300, 3, 4, 64)
+cu = torch.tensor([0, 100, 100, 300], dtype=torch.int32, device=dev)
+fm.fmha_fwd_varlen(qkv, cu, 200)
+fm.fmha_fwd_varlen(qkv, cu, 200, causal=True)
+a, w, b = r(300, 136), r(264, 136) * 0.1, r(264)
+fm.gemm_bias_act(a, w, b, act="gelu")
+fm.gemm_bias_act(r(600, 1024), r(1024, 1024) * 0.03, b.new_zeros(1024), act="relu")  # CTA-pair kernel
+fm.dual_gemm_bias_act(a, w, a, w, b, act="tanh")
+for n in (64, 128):
+    fm.mlp_fused(r(700, n), r(3, n, n) * 0.1, r(3, n))
+torch.cuda.synchronize()
+print("sanitize workload done")
