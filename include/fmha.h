@@ -101,7 +101,11 @@ FMHA_API int fmha_fwd_varlen(const void* QKV, void* O, const int32_t* cu_seqlens
 
 /* End-to-end variant: Q/K/V/O and kv_len are HOST buffers (pinned memory for asynchronous copies).
  * Copies Q, K, V (and kv_len) host->device into `workspace`, runs the same kernel, copies O
- * device->host, all enqueued on `stream` (no synchronisation: the caller syncs before reading O).
+ * device->host.  The work is ordered after everything already queued on `stream` and pipelined over
+ * up to 4 batch chunks on three streams created and released inside the call (the copy-in of chunk
+ * c+1 and the copy-out of chunk c-1 overlap the kernel on chunk c); `stream` is made to wait for the
+ * last copy-out, so syncing `stream` (no synchronisation happens inside) makes O complete on the host.
+ * Results are bitwise those of fmha_fwd (every (b, h) is independent of the batch it runs in).
  * dtype: 0 = fp16, 1 = bf16.  `workspace` is a DEVICE buffer of at least
  * fmha_workspace_bytes(batch, heads, seq_q, seq_kv, head_dim) bytes, 256-byte aligned.
  * For this entry point mask->kv_len is a HOST pointer. */

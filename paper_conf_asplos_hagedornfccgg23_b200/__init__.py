@@ -151,7 +151,7 @@ def fmha_fwd_from_host(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, out: t
                        workspace: torch.Tensor, kv_len: torch.Tensor | None = None, causal: bool = False,
                        scale: float | None = None, stream: torch.cuda.Stream | None = None) -> torch.Tensor:
     """End-to-end call with HOST (pinned) q/k/v/out and a device workspace: H2D copies, kernel and
-    D2H copy are all enqueued on ``stream`` by ``fmha_fwd_from_host`` of the C ABI (async; the
+    D2H copy are ordered after ``stream``'s queued work and joined back into it by ``fmha_fwd_from_host`` of the C ABI (async; the
     caller synchronises before reading ``out``)."""
     lib = _lib.load()
     b, h, sq, d = q.shape

@@ -436,14 +436,78 @@ int fmha_fwd_from_host(int dtype, const void* hQ, const void* hK, const void* hV
       dmask.kv_len = dL;
     }
   }
+  // Pipelined over batch chunks on three streams that live only for this call: the host->device
+  // copy of chunk c+1 and the device->host copy of chunk c-1 overlap the kernel on chunk c (PCIe is
+  // full duplex), ordered by events; `stream` waits for the last copy-out, so a caller that syncs
+  // `stream` sees O complete.  Each (b, h) is independent, so a chunk is just a smaller batch.
   cudaError_t e;
-  if ((e = cudaMemcpyAsync(dQ, hQ, qb, cudaMemcpyHostToDevice, stream)) != cudaSuccess) return cuda_fail(e, "H2D Q");
-  if ((e = cudaMemcpyAsync(dK, hK, kvb, cudaMemcpyHostToDevice, stream)) != cudaSuccess) return cuda_fail(e, "H2D K");
-  if ((e = cudaMemcpyAsync(dV, hV, kvb, cudaMemcpyHostToDevice, stream)) != cudaSuccess) return cuda_fail(e, "H2D V");
-  int st = fmha_common(dtype == 1, dQ, dK, dV, dO, &dmask, batch, heads, seq_q, seq_kv, head_dim, scale, stream);
-  if (st != FMHA_OK) return st;
-  if ((e = cudaMemcpyAsync(hO, dO, qb, cudaMemcpyDeviceToHost, stream)) != cudaSuccess) return cuda_fail(e, "D2H O");
-  return FMHA_OK;
+  const int chunks = std::min(batch, 4);
+  const size_t qb1 = qb / batch, kvb1 = kvb / batch;  // bytes per batch element
+  cudaStream_t sh = nullptr, sc = nullptr, sd = nullptr;
+  cudaEvent_t ev_start = nullptr, ev_h[8] = {}, ev_c[8] = {}, ev_d = nullptr;
+  auto cleanup = [&]() {
+    for (int c = 0; c < 8; ++c) {
+      if (ev_h[c]) cudaEventDestroy(ev_h[c]);
+      if (ev_c[c]) cudaEventDestroy(ev_c[c]);
+    }
+    if (ev_start) cudaEventDestroy(ev_start);
+    if (ev_d) cudaEventDestroy(ev_d);
+    if (sh) cudaStreamDestroy(sh);  // (returns at once; queued work still completes)
+    if (sc) cudaStreamDestroy(sc);
+    if (sd) cudaStreamDestroy(sd);
+  };
+  bool ok = cudaStreamCreateWithFlags(&sh, cudaStreamNonBlocking) == cudaSuccess &&
+            cudaStreamCreateWithFlags(&sc, cudaStreamNonBlocking) == cudaSuccess &&
+            cudaStreamCreateWithFlags(&sd, cudaStreamNonBlocking) == cudaSuccess &&
+            cudaEventCreateWithFlags(&ev_start, cudaEventDisableTiming) == cudaSuccess &&
+            cudaEventCreateWithFlags(&ev_d, cudaEventDisableTiming) == cudaSuccess;
+  for (int c = 0; ok && c < chunks; ++c)
+    ok = cudaEventCreateWithFlags(&ev_h[c], cudaEventDisableTiming) == cudaSuccess &&
+         cudaEventCreateWithFlags(&ev_c[c], cudaEventDisableTiming) == cudaSuccess;
+  if (!ok) {
+    e = cudaGetLastError();
+    cleanup();
+    return cuda_fail(e, "fmha_fwd_from_host streams/events");
+  }
+  // everything already queued on `stream` (incl. the kv_len copy) happens first
+  if ((e = cudaEventRecord(ev_start, stream)) != cudaSuccess ||
+      (e = cudaStreamWaitEvent(sh, ev_start, 0)) != cudaSuccess) {
+    cleanup();
+    return cuda_fail(e, "fmha_fwd_from_host ordering");
+  }
+  int st = FMHA_OK;
+  for (int c = 0; c < chunks && st == FMHA_OK; ++c) {
+    const int b0 = static_cast<int>(static_cast<long long>(batch) * c / chunks);
+    const int b1 = static_cast<int>(static_cast<long long>(batch) * (c + 1) / chunks);
+    const int nb = b1 - b0;
+    const size_t oq = b0 * qb1, okv = b0 * kvb1;
+    const uint8_t* hq = static_cast<const uint8_t*>(hQ) + oq;
+    const uint8_t* hk = static_cast<const uint8_t*>(hK) + okv;
+    const uint8_t* hv = static_cast<const uint8_t*>(hV) + okv;
+    if ((e = cudaMemcpyAsync(dQ + oq, hq, nb * qb1, cudaMemcpyHostToDevice, sh)) != cudaSuccess ||
+        (e = cudaMemcpyAsync(dK + okv, hk, nb * kvb1, cudaMemcpyHostToDevice, sh)) != cudaSuccess ||
+        (e = cudaMemcpyAsync(dV + okv, hv, nb * kvb1, cudaMemcpyHostToDevice, sh)) != cudaSuccess ||
+        (e = cudaEventRecord(ev_h[c], sh)) != cudaSuccess || (e = cudaStreamWaitEvent(sc, ev_h[c], 0)) != cudaSuccess) {
+      st = cuda_fail(e, "H2D chunk");
+      break;
+    }
+    fmha_mask_t cm = dmask;
+    if (cm.kv_len) cm.kv_len = dL + b0;
+    st = fmha_common(dtype == 1, dQ + oq, dK + okv, dV + okv, dO + oq, &cm, nb, heads, seq_q, seq_kv, head_dim, scale,
+                     sc);
+    if (st != FMHA_OK) break;
+    if ((e = cudaEventRecord(ev_c[c], sc)) != cudaSuccess || (e = cudaStreamWaitEvent(sd, ev_c[c], 0)) != cudaSuccess ||
+        (e = cudaMemcpyAsync(static_cast<uint8_t*>(hO) + oq, dO + oq, nb * qb1, cudaMemcpyDeviceToHost, sd)) !=
+            cudaSuccess) {
+      st = cuda_fail(e, "D2H chunk");
+      break;
+    }
+  }
+  // `stream` continues after the last copy-out (sd is in order, so it covers every chunk)
+  if ((e = cudaEventRecord(ev_d, sd)) != cudaSuccess || (e = cudaStreamWaitEvent(stream, ev_d, 0)) != cudaSuccess)
+    if (st == FMHA_OK) st = cuda_fail(e, "fmha_fwd_from_host join");
+  cleanup();
+  return st;
 }
 
 int gemm_bias_act(const void* A, const void* W, const void* bias, void* Cm, int M, int N, int K, int act,

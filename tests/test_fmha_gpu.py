@@ -150,9 +150,12 @@ def test_tiny_config_full_oracle():
     check(run(cfg, q, k, v, None), attention_fp64(q, k, v, cfg.scale), "fp16", "tiny")
 
 
-@pytest.mark.parametrize("name", ["bert_base_pad", "gpt_causal"])
-def test_from_host_entry_point_matches(name):
-    cfg = CONFIGS[name].with_(batch=2)
+@pytest.mark.parametrize("name,batch", [("bert_base_pad", 2), ("gpt_causal", 2), ("bert_base_pad", 5),
+                                        ("bert_large_384", 7), ("bert_base_pad", 19), ("tiny", 1)])
+def test_from_host_entry_point_matches(name, batch):
+    """fmha_fwd_from_host pipelines over up to 4 batch chunks on its own streams and joins `stream`:
+    bitwise equal to fmha_fwd, and complete after synchronising only the stream passed in."""
+    cfg = CONFIGS[name].with_(batch=batch)
     q, k, v, kl = make_fmha_inputs(cfg)
     o = run(cfg, q, k, v, kl)
     pq, pk, pv = q.pin_memory(), k.pin_memory(), v.pin_memory()
@@ -160,8 +163,10 @@ def test_from_host_entry_point_matches(name):
     ws = torch.empty(fm.workspace_bytes(cfg.batch, cfg.heads, cfg.seq_q, cfg.seq_kv, cfg.head_dim),
                      dtype=torch.uint8, device=DEV)
     klh = None if kl is None else torch.from_numpy(kl).pin_memory()
-    fm.fmha_fwd_from_host(pq, pk, pv, out, ws, kv_len=klh, causal=cfg.mask == MASK_CAUSAL, scale=cfg.scale)
     torch.cuda.synchronize()
+    s = torch.cuda.Stream(DEV)
+    fm.fmha_fwd_from_host(pq, pk, pv, out, ws, kv_len=klh, causal=cfg.mask == MASK_CAUSAL, scale=cfg.scale, stream=s)
+    s.synchronize()
     assert torch.equal(out, o.cpu())
 
 
