@@ -146,7 +146,17 @@ struct FmhaCfg {
   static constexpr int OFF_Q = 0;               // Q[stage][tile]
   static constexpr int OFF_RING = 2 * QS * TILE;
   static constexpr int OFF_STG = OFF_RING + NS * TILE;
-  static constexpr int OFF_LSUM = OFF_STG + NSTG * TILE;  // float l[2 tiles][128 rows]
+  // LSUM_MMA (D = 64): the row sum l comes out of the PV MMA -- V gets 16 extra columns of ones
+  // (a constant 16 KB SW128 atom that the V descriptor's leading-byte offset points at), so
+  // O_t[:, 64] = sum_k P[:, k]; P then overwrites S_t (as at D = 128) to make room in TMEM for the
+  // 80-column O_t.  The softmax threads drop their row-sum adds.
+#ifndef FMHA_LSUM_MMA
+#define FMHA_LSUM_MMA 0
+#endif
+  static constexpr bool LSUM_MMA = FMHA_LSUM_MMA && D == 64;
+  static constexpr int OW = LSUM_MMA ? D + 16 : D;  // O_t columns in TMEM (and PV MMA N)
+  static constexpr int OFF_ONES = OFF_STG + NSTG * TILE;  // LSUM_MMA: 128 x 64 ones (16 KB)
+  static constexpr int OFF_LSUM = OFF_ONES + (LSUM_MMA ? CHUNK : 0);  // float l[2 tiles][128 rows]
   static constexpr int OFF_MC = OFF_LSUM + 2 * 128 * 4;    // float mc[2 tiles][128 rows] (turn fence)
   static constexpr int OFF_BAR = OFF_MC + 2 * 128 * 4;
   // barrier slots
@@ -161,7 +171,7 @@ struct FmhaCfg {
   static constexpr int TMEM_COLS = 512;
   static constexpr int THREADS = 512;
   static constexpr int W_CORR = 8, W_MMA = 12, W_TMA = 14;  // first warp of each role
-  static constexpr bool SEP_P = (D == 64);
+  static constexpr bool SEP_P = (D == 64) && !LSUM_MMA;
   static constexpr int TMEM_P = 384;
   // registers after setmaxnreg.  setmaxnreg.inc only draws on the CTA's launch allocation
   // (128 x 512 = 65536), so 8 x 32 x 192 + 4 x 32 x 56 + 4 x 32 x 72 = 65536 must not be exceeded
@@ -185,6 +195,10 @@ struct FmhaCfg {
 #define FMHA_PRE_CHUNKS ((D == 128) ? 0 : 1)
 #endif
   static constexpr int PRE_CHUNKS = TURNS ? FMHA_PRE_CHUNKS : 4;
+#ifndef FMHA_DEFER_ST
+#define FMHA_DEFER_ST 0
+#endif
+  static constexpr int DEFER_ST = FMHA_DEFER_ST;
   static_assert(!TURNS || (PRE_CHUNKS >= 0 && PRE_CHUNKS < 4), "the turn barrier sits before chunk PRE_CHUNKS");
   // exp2 of element pairs q (of 64 per row) with (q % POLY_MOD) < POLY_CNT runs on the FMA pipe
   // (exp2_poly2) instead of MUFU: at D = 64 MUFU (16/clk/SM) is the bound.
@@ -454,6 +468,13 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     tma_prefetch_desc(&p.tmV);
     tma_prefetch_desc(&p.tmO);
   }
+  if constexpr (C::LSUM_MMA) {  // the ones atom for the row-sum columns of the PV MMA (1.0 in fp16 / bf16)
+    const uint32_t one2 = BF16 ? 0x3F803F80u : 0x3C003C00u;
+    const uint32_t a = sbase + C::OFF_ONES + threadIdx.x * 32;
+    st_shared_v4(a, one2, one2, one2, one2);
+    st_shared_v4(a + 16, one2, one2, one2, one2);
+    fence_proxy_async_smem();  // visible to the tensor core's operand reads
+  }
   if (warp == C::W_MMA) {
     tmem_alloc(smem_u32(tmem_holder), C::TMEM_COLS);
     tmem_relinquish();
@@ -520,12 +541,12 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       // PV) depends only on its own softmax warps.  Both warps release every K/V entry (count 2).
       const int t = warp - C::W_MMA;
       constexpr uint32_t IDESC_QK = idesc_f16(BF16, 128, 128, false, false);  // Q, K: K-major
-      constexpr uint32_t IDESC_PV = idesc_f16(BF16, 128, D, false, true);     // P: K-major (TMEM), V: MN-major
+      constexpr uint32_t IDESC_PV = idesc_f16(BF16, 128, C::OW, false, true);  // P: K-major (TMEM), V: MN-major
       // descriptors differ only in the start-address field: one base, plus (offset >> 4)
       const uint64_t desc0 = sdesc_sw128(sbase, 16, 1024);         // K-major Q / K tiles
       const uint64_t vdesc0 = sdesc_sw128(sbase, C::CHUNK, 1024);  // MN-major V tiles
       const uint32_t tS = tmem + 128 * t;
-      const uint32_t tO = tmem + 256 + t * D;
+      const uint32_t tO = tmem + 256 + t * C::OW;
       const uint32_t tP = tmem + (C::SEP_P ? C::TMEM_P + 64 * t : 128 * t);
       const uint32_t S_FULL = BAR(C::B_S_FULL + t), P_FULL = BAR(C::B_P_FULL + t);
       const uint32_t O_FULL = BAR(C::B_O_FULL + t), O_EMPTY = BAR(C::B_O_EMPTY + t);
@@ -624,9 +645,12 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         ++pc;
         TRACE_EV(EV_MMA_P, t * 64 + cu.j);
         tc_fence_after();
+        // LSUM_MMA: the second 64-column N chunk of B (columns 64..79 used) is the ones atom, one
+        // leading-byte offset above this ring slot
+        const uint64_t vdesc = C::LSUM_MMA ? sdesc_sw128(sbase, C::OFF_ONES - (sV - sbase), 1024) : vdesc0;
 #pragma unroll
         for (int kk = 0; kk < 8; ++kk)
-          umma_ts_elect(tO, tP + kk * 8, vdesc0 + ((sV - sbase + kk * 2048) >> 4), IDESC_PV, (cu.j > 0 || kk > 0));
+          umma_ts_elect(tO, tP + kk * 8, vdesc + ((sV - sbase + kk * 2048) >> 4), IDESC_PV, (cu.j > 0 || kk > 0));
         if (C::SEP_P) umma_commit_elect(PV_DONE);   // P_t may be overwritten
         if (cu.j + 1 == cu.w.n(t)) umma_commit_elect(O_FULL);  // O_t final: epilogue
         TRACE_EV(EV_MMA_PV, t * 64 + cu.j);
@@ -688,7 +712,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     const uint32_t S_FULL = BAR(C::B_S_FULL + t), P_FULL = BAR(C::B_P_FULL + t);
     const uint32_t PV_DONE = BAR(C::B_PV_DONE + t), S_FREE = BAR(C::B_S_FREE + t);
     const uint32_t L_FULL = BAR(C::B_L_FULL + t), L_EMPTY = BAR(C::B_L_EMPTY + t);
-    const uint32_t tO = tmem + lane_off + 256 + t * D;  // this row of O_t
+    const uint32_t tO = tmem + lane_off + 256 + t * C::OW;  // this row of O_t
     const uint32_t my_turn = 2 + 2 * quad + t, other_turn = 3 + 2 * quad - t;  // 64-thread barriers
     if (C::TURNS && t == 1) named_bar_arrive(2 + 2 * quad, 64);  // tile 0 goes first
     const float c = p.scale_log2;
@@ -769,6 +793,11 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         // interleave the chunks freely; per-chunk skipping on steps with masked columns
         auto exp_phase = [&](auto skip_tag) {
           constexpr bool SKIP = decltype(skip_tag)::value;
+          // DEFER_ST: the tcgen05.st of a post-turn chunk's P is issued after the next chunk's math
+          // (1: all at the end of the phase; 2: one chunk later) -- ptxas does not move MUFU work of
+          // a later chunk above a tcgen05.st, so storing each chunk right away left a burst of
+          // back-to-back MUFUs with nothing else to issue at the end of every chunk.
+          uint32_t pk_all[4][16];
 #pragma unroll
         for (int hh = 0; hh < 4; ++hh) {
           if (hh == C::PRE_CHUNKS) {
@@ -779,11 +808,13 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             named_bar_sync(my_turn, 64);
             asm volatile("ld.volatile.shared.f32 %0, [%1];" : "=f"(mcv) : "r"(slot) : "memory");
           }
-          uint32_t pk[16];
+          uint32_t (&pk)[16] = pk_all[hh];
+          const bool defer = C::DEFER_ST != 0 && hh >= C::PRE_CHUNKS;
+          if (C::DEFER_ST == 2 && hh > C::PRE_CHUNKS) tmem_st_32x32b_x16(tP + 16 * (hh - 1), pk_all[hh - 1]);
           if (SKIP && 32 * hh >= rem_w) {
 #pragma unroll
             for (int u = 0; u < 16; ++u) pk[u] = 0u;
-            tmem_st_32x32b_x16(tP + 16 * hh, pk);
+            if (!defer) tmem_st_32x32b_x16(tP + 16 * hh, pk);
             continue;
           }
 #pragma unroll
@@ -813,12 +844,20 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
               x1.x = ex2(x1.x);
               x1.y = ex2(x1.y);
             }
-            acc0 = fadd2(acc0, x0);
-            acc1 = fadd2(acc1, x1);
+            if constexpr (!C::LSUM_MMA) {  // (LSUM_MMA: the PV MMA sums P)
+              acc0 = fadd2(acc0, x0);
+              acc1 = fadd2(acc1, x1);
+            }
             pk[u] = pack2<BF16>(x0.x, x0.y);
             pk[u + 1] = pack2<BF16>(x1.x, x1.y);
           }
-          tmem_st_32x32b_x16(tP + 16 * hh, pk);
+          if (!defer) tmem_st_32x32b_x16(tP + 16 * hh, pk);
+        }
+        if constexpr (C::DEFER_ST == 1) {
+#pragma unroll
+          for (int hh = C::PRE_CHUNKS; hh < 4; ++hh) tmem_st_32x32b_x16(tP + 16 * hh, pk_all[hh]);
+        } else if constexpr (C::DEFER_ST == 2) {
+          tmem_st_32x32b_x16(tP + 16 * 3, pk_all[3]);
         }
         };
         if (rem_w >= 128)
@@ -840,6 +879,15 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             for (int k = 0; k < 32; ++k) o[k] = __float_as_uint(__uint_as_float(o[k]) * alpha);
             tmem_st_32x32b_x32(tO + 32 * q, o);
           }
+          if constexpr (C::LSUM_MMA) {  // the row-sum columns share O_t's reference
+            uint32_t o[16];
+            tmem_ld_32x32b_x16(tO + D, o);
+            tmem_wait_ld();
+            reg_fence(o);
+#pragma unroll
+            for (int k = 0; k < 16; ++k) o[k] = __float_as_uint(__uint_as_float(o[k]) * alpha);
+            tmem_st_32x32b_x16(tO + D, o);
+          }
         }
         tmem_wait_st();
         TRACE_EV(EV_EPI, j);  // P stores landed
@@ -859,7 +907,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         if (qi < p.seq_q) {
           const size_t o = (static_cast<size_t>(w.split) * p.num_units + w.bh(t)) * p.seq_q + qi;
           p.ws_m[o] = (m_ref == -INFINITY) ? -INFINITY : m_ref * c;
-          p.ws_l[o] = l;
+          if constexpr (!C::LSUM_MMA) p.ws_l[o] = l;  // (LSUM_MMA: the epilogue reads l from TMEM)
         }
       }
       mbar_arrive(L_FULL);
@@ -881,7 +929,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         mbar_wait_at(BAR(C::B_L_FULL + t), lc[t] & 1, 13, lc[t], idx);
         TRACE_EV(EV_EPI, 100 + t);
         ++lc[t];
-        const float l = s_lsum[t * 128 + row];
+        float l = s_lsum[t * 128 + row];
         mbar_arrive(BAR(C::B_L_EMPTY + t));
         const int n = w.n(t);
         if (n > 0) {
@@ -890,6 +938,19 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           ++ofc[t];
           tc_fence_after();
         }
+        if constexpr (C::LSUM_MMA) {  // l = O_t[row, D] (the ones column of the PV MMA)
+          l = 0.f;
+          if (n > 0) {
+            uint32_t lv[1];
+            tmem_ld_32x32b_x1(tmem + lane_off + 256 + t * C::OW + D, lv);
+            tmem_wait_ld();
+            l = __uint_as_float(lv[0]);
+          }
+          if constexpr (SPLIT) {
+            const int qi = w.row0(t) + row;
+            if (qi < p.seq_q) p.ws_l[(static_cast<size_t>(w.split) * p.num_units + w.bh(t)) * p.seq_q + qi] = l;
+          }
+        }
         const float inv_l = (l > 0.f) ? 1.f / l : 0.f;  // fully masked row -> 0 (R4)
         // varlen tile that crosses its sequence's end: a TMA store would overwrite the next
         // sequence's rows, so each thread stores its own row (if inside the sequence) instead
@@ -897,7 +958,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         const uint32_t stg = sbase + C::OFF_STG + (t % C::NSTG) * C::TILE;
         if (row == 0) tma_store_wait_read0();  // previous store out of this staging buffer done
         named_bar_sync(1, 128);
-        const uint32_t tO = tmem + lane_off + 256 + t * D;
+        const uint32_t tO = tmem + lane_off + 256 + t * C::OW;
 #pragma unroll 1
         for (int q = 0; q < D / 32; ++q) {
           uint32_t o[32];
