@@ -919,23 +919,25 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     const int quad = warp & 3;
     const int row = quad * 32 + lane;
     const uint32_t lane_off = static_cast<uint32_t>(quad * 32) << 16;
-    uint32_t ofc[2] = {0, 0}, lc[2] = {0, 0};
+    // phase parities of L_FULL / O_FULL per tile (bit t): registers, not a runtime-indexed array
+    // (which lived in local memory)
+    uint32_t ofbits = 0, lbits = 0;
     for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
       const WorkItem w = decode_item<PAIRX, VL, SPLIT>(p, idx);
       // ------------------------------------------------------------ epilogue per tile (a9)
 #pragma unroll 1
       for (int t = 0; t < 2; ++t) {
         if (!w.has(t)) continue;
-        mbar_wait_at(BAR(C::B_L_FULL + t), lc[t] & 1, 13, lc[t], idx);
+        mbar_wait_at(BAR(C::B_L_FULL + t), (lbits >> t) & 1, 13, t, idx);
         TRACE_EV(EV_EPI, 100 + t);
-        ++lc[t];
+        lbits ^= 1u << t;
         float l = s_lsum[t * 128 + row];
         mbar_arrive(BAR(C::B_L_EMPTY + t));
         const int n = w.n(t);
         if (n > 0) {
-          mbar_wait_at(BAR(C::B_O_FULL + t), ofc[t] & 1, 14, ofc[t], idx);  // last PV of this tile
+          mbar_wait_at(BAR(C::B_O_FULL + t), (ofbits >> t) & 1, 14, t, idx);  // last PV of this tile
           TRACE_EV(EV_EPI, 110 + t);
-          ++ofc[t];
+          ofbits ^= 1u << t;
           tc_fence_after();
         }
         if constexpr (C::LSUM_MMA) {  // l = O_t[row, D] (the ones column of the PV MMA)
