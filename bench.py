@@ -509,6 +509,15 @@ def run_varlen(args, world, rank, local):
         dist.destroy_process_group()
 
 
+def traffic_for(name):
+    """ncu DRAM bytes per launch of the workload's dominant kernel (profiles/traffic.json) or None."""
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        return json.load(open(tp)).get(name)
+    except Exception:
+        return None
+
+
 def _time_graph(fn, steps, stream):
     g = torch.cuda.CUDAGraph()
     with torch.cuda.graph(g):
@@ -799,7 +808,7 @@ def run_mlp_fused(args, world, rank, local):
             "clocks": sampler.summary(), "gpu_launches": args.steps,
             "roofline": {"bound": "tensor", "achieved": round(val, 2), "peak": peak_burst, "unit": "TFLOP/s",
                          "frac": round(val / peak_burst, 4), "peak_source": f"{src} bf16 dense burst",
-                         "kernel": "mlp_fused_kernel"},
+                         "kernel": "mlp_fused_kernel", "traffic": traffic_for(cfg.name)},
             "check_max_abs_err": err}), flush=True)
 
 
@@ -869,7 +878,8 @@ def run_splitkv(args, world, rank, local):
             "clocks": sampler.summary(), "gpu_launches": 2 * args.steps,
             "roofline": {"bound": "hbm", "achieved": round(gbs, 1), "peak": hbm, "unit": "GB/s",
                          "frac": round(gbs / hbm, 4), "peak_source": f"{src} HBM copy bandwidth",
-                         "kernel": "fmha_fwd_kernel (split) + fmha_splitkv_combine_kernel"},
+                         "kernel": "fmha_fwd_kernel (split) + fmha_splitkv_combine_kernel",
+                         "traffic": traffic_for(cfg.name)},
             "check_max_abs_err": err}), flush=True)
 
 
