@@ -28,6 +28,11 @@ Masking readings (the paper's FMHA has no mask; BASELINE.json configs add them):
       heads; query rows are computed regardless of kv_len.
   R6  causal is bottom-right aligned: key j is visible to query i iff
       j <= i + (Skv - Sq); with Sq == Skv this is j <= i.
+  R20 additive key bias (the HF BERT "extended attention mask"; SURVEY §8(f) f2
+      "arbitrary boolean/additive masks"): step 1 becomes
+      S = (Q @ K^T) * scale + bias[b, None, :], bias in natural-log units, shared by
+      all heads and queries of batch b; bias = -inf excludes the key (R3), and a row
+      whose every score is -inf yields O_i = 0 (R4).
 """
 
 from __future__ import annotations
@@ -60,7 +65,7 @@ def visible_mask(sq: int, skv: int, kv_len: int | None, causal: bool) -> np.ndar
 
 
 def softmax_probs_fp64(q_bh, k_bh, scale: float, kv_len: int | None = None,
-                       causal: bool = False) -> np.ndarray:
+                       causal: bool = False, key_bias=None) -> np.ndarray:
     """Steps 1-6 for one (b,h): the row-stochastic matrix P [Sq, Skv] (rows of zeros
     where every key is masked, R4).  Exposed so tests can pin sum_j P[i,j] = 1."""
     q = _as_f64(q_bh)
@@ -68,6 +73,10 @@ def softmax_probs_fp64(q_bh, k_bh, scale: float, kv_len: int | None = None,
     sq, skv = q.shape[0], k.shape[0]
     s = (q @ k.T) * _scale_f64(scale)                       # step 1 (GEMM #1, scale)
     vis = visible_mask(sq, skv, kv_len, causal)
+    if key_bias is not None:                                 # R20: additive key bias
+        kb = np.asarray(key_bias, dtype=np.float64)[:skv]
+        s = s + kb[None, :]
+        vis = vis & (kb > -np.inf)[None, :]
     s = np.where(vis, s, -np.inf)                            # step 2 (mask)
     any_vis = vis.any(axis=1)
     m = np.where(any_vis, s.max(axis=1, initial=-np.inf), 0.0)  # step 3 (max reduction)
@@ -77,10 +86,11 @@ def softmax_probs_fp64(q_bh, k_bh, scale: float, kv_len: int | None = None,
     return p
 
 
-def attention_fp64(q, k, v, scale: float, kv_len=None, causal: bool = False) -> np.ndarray:
+def attention_fp64(q, k, v, scale: float, kv_len=None, causal: bool = False, key_bias=None) -> np.ndarray:
     """O = softmax(scale * Q K^T + mask) V for Q:[B,H,Sq,D], K,V:[B,H,Skv,D].
 
-    ``kv_len`` is None or a length-B integer sequence (R5).  Returns float64
+    ``kv_len`` is None or a length-B integer sequence (R5); ``key_bias`` None or
+    [B, >= Skv] additive bias (R20).  Returns float64
     [B,H,Sq,D].  One (b,h) at a time, exactly steps 1-7 above.
     """
     q = _as_f64(q)
@@ -93,13 +103,14 @@ def attention_fp64(q, k, v, scale: float, kv_len=None, causal: bool = False) -> 
     for b in range(b_):
         kl = None if kv_len is None else int(kv_len[b])
         for h in range(h_):
-            p = softmax_probs_fp64(q[b, h], k[b, h], scale, kl, causal)
+            kb = None if key_bias is None else np.asarray(key_bias, dtype=np.float64)[b]
+            p = softmax_probs_fp64(q[b, h], k[b, h], scale, kl, causal, kb)
             out[b, h] = p @ v[b, h]                          # step 7 (GEMM #2)
     return out
 
 
 def attention_rows_fp64(q, k, v, scale: float, units, kv_len=None,
-                        causal: bool = False) -> np.ndarray:
+                        causal: bool = False, key_bias=None) -> np.ndarray:
     """Steps 1-7 for a sample of output rows only: ``units`` is a list of
     (b, h, i) triples; returns float64 [len(units), D].  Used for parity at full
     BASELINE sizes, where the whole oracle would take too long on the sampled
@@ -114,6 +125,10 @@ def attention_rows_fp64(q, k, v, scale: float, units, kv_len=None,
         kl = None if kv_len is None else int(kv_len[b])
         s = (qi @ kb.T)[0] * _scale_f64(scale)
         vis = visible_mask(sq, skv, kl, causal)[i]
+        if key_bias is not None:                             # R20
+            bb = np.asarray(key_bias, dtype=np.float64)[b][:skv]
+            s = s + bb
+            vis = vis & (bb > -np.inf)
         if not vis.any():
             res.append(np.zeros(vb.shape[1]))
             continue

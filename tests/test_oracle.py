@@ -492,3 +492,60 @@ def test_mlp_tolerance_covers_fp32_kernel_model():
     assert not (d > 1e-3 * (1 + np.sqrt(20)) + 2 ** -8 * np.abs(ref)).any()
     assert np.linalg.norm(d) / np.linalg.norm(ref) <= 1e-3
     assert (d > 2e-3 + 2 ** -9 * np.abs(ref)).any()
+
+
+# ---------------------------------------------------------------------------------------------
+# Additive key bias (R20): pins for attention_fp64(..., key_bias=)
+
+
+def _bias_case(seed=0, b=2, h=2, sq=5, skv=7, d=4):
+    rng = np.random.default_rng(seed)
+    q = rng.standard_normal((b, h, sq, d)).astype(np.float16)
+    k = rng.standard_normal((b, h, skv, d)).astype(np.float16)
+    v = rng.uniform(-1, 1, (b, h, skv, d)).astype(np.float16)
+    return q, k, v
+
+
+@pytest.mark.parametrize("seed", [0, 1])
+def test_key_bias_brute_force(seed):
+    q, k, v = _bias_case(seed)
+    rng = np.random.default_rng(100 + seed)
+    kb = rng.uniform(-3, 3, (2, 7))
+    kb[1, 2] = -np.inf
+    got = attention_fp64(q, k, v, 0.5, key_bias=kb)
+    want = np.array(attention_brute(q.astype(np.float64).tolist(), k.astype(np.float64).tolist(),
+                                    v.astype(np.float64).tolist(), 0.5, key_bias=kb.tolist()))
+    np.testing.assert_allclose(got, want, rtol=0, atol=1e-12)
+
+
+def test_key_bias_special_cases():
+    q, k, v = _bias_case(3)
+    base = attention_fp64(q, k, v, 0.5)
+    # zero bias = no mask; a constant bias cancels in the softmax (shift invariance)
+    np.testing.assert_allclose(attention_fp64(q, k, v, 0.5, key_bias=np.zeros((2, 7))), base, rtol=0, atol=1e-14)
+    np.testing.assert_allclose(attention_fp64(q, k, v, 0.5, key_bias=np.full((2, 7), 123.25)), base, rtol=0, atol=1e-12)
+    # -inf past kv_len is exactly key padding (R5)
+    kl = np.array([7, 3])
+    kb = np.where(np.arange(7)[None, :] < kl[:, None], 0.0, -np.inf)
+    np.testing.assert_array_equal(attention_fp64(q, k, v, 0.5, key_bias=kb), attention_fp64(q, k, v, 0.5, kv_len=kl))
+    # all keys excluded -> zero rows (R4)
+    assert not attention_fp64(q, k, v, 0.5, key_bias=np.full((2, 7), -np.inf)).any()
+
+
+def test_key_bias_reweighting_closed_form():
+    """scale = 0: the weights are softmax(bias), so bias = log w gives O_i = sum_j w_j v_j / sum_j w_j."""
+    q, k, v = _bias_case(4)
+    w = np.array([[1.0, 2.0, 0.5, 4.0, 1.0, 3.0, 0.25], [2.0, 2.0, 2.0, 1.0, 1.0, 1.0, 8.0]])
+    got = attention_fp64(q, k, v, 0.0, key_bias=np.log(w))
+    vv = v.astype(np.float64)
+    want = np.einsum("bj,bhjd->bhd", w / w.sum(1, keepdims=True), vv)[:, :, None, :].repeat(5, axis=2)
+    np.testing.assert_allclose(got, want, rtol=0, atol=1e-12)
+
+
+def test_key_bias_rows_sampler_matches_full():
+    q, k, v = _bias_case(5)
+    kb = np.random.default_rng(6).uniform(-2, 2, (2, 7))
+    full = attention_fp64(q, k, v, 0.25, key_bias=kb)
+    units = [(0, 0, 0), (1, 1, 4), (0, 1, 2)]
+    np.testing.assert_allclose(attention_rows_fp64(q, k, v, 0.25, units, key_bias=kb),
+                               np.stack([full[b, h, i] for b, h, i in units]), rtol=0, atol=1e-13)
