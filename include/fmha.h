@@ -20,7 +20,13 @@
  *   FMHA_MASK_KEY_PADDING  key j visible iff j < kv_len[b] (right padding, shared by all heads).
  *                          kv_len is a DEVICE int32 array [batch]; values are clamped to [0, seq_kv].
  *   FMHA_MASK_CAUSAL       key j visible iff j <= i + (seq_kv - seq_q)  (bottom-right aligned).
- * A query row with no visible key produces O = 0 (never NaN).
+ *   FMHA_MASK_KEY_BIAS     additive per-key bias (the HF BERT "extended attention mask"; DESIGN.md
+ *                          R20): S[i,j] = scale * <q_i, k_j> + key_bias[b * key_bias_stride + j],
+ *                          natural-log units, shared by all heads and queries of batch b; -inf
+ *                          excludes the key.  key_bias: DEVICE fp32, 16-byte aligned;
+ *                          key_bias_stride >= seq_kv and a multiple of 4; scale must be > 0.
+ *                          fmha_fwd / fmha_fwd_bf16 only (other entry points: FMHA_ERR_UNSUPPORTED).
+ * The kinds are exclusive.  A query row with no visible key produces O = 0 (never NaN).
  *
  * Ownership and errors: every tensor pointer is caller-owned; the library never allocates device
  * memory, never synchronises the stream and retains no pointer past the call (kv_len must stay
@@ -58,11 +64,18 @@ typedef enum {
   FMHA_ERR_NO_DEVICE = 5    /* no sm_100 device is current                                    */
 } fmha_status_t;
 
-typedef enum { FMHA_MASK_NONE = 0, FMHA_MASK_KEY_PADDING = 1, FMHA_MASK_CAUSAL = 2 } fmha_mask_kind_t;
+typedef enum {
+  FMHA_MASK_NONE = 0,
+  FMHA_MASK_KEY_PADDING = 1,
+  FMHA_MASK_CAUSAL = 2,
+  FMHA_MASK_KEY_BIAS = 3
+} fmha_mask_kind_t;
 
 typedef struct {
-  int32_t kind;          /* fmha_mask_kind_t                                          */
-  const int32_t* kv_len; /* DEVICE pointer, [batch]; required for KEY_PADDING, else ignored */
+  int32_t kind;            /* fmha_mask_kind_t                                                 */
+  const int32_t* kv_len;   /* DEVICE pointer, [batch]; required for KEY_PADDING, else ignored  */
+  const float* key_bias;   /* DEVICE pointer, [batch, key_bias_stride]; KEY_BIAS only          */
+  int32_t key_bias_stride; /* elements between batches of key_bias; KEY_BIAS only              */
 } fmha_mask_t;
 
 /* FMHA forward, fp16 in / fp16 out.

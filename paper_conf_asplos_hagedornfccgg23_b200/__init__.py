@@ -26,7 +26,7 @@ from ._lib import FmhaError, FmhaMask
 __all__ = ["fmha_fwd", "fmha_fwd_splitkv", "fmha_fwd_varlen", "fmha_fwd_from_host", "gemm_bias_act", "dual_gemm_bias_act", "mlp_fused", "transformer_layer", "layer_workspace_bytes", "workspace_bytes", "FmhaError",
            "MASK_NONE", "MASK_KEY_PADDING", "MASK_CAUSAL", "ACTS", "version"]
 
-MASK_NONE, MASK_KEY_PADDING, MASK_CAUSAL = 0, 1, 2
+MASK_NONE, MASK_KEY_PADDING, MASK_CAUSAL, MASK_KEY_BIAS = 0, 1, 2, 3
 ACTS = {"none": 0, "relu": 1, "gelu": 2, "gelu_erf": 2, "gelu_tanh": 3, "tanh": 4}
 
 
@@ -49,10 +49,13 @@ def _mask(kv_len, causal: bool):
 
 
 def fmha_fwd(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, kv_len: torch.Tensor | None = None,
-             causal: bool = False, scale: float | None = None, out: torch.Tensor | None = None) -> torch.Tensor:
+             causal: bool = False, scale: float | None = None, out: torch.Tensor | None = None,
+             key_bias: torch.Tensor | None = None) -> torch.Tensor:
     """O = softmax(scale * Q K^T + mask) V.  q: [B,H,Sq,D], k/v: [B,H,Skv,D] contiguous CUDA
-    fp16/bf16 tensors; kv_len: CUDA int32 [B] (key padding) or None; causal: bottom-right mask.
-    Calls ``fmha_fwd`` / ``fmha_fwd_bf16`` of the C ABI on the current stream."""
+    fp16/bf16 tensors; kv_len: CUDA int32 [B] (key padding) or None; causal: bottom-right mask;
+    key_bias: CUDA fp32 [B, stride >= Skv] additive per-key bias (stride % 4 == 0; -inf excludes a
+    key), exclusive with the other masks.  Calls ``fmha_fwd`` / ``fmha_fwd_bf16`` of the C ABI on
+    the current stream."""
     lib = _lib.load()
     if q.dtype not in (torch.float16, torch.bfloat16) or k.dtype != q.dtype or v.dtype != q.dtype:
         raise TypeError("q, k, v must share dtype fp16 or bf16")
@@ -71,7 +74,16 @@ def fmha_fwd(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, kv_len: torch.Te
     if out is None:
         out = torch.empty_like(q)
     scale = 1.0 / math.sqrt(d) if scale is None else float(scale)
-    m = _mask(kv_len, causal)
+    if key_bias is not None:
+        if kv_len is not None or causal:
+            raise ValueError("key_bias is exclusive with kv_len / causal")
+        if key_bias.dtype != torch.float32 or not key_bias.is_cuda or key_bias.dim() != 2 or key_bias.shape[0] != b:
+            raise ValueError("key_bias must be a CUDA float32 tensor [batch, stride]")
+        if key_bias.stride(1) != 1:
+            raise ValueError("key_bias rows must be contiguous")
+        m = FmhaMask(MASK_KEY_BIAS, None, key_bias.data_ptr(), key_bias.stride(0))
+    else:
+        m = _mask(kv_len, causal)
     fn = lib.fmha_fwd if q.dtype == torch.float16 else lib.fmha_fwd_bf16
     st = fn(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), ctypes.byref(m), b, h, sq, skv, d,
             scale, _stream_ptr(q.device))

@@ -45,7 +45,8 @@ EXPORTED_SYMBOLS = (
 
 
 class FmhaMask(ctypes.Structure):
-    _fields_ = [("kind", ctypes.c_int32), ("kv_len", ctypes.c_void_p)]
+    _fields_ = [("kind", ctypes.c_int32), ("kv_len", ctypes.c_void_p), ("key_bias", ctypes.c_void_p),
+                ("key_bias_stride", ctypes.c_int32)]
 
 
 class FmhaError(RuntimeError):

@@ -127,14 +127,16 @@ template <int D, bool BF16>
 int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) {
   using C = b200::FmhaCfg<D>;
   const int mode = prm.num_splits > 1 ? b200::MODE_SPLIT
+                   : prm.key_bias   ? b200::MODE_BIAS
                    : prm.cu_seqlens ? (prm.sched ? b200::MODE_VARLEN_SCHED : b200::MODE_VARLEN)
                                     : (prm.pair_mode ? b200::MODE_PAIRX : b200::MODE_DENSE);
   void (*kern)(b200::FmhaParams) = mode == b200::MODE_DENSE    ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_DENSE>
                                    : mode == b200::MODE_PAIRX  ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_PAIRX>
                                    : mode == b200::MODE_VARLEN ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_VARLEN>
                                    : mode == b200::MODE_SPLIT  ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_SPLIT>
+                                   : mode == b200::MODE_BIAS   ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_BIAS>
                                                                : b200::fmha_fwd_sm100<D, BF16, b200::MODE_VARLEN_SCHED>;
-  static bool attr_done[64][5];
+  static bool attr_done[64][6];
   int dev = 0;
   cudaGetDevice(&dev);
   if (dev >= 64 || !attr_done[dev][mode]) {
@@ -195,13 +197,20 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   if (head_dim != 64 && head_dim != 128) return FMHA_ERR_UNSUPPORTED;
   if (scale < 0.f) return FMHA_ERR_UNSUPPORTED;
   const int kind = mask ? mask->kind : FMHA_MASK_NONE;
-  if (kind != FMHA_MASK_NONE && kind != FMHA_MASK_KEY_PADDING && kind != FMHA_MASK_CAUSAL)
+  if (kind != FMHA_MASK_NONE && kind != FMHA_MASK_KEY_PADDING && kind != FMHA_MASK_CAUSAL &&
+      kind != FMHA_MASK_KEY_BIAS)
     return FMHA_ERR_UNSUPPORTED;
+  if (kind == FMHA_MASK_KEY_BIAS) {  // (R20) fmha_fwd / fmha_fwd_bf16 only; the bias is added as bias / scale
+    if (splits != 1 || !(scale > 0.f)) return FMHA_ERR_UNSUPPORTED;
+    if (mask->key_bias_stride < seq_kv || (mask->key_bias_stride % 4) != 0) return FMHA_ERR_INVALID_ARG;
+  }
   const long long units = static_cast<long long>(batch) * heads;
   if (units == 0 || seq_q == 0) return FMHA_OK;
   if (seq_kv == 0) return FMHA_ERR_INVALID_ARG;
   if (!Q || !K || !V || !O) return FMHA_ERR_INVALID_ARG;
   if (kind == FMHA_MASK_KEY_PADDING && !mask->kv_len) return FMHA_ERR_INVALID_ARG;
+  if (kind == FMHA_MASK_KEY_BIAS && !mask->key_bias) return FMHA_ERR_INVALID_ARG;
+  if (kind == FMHA_MASK_KEY_BIAS && !aligned16(mask->key_bias)) return FMHA_ERR_MISALIGNED;
   if (!aligned16(Q) || !aligned16(K) || !aligned16(V) || !aligned16(O)) return FMHA_ERR_MISALIGNED;
   if (units > 2147483647LL || static_cast<long long>(seq_q) * head_dim * units * 2 > (1LL << 40))
     return FMHA_ERR_INVALID_ARG;
@@ -230,7 +239,14 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   // odd q-tile counts >= 3 (non-causal): pair tiles across units so no item has an empty second
   // tile (BERT-large-384: +8%).  With a single q-tile per unit (short sequences) every item is one
   // latency-bound step and pairing across units measured slower, so those keep pair_mode 0.
-  prm.pair_mode = (kind != FMHA_MASK_CAUSAL && (prm.num_q_tiles & 1) && prm.num_q_tiles >= 3) ? 1 : 0;
+  prm.pair_mode = (kind != FMHA_MASK_CAUSAL && kind != FMHA_MASK_KEY_BIAS && (prm.num_q_tiles & 1) &&
+                   prm.num_q_tiles >= 3) ? 1 : 0;
+  if (kind == FMHA_MASK_KEY_BIAS) {
+    prm.key_bias = mask->key_bias;
+    prm.key_bias_stride = mask->key_bias_stride;
+    prm.inv_scale = 1.f / scale;
+    prm.mask_kind = FMHA_MASK_NONE;  // no key bound beyond seq_kv; the bias does the masking
+  }
   const long long items = prm.pair_mode ? (units * prm.num_q_tiles + 1) / 2 : units * ((prm.num_q_tiles + 1) / 2);
   if (items > 2147483647LL || units * prm.num_q_tiles > 2147483647LL) return FMHA_ERR_UNSUPPORTED;
   prm.num_items = static_cast<int>(items);
@@ -426,7 +442,8 @@ int fmha_fwd_from_host(int dtype, const void* hQ, const void* hK, const void* hV
   uint8_t* dK = dO + round_up(qb, 256);
   uint8_t* dV = dK + round_up(kvb, 256);
   int32_t* dL = reinterpret_cast<int32_t*>(dV + round_up(kvb, 256));
-  fmha_mask_t dmask = {FMHA_MASK_NONE, nullptr};
+  fmha_mask_t dmask = {FMHA_MASK_NONE, nullptr, nullptr, 0};
+  if (mask && mask->kind == FMHA_MASK_KEY_BIAS) return FMHA_ERR_UNSUPPORTED;  // (fmha_fwd only)
   if (mask) {
     dmask.kind = mask->kind;
     if (mask->kind == FMHA_MASK_KEY_PADDING) {

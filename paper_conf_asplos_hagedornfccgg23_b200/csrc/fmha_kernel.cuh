@@ -67,7 +67,7 @@ __device__ unsigned int g_fmha_trace_n = 0;
 enum : int { EV_S_WAIT = 1, EV_S_READY, EV_MAX_DONE, EV_XCHG, EV_EXP_DONE, EV_MMA_P, EV_MMA_O, EV_MMA_PV,
              EV_MMA_QK, EV_COR_ST, EV_COR_PV, EV_COR_ORDY, EV_EPI, EV_TMA_KV, EV_ITEM };
 
-enum : int { MASK_NONE = 0, MASK_KEY_PADDING = 1, MASK_CAUSAL = 2 };
+enum : int { MASK_NONE = 0, MASK_KEY_PADDING = 1, MASK_CAUSAL = 2, MASK_KEY_BIAS = 3 };
 
 // Division by a launch constant without the integer-divide sequence (whose MUFU.RCP would queue
 // behind the softmax's exponentials): q = (umulhi(n, m) + n) >> s, exact for 0 <= n < 2^31.
@@ -132,6 +132,11 @@ struct FmhaParams {
   float* ws_o;   // [num_splits][num_units][seq_q][D]
   float* ws_m;   // [num_splits][num_units][seq_q]
   float* ws_l;   // [num_splits][num_units][seq_q]
+  // Additive key bias (MODE_BIAS; R20): raw scores get key_bias[b][j] / scale added, so
+  // c * s' = c * s + log2(e) * bias and the rest of the softmax is unchanged.
+  const float* key_bias;
+  int key_bias_stride;
+  float inv_scale;
 };
 
 template <int D>
@@ -416,13 +421,13 @@ __device__ __forceinline__ int item_at(const FmhaParams& p, const SchedTable* tb
 // Kernel instances (MODE): dense [B,H,S,D]; dense with cross-unit tile pairing (pair_mode 1, see
 // FmhaParams::pair_mode); varlen packed; varlen packed with the cost-sorted schedule.  Separate
 // instances keep the varlen and scheduling code out of the dense kernels entirely.
-enum : int { MODE_DENSE = 0, MODE_PAIRX = 1, MODE_VARLEN = 2, MODE_VARLEN_SCHED = 3, MODE_SPLIT = 4 };
+enum : int { MODE_DENSE = 0, MODE_PAIRX = 1, MODE_VARLEN = 2, MODE_VARLEN_SCHED = 3, MODE_SPLIT = 4, MODE_BIAS = 5 };
 
 template <int D, bool BF16, int MODE>
 __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
   using C = FmhaCfg<D>;
   constexpr bool PAIRX = MODE == MODE_PAIRX, VL = MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
-                 SCHED = MODE == MODE_VARLEN_SCHED, SPLIT = MODE == MODE_SPLIT;
+                 SCHED = MODE == MODE_VARLEN_SCHED, SPLIT = MODE == MODE_SPLIT, BIAS = MODE == MODE_BIAS;
   // Dynamic shared memory starts at the (1024-byte aligned) base of the CTA's shared window; the
   // SWIZZLE_128B tiles need that alignment.  Using the base directly keeps smem addresses uniform.
   extern __shared__ __align__(1024) uint8_t smem[];
@@ -754,6 +759,35 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         const int rem = lim - (w.jb + j) * 128;
         // 32-key chunks no row of this warp can see are skipped: their P is stored as zeros
         const int rem_w = lim_w - (w.jb + j) * 128;
+        if constexpr (BIAS) {  // s' = s + bias / scale (R20), 32 keys at a time; L1-resident, the
+                               // next step's keys prefetched (every softmax warp reads the same row)
+          const int b = p.div_heads.div(w.bh(t));
+          const float* brow = p.key_bias + static_cast<size_t>(b) * p.key_bias_stride;
+          const int key0 = (w.jb + j) * 128;
+          if (key0 + 128 < p.seq_kv) asm volatile("prefetch.global.L1 [%0];" ::"l"(brow + key0 + 128));
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            float4 bq[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+              const int col = key0 + 32 * q + 4 * u;
+              bq[u] = col < p.seq_kv ? __ldg(reinterpret_cast<const float4*>(brow + col)) : make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+              const int k = 32 * q + 4 * u;
+              const float2 is2 = make_float2(p.inv_scale, p.inv_scale);
+              const float2 a = ffma2(make_float2(bq[u].x, bq[u].y), is2,
+                                     make_float2(__uint_as_float(s[k]), __uint_as_float(s[k + 1])));
+              const float2 bb2 = ffma2(make_float2(bq[u].z, bq[u].w), is2,
+                                       make_float2(__uint_as_float(s[k + 2]), __uint_as_float(s[k + 3])));
+              s[k] = __float_as_uint(a.x);
+              s[k + 1] = __float_as_uint(a.y);
+              s[k + 2] = __float_as_uint(bb2.x);
+              s[k + 3] = __float_as_uint(bb2.y);
+            }
+          }
+        }
         if (rem < 128) {  // boundary tile for this row (a5)
 #pragma unroll
           for (int k = 0; k < 128; ++k)

@@ -61,6 +61,11 @@ def test_validation_codes(lib):
     assert call_fmha(lib, mask=_lib.FmhaMask(7, None)) == 2
     assert call_fmha(lib, q=None) == 1
     assert call_fmha(lib, mask=_lib.FmhaMask(1, None)) == 1           # KEY_PADDING needs kv_len
+    assert call_fmha(lib, mask=_lib.FmhaMask(3, None, None, 8)) == 1   # KEY_BIAS needs key_bias
+    assert call_fmha(lib, mask=_lib.FmhaMask(3, None, 16, 6)) == 1     # stride % 4
+    assert call_fmha(lib, mask=_lib.FmhaMask(3, None, 16, 4)) == 1     # stride < seq_kv
+    assert call_fmha(lib, mask=_lib.FmhaMask(3, None, 24, 8)) == 3     # misaligned bias
+    assert call_fmha(lib, mask=_lib.FmhaMask(3, None, 16, 8), scale=0.0) == 2  # bias / scale needs scale > 0
     assert call_fmha(lib, q=24) == 3                                   # 8-byte aligned only
     assert call_fmha(lib, skv=0) == 1
     # zero work: OK without touching the device
