@@ -247,7 +247,17 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
     prm.inv_scale = 1.f / scale;
     prm.mask_kind = FMHA_MASK_NONE;  // no key bound beyond seq_kv; the bias does the masking
   }
-  const long long items = prm.pair_mode ? (units * prm.num_q_tiles + 1) / 2 : units * ((prm.num_q_tiles + 1) / 2);
+  long long items = prm.pair_mode ? (units * prm.num_q_tiles + 1) / 2 : units * ((prm.num_q_tiles + 1) / 2);
+  prm.single_from = 0x7fffffff;
+  if (prm.pair_mode) {  // a last, partial round of tile pairs runs as single tiles (half as long)
+    const long long tiles = units * prm.num_q_tiles;
+    const long long full = items / sm_count * sm_count;  // pair items in full rounds
+    const long long rest = tiles - 2 * full;              // tiles left for the last round
+    if (full > 0 && rest > 0 && rest <= sm_count) {
+      prm.single_from = static_cast<int>(full);
+      items = full + rest;
+    }
+  }
   if (items > 2147483647LL || units * prm.num_q_tiles > 2147483647LL) return FMHA_ERR_UNSUPPORTED;
   prm.num_items = static_cast<int>(items);
   prm.div_units.init(static_cast<uint32_t>(std::max(prm.num_units, 1)));

@@ -117,6 +117,7 @@ struct FmhaParams {
   int num_q_tiles;
   int num_units;  // B*H
   int num_items;  // see pair_mode
+  int single_from;  // pair_mode 1: items >= single_from hold one tile (see decode_item)
   int pair_mode;  // 0: items are q-tiles {2i, 2i+1} of one unit (num_units * ceil(num_q_tiles / 2) items)
                   // 1: items are tiles {2i, 2i+1} of the flattened (unit, q-tile) list, so a tile pair
                   //    may straddle two units (odd num_q_tiles, non-causal): no half-empty items
@@ -291,12 +292,16 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
     w.r0 = qt0 * 128;
     w.r1 = w.r0 + 128;
   } else {
-    const int a = 2 * idx, b = 2 * idx + 1;
+    // items < single_from pair tiles {2 idx, 2 idx + 1}; later items (the last, partial round of
+    // the static schedule) are single tiles, so that round takes about half as long
+    const bool single = idx >= p.single_from;
+    const int a = single ? 2 * p.single_from + (idx - p.single_from) : 2 * idx;
+    const int b = single ? a : a + 1;
     w.bh0 = p.div_qtiles.div(a);
     qt0 = a - w.bh0 * p.num_q_tiles;
     w.bh1 = p.div_qtiles.div(b);
     const int qt1 = b - w.bh1 * p.num_q_tiles;
-    w.has1 = b < p.num_units * p.num_q_tiles;
+    w.has1 = !single && b < p.num_units * p.num_q_tiles;
     w.shared = w.has1 && w.bh1 == w.bh0;
     w.r0 = qt0 * 128;
     w.r1 = qt1 * 128;
