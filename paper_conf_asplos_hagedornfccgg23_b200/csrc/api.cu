@@ -5,6 +5,7 @@
 
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <algorithm>
 #include <mutex>
@@ -23,6 +24,7 @@ int cuda_fail(cudaError_t e, const char* where) {
   snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "%s: %s", where, cudaGetErrorString(e));
   return FMHA_ERR_CUDA;
 }
+
 
 using EncodeTiledFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                    const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
@@ -146,8 +148,9 @@ int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) 
   }
   // persistent: one CTA per SM (or fewer when there is less work)
   dim3 grid(static_cast<unsigned>(std::min(prm.num_items, sm_count)), 1, 1);
-  kern<<<grid, C::THREADS, C::SMEM_ALLOC, stream>>>(prm);
-  cudaError_t e = cudaGetLastError();
+  // PDL measured: +0.5% (BERT-large-512) to +4.5% (BERT-base, padded); -5% on the varlen schedule
+  const bool pdl = mode != b200::MODE_VARLEN && mode != b200::MODE_VARLEN_SCHED;
+  cudaError_t e = b200::launch_pdl(pdl, kern, grid, dim3(C::THREADS), C::SMEM_ALLOC, stream, prm);
   if (e != cudaSuccess) return cuda_fail(e, "fmha_fwd_kernel launch");
   if (mode == b200::MODE_SPLIT) {  // merge the splits into O (same stream, so after the kernel)
     const long long rows = static_cast<long long>(prm.num_units) * prm.seq_q;

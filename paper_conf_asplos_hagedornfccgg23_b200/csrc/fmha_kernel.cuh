@@ -489,6 +489,9 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     tmem_alloc(smem_u32(tmem_holder), C::TMEM_COLS);
     tmem_relinquish();
   }
+  // PDL: the setup above overlaps the previous kernel's tail; global memory only from here on
+  pdl_wait();
+  pdl_trigger();
   const SchedTable* sched = reinterpret_cast<const SchedTable*>(smem + C::OFF_SCHED);
   if (SCHED && warp == C::W_TMA + 1) build_sched(p, reinterpret_cast<SchedTable*>(smem + C::OFF_SCHED), lane);
   tc_fence_before();

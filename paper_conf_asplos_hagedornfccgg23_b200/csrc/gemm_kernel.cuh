@@ -157,6 +157,8 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
+  pdl_wait();  // global memory only from here on (PDL)
+  pdl_trigger();
   const uint32_t tmem = *tmem_holder;
 
   if (warp == 0) {
@@ -344,6 +346,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
   tc_fence_before();
   cluster_sync_all();  // both CTAs' barriers initialised and TMEM allocated before any signal crosses
   tc_fence_after();
+  pdl_wait();  // global memory only from here on (PDL)
+  pdl_trigger();
   const uint32_t tmem = *tmem_holder;
   if (warp == 1) tmem_relinquish_2sm();
 
@@ -526,8 +530,8 @@ inline int launch_gemm_bias_act(const void* A, const void* W, const void* A2, co
       if (dev2 < 64) attr2[dev2][act] = true;
     }
     const long long clusters = std::min<long long>(pair_tiles, sms / 2);
-    k2<<<static_cast<unsigned>(2 * clusters), Gemm2Cfg::THREADS, Gemm2Cfg::SMEM_ALLOC, stream>>>(prm);
-    cudaError_t e = cudaGetLastError();
+    cudaError_t e = launch_pdl(true, k2, dim3(static_cast<unsigned>(2 * clusters)), dim3(Gemm2Cfg::THREADS),
+                               Gemm2Cfg::SMEM_ALLOC, stream, prm);
     if (e != cudaSuccess) {
       snprintf(err, errlen, "gemm_bias_act_2sm_kernel launch: %s", cudaGetErrorString(e));
       return 4;
@@ -557,8 +561,7 @@ inline int launch_gemm_bias_act(const void* A, const void* W, const void* A2, co
   prm.split_from = static_cast<int>(tiles - split);
   prm.num_units = static_cast<int>(tiles + split);
   dim3 grid(static_cast<unsigned>(tiles < sms ? tiles : sms), 1, 1);
-  kern<<<grid, GemmCfg::THREADS, GemmCfg::SMEM_ALLOC, stream>>>(prm);
-  cudaError_t e = cudaGetLastError();
+  cudaError_t e = launch_pdl(true, kern, grid, dim3(GemmCfg::THREADS), GemmCfg::SMEM_ALLOC, stream, prm);
   if (e != cudaSuccess) {
     snprintf(err, errlen, "gemm_bias_act_kernel launch: %s", cudaGetErrorString(e));
     return 4;

@@ -134,6 +134,8 @@ __global__ void __launch_bounds__(MlpCfg<NW, TA>::THREADS, 1) mlp_fused_kernel(c
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
+  pdl_wait();  // global memory only from here on (PDL)
+  pdl_trigger();
   const uint32_t tmem = *tmem_holder;
   // tiles of group g: g * S + r for r < ntiles(g)
   auto ntiles = [&](int g) { return min(S, p.num_tiles - g * S); };
@@ -376,8 +378,7 @@ inline int launch_mlp_fused_w(MlpParams& prm, int act, int sms, cudaStream_t str
   }
   prm.num_groups = (prm.num_tiles + prm.slots - 1) / prm.slots;
   const int grid = std::min(prm.num_groups, sms);
-  kern<<<grid, C::THREADS, C::SMEM_ALLOC, stream>>>(prm);
-  cudaError_t e = cudaGetLastError();
+  cudaError_t e = launch_pdl(true, kern, dim3(grid), dim3(C::THREADS), C::SMEM_ALLOC, stream, prm);
   if (e != cudaSuccess) {
     snprintf(err, errlen, "mlp_fused_kernel launch: %s", cudaGetErrorString(e));
     return 4;

@@ -10,6 +10,8 @@
 #include <cuda_fp16.h>
 #include <cuda_bf16.h>
 #include <cstdio>
+#include <cstdlib>
+#include <cuda_runtime.h>
 
 #include "tmem_ops.cuh"
 
@@ -132,6 +134,44 @@ __device__ __forceinline__ void tma_store_wait0() { asm volatile("cp.async.bulk.
 // Generic-proxy smem writes -> visible to the async proxy (TMA store / UMMA reads).
 __device__ __forceinline__ void fence_proxy_async_smem() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+// ------------------------------------------------------------------ programmatic dependent launch
+// A kernel launched with cudaLaunchAttributeProgrammaticStreamSerialization may start while the
+// previous kernel on the stream is still running: everything before pdl_wait() (barrier init, TMEM
+// allocation, descriptor prefetch) overlaps that kernel's tail.  pdl_wait() returns once every
+// prerequisite grid has completed and its memory is visible; no global memory is read or written
+// before it.  pdl_trigger() lets the next PDL launch on the stream start scheduling its CTAs.
+// Both are no-ops for an ordinary launch.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
+// Host side of programmatic dependent launch (PDL) for the persistent kernels: the next kernel's prologue
+// (barrier init, TMEM allocation, descriptor prefetch) overlaps the previous kernel's tail; the
+// kernel's pdl_wait() orders every global access after the previous grid.  B200_PDL=0 turns it off
+// (A/B measurements).
+inline bool pdl_enabled() {
+  static const bool on = [] {
+    const char* v = std::getenv("B200_PDL");
+    return !(v && v[0] == '0');
+  }();
+  return on;
+}
+
+template <typename... Args>
+inline cudaError_t launch_pdl(bool use, void (*kern)(Args...), dim3 grid, dim3 block, size_t smem,
+                              cudaStream_t stream, Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = use && pdl_enabled() ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, kern, args...);
 }
 
 // ------------------------------------------------------------------ named barriers
