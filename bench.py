@@ -62,6 +62,24 @@ def measured_peaks():
     return 1590.0, 1400.0, 6650.0, "fallback"
 
 
+def fmha_roofline(achieved_tf, ai, ms_step, bytes_step, traffic, peak_tf, hbm_gbs, peak_src) -> dict:
+    """Roofline of the dense FMHA kernel: arithmetic intensity AI = algorithmic flops /
+    algorithmic bytes (Q + K + V + O).  Below the measured ridge (peak TFLOP/s / HBM GB/s, ~258 flop/B)
+    the bound is HBM and the line reports GB/s against the measured copy bandwidth (BERT-base padded,
+    AI <= 64; BERT-large-384, AI 192); at or above it (BERT-large-512, AI 256 -- 1% below the ridge,
+    where the two roofs coincide within 1%; GPT causal) the tensor peak."""
+    kernel = "fmha_fwd_kernel"
+    if ai * hbm_gbs / 1e3 < 0.97 * peak_tf:
+        gbs = bytes_step / (ms_step * 1e-3) / 1e9
+        return {"bound": "hbm", "achieved": round(gbs, 1), "peak": hbm_gbs, "unit": "GB/s",
+                "frac": round(gbs / hbm_gbs, 4), "traffic": traffic, "arith_intensity": round(ai, 1),
+                "peak_source": f"{peak_src} HBM copy bandwidth", "kernel": kernel,
+                "tensor_frac": round(achieved_tf / peak_tf, 4)}
+    return {"bound": "tensor", "achieved": round(achieved_tf, 2), "peak": peak_tf, "unit": "TFLOP/s",
+            "frac": round(achieved_tf / peak_tf, 4), "traffic": traffic, "arith_intensity": round(ai, 1),
+            "peak_source": f"{peak_src} bf16 dense burst (fp16 = bf16 rate)", "kernel": kernel}
+
+
 class ClockSampler:
     """Samples SM clock and throttle reasons through NVML while the timed region runs."""
 
@@ -309,10 +327,8 @@ def main():
             "clocks": sampler.summary(),
             "e2e": e2e,
             "gpu_launches": args.steps,
-            "roofline": {"bound": "tensor", "achieved": round(achieved, 2), "peak": peak_burst, "unit": "TFLOP/s",
-                         "frac": round(achieved / peak_burst, 4), "traffic": traffic,
-                         "peak_source": f"{peak_src} bf16 dense burst (fp16 = bf16 rate)",
-                         "kernel": "fmha_fwd_kernel"},
+            "roofline": fmha_roofline(achieved, flops_rank / alg_bytes(cfg), ms_step, alg_bytes(cfg),
+                                      traffic, peak_burst, hbm, peak_src),
             "roofline_exp": exp_roofline(alg_flops(cfg, kv_len) / (4.0 * cfg.head_dim), ms_step, sampler),
             "cpu_baseline": cpu,
             "check_max_abs_err": check_err,
@@ -469,7 +485,7 @@ def run_varlen(args, world, rank, local):
         a, b = int(cu[s_]), int(cu[s_ + 1])
         ref = attention_varlen_fp64(x[a:b], np.array([0, b - a]), cfg.scale, cfg.causal)
         err = max(err, float(np.abs(o_last[a:b].double().cpu().numpy() - ref).max()))
-    peak_burst, _, _, peak_src = measured_peaks()
+    peak_burst, _, hbm, peak_src = measured_peaks()
     if dist:
         dist.barrier()
     if rank == 0:
@@ -486,6 +502,7 @@ def run_varlen(args, world, rank, local):
             cpu = {"value": done / el / 1e12, "unit": "TFLOP/s", "cores": os.cpu_count(), "kind": "oracle",
                    "sample": f"{k} whole sequences (all heads) of {cfg.name}, numpy fp64, {el:.1f} s"}
         achieved = flops_rank / (ms_step * 1e-3) / 1e12
+        vl_bytes = 4.0 * int(cu[-1]) * cfg.heads * cfg.head_dim * 2  # packed Q, K, V read + O written
         line = {
             "metric": METRIC, "value": round(value, 2), "unit": "TFLOP/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 5),
@@ -498,10 +515,8 @@ def run_varlen(args, world, rank, local):
                        "l2": f"rotating {n_sets} input/output sets ({n_sets * set_bytes / 1e6:.0f} MB > 126 MB L2)"},
             "pct_of_spec_2250": round(100 * achieved / SPEC_TFLOPS, 2),
             "clocks": sampler.summary(), "e2e": e2e, "gpu_launches": args.steps,
-            "roofline": {"bound": "tensor", "achieved": round(achieved, 2), "peak": peak_burst, "unit": "TFLOP/s",
-                         "frac": round(achieved / peak_burst, 4), "traffic": None,
-                         "peak_source": f"{peak_src} bf16 dense burst (fp16 = bf16 rate)",
-                         "kernel": "fmha_fwd_kernel (varlen)"},
+            "roofline": dict(fmha_roofline(achieved, flops_rank / vl_bytes, ms_step, vl_bytes, None, peak_burst, hbm,
+                                           peak_src), kernel="fmha_fwd_kernel (varlen)"),
             "cpu_baseline": cpu, "check_max_abs_err": err,
         }
         print(json.dumps(line), flush=True)

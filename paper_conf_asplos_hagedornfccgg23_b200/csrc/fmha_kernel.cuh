@@ -195,6 +195,16 @@ struct FmhaCfg {
 #define FMHA_TURNS 1
 #endif
   static constexpr bool TURNS = FMHA_TURNS;
+  // Split S load: max of the first 64 columns overlaps the TMEM load of the last 64 (A/B knob)
+#ifndef FMHA_SPLIT_LD
+#define FMHA_SPLIT_LD 0
+#endif
+  static constexpr bool SPLIT_LD = FMHA_SPLIT_LD;
+  // Prefetch S_{t,j+1} into registers at the end of step j, before P_FULL (separate P only)
+#ifndef FMHA_PREFETCH_S
+#define FMHA_PREFETCH_S 0
+#endif
+  static constexpr bool PREFETCH_S = FMHA_PREFETCH_S && SEP_P && !SPLIT_LD;
   // The first PRE_CHUNKS of the four 32-column chunks of a row are exponentiated before the turn
   // (overlapping the other tile's turn), the rest inside it.
 #ifndef FMHA_PRE_CHUNKS
@@ -744,22 +754,63 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       const int lim_w = __reduce_max_sync(0xffffffffu, lim);  // keys >= lim_w: masked for the warp
       float m_ref = -INFINITY;  // max used as the exp2 reference (lags the true max by < 2^8)
       float l = 0.f;            // row sum relative to m_ref
+      uint32_t s[128];  // this row's scores S_{t,j}
+      bool pre = false;  // PREFETCH_S: S_{t,j} already requested into s
       for (int j = 0; j < N; ++j) {
         if (j >= n) {  // no KV tile j for this tile: pass the turn on
           named_bar_sync(my_turn, 64);
+          TRACE_EV(EV_XCHG, 100 + j);
           named_bar_arrive(other_turn, 64);
           continue;
         }
-        TRACE_EV(EV_S_WAIT, j);
-        mbar_wait_at(S_FULL, g & 1, 8, g, idx);
-        TRACE_EV(EV_S_READY, j);
-        tc_fence_after();
-        uint32_t s[128];
+        if (!pre) {
+          TRACE_EV(EV_S_WAIT, j);
+          mbar_wait_at(S_FULL, g & 1, 8, g, idx);
+          TRACE_EV(EV_S_READY, j);
+          tc_fence_after();
+          if constexpr (C::PREFETCH_S) {
 #pragma unroll
-        for (int q = 0; q < 4; ++q)
-          tmem_ld_32x32b_x32(tS + 32 * q, *reinterpret_cast<uint32_t(*)[32]>(&s[32 * q]));
-        tmem_wait_ld();
-        reg_fence(s);
+            for (int q = 0; q < 4; ++q)
+              tmem_ld_32x32b_x32(tS + 32 * q, *reinterpret_cast<uint32_t(*)[32]>(&s[32 * q]));
+          }
+        }
+        if constexpr (C::PREFETCH_S) {
+          tmem_wait_ld();
+          reg_fence(s);
+        }
+        // SPLIT_LD: load the first 64 columns, wait, start the second 64 and take the first half's
+        // max while they land (the max of the second half follows the second wait)
+        float mxh = -INFINITY;
+        if constexpr (C::PREFETCH_S) {
+          // (loaded above)
+        } else if constexpr (C::SPLIT_LD) {
+          tmem_ld_32x32b_x32(tS, *reinterpret_cast<uint32_t(*)[32]>(&s[0]));
+          tmem_ld_32x32b_x32(tS + 32, *reinterpret_cast<uint32_t(*)[32]>(&s[32]));
+          tmem_wait_ld();
+          reg_fence(*reinterpret_cast<uint32_t(*)[64]>(&s[0]));
+          tmem_ld_32x32b_x32(tS + 64, *reinterpret_cast<uint32_t(*)[32]>(&s[64]));
+          tmem_ld_32x32b_x32(tS + 96, *reinterpret_cast<uint32_t(*)[32]>(&s[96]));
+          const int rem0 = lim - (w.jb + j) * 128;
+          if (!BIAS && rem0 >= 64) {
+            float a0 = -INFINITY, a1 = -INFINITY, a2 = -INFINITY, a3 = -INFINITY;
+#pragma unroll
+            for (int k = 0; k < 64; k += 8) {
+              a0 = fmax3(a0, __uint_as_float(s[k]), __uint_as_float(s[k + 1]));
+              a1 = fmax3(a1, __uint_as_float(s[k + 2]), __uint_as_float(s[k + 3]));
+              a2 = fmax3(a2, __uint_as_float(s[k + 4]), __uint_as_float(s[k + 5]));
+              a3 = fmax3(a3, __uint_as_float(s[k + 6]), __uint_as_float(s[k + 7]));
+            }
+            mxh = fmaxf(fmaxf(a0, a1), fmaxf(a2, a3));
+          }
+          tmem_wait_ld();
+          reg_fence(*reinterpret_cast<uint32_t(*)[64]>(&s[64]));
+        } else {
+#pragma unroll
+          for (int q = 0; q < 4; ++q)
+            tmem_ld_32x32b_x32(tS + 32 * q, *reinterpret_cast<uint32_t(*)[32]>(&s[32 * q]));
+          tmem_wait_ld();
+          reg_fence(s);
+        }
         if (C::SEP_P) {  // S_t read: the tensor core may overwrite it with S_{t,j+1}
           tc_fence_before();
           mbar_arrive(S_FREE);
@@ -801,9 +852,12 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           for (int k = 0; k < 128; ++k)
             if (k >= rem) s[k] = __float_as_uint(-INFINITY);
         }
-        float mx0 = m_ref, mx1 = -INFINITY, mx2 = -INFINITY, mx3 = -INFINITY;
+        // (SPLIT_LD: the first 64 columns' max is mxh when none of them is masked, else recomputed)
+        const int k_max0 = (C::SPLIT_LD && mxh != -INFINITY) ? 64 : 0;
+        float mx0 = fmaxf(m_ref, mxh), mx1 = -INFINITY, mx2 = -INFINITY, mx3 = -INFINITY;
 #pragma unroll
         for (int k = 0; k < 128; k += 8) {
+          if (C::SPLIT_LD && k < k_max0) continue;
           mx0 = fmax3(mx0, __uint_as_float(s[k]), __uint_as_float(s[k + 1]));
           mx1 = fmax3(mx1, __uint_as_float(s[k + 2]), __uint_as_float(s[k + 3]));
           mx2 = fmax3(mx2, __uint_as_float(s[k + 4]), __uint_as_float(s[k + 5]));
@@ -848,6 +902,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             const uint32_t slot = sbase + C::OFF_MC + (t * 128 + row) * 4;
             asm volatile("st.shared.f32 [%0], %1;" ::"r"(slot), "f"(mc) : "memory");
             named_bar_sync(my_turn, 64);
+            TRACE_EV(EV_XCHG, j);  // turn granted
             asm volatile("ld.volatile.shared.f32 %0, [%1];" : "=f"(mcv) : "r"(slot) : "memory");
           }
           uint32_t (&pk)[16] = pk_all[hh];
@@ -930,6 +985,19 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             for (int k = 0; k < 16; ++k) o[k] = __float_as_uint(__uint_as_float(o[k]) * alpha);
             tmem_st_32x32b_x16(tO + D, o);
           }
+        }
+        // PREFETCH_S: request S_{t,j+1} before releasing P_{t,j}, so its TMEM load overlaps the P
+        // stores draining and the loop turnaround.  Safe only with a separate P buffer: QK_{t,j+1} is
+        // then issued before PV_{t,j} (it waits for S_FREE_{t,j}, not for P_FULL_{t,j}), and its K
+        // tile never waits for a V slot released by PV_{t,j} (ring order, NS = 6).
+        // Only when S_{t,j+1} is already there (a blocking wait here would hold back P_FULL_{t,j}).
+        pre = C::PREFETCH_S && j + 1 < n && __all_sync(0xffffffffu, mbar_try_wait(S_FULL, g & 1));
+        if (pre) {
+          TRACE_EV(EV_S_READY, j + 1);
+          tc_fence_after();
+#pragma unroll
+          for (int q = 0; q < 4; ++q)
+            tmem_ld_32x32b_x32(tS + 32 * q, *reinterpret_cast<uint32_t(*)[32]>(&s[32 * q]));
         }
         tmem_wait_st();
         TRACE_EV(EV_EPI, j);  // P stores landed
