@@ -190,3 +190,57 @@ def test_back_to_back_launches_do_not_hang(name, batch):
             first = out.clone()
     torch.cuda.synchronize()
     assert torch.equal(out, first)
+
+
+# ------------------------------------------------------------------ programmatic dependent launch
+@pytest.mark.timeout(240)
+def test_pdl_chained_launches_keep_stream_order():
+    """Launches overlap their prologue with the previous kernel (PDL), but every global access sits
+    behind griddepcontrol.wait.  RAW: the second FMHA reads the first one's output as its Q.  WAR:
+    the third writes its output into the buffer the second one read.  Both must match the same
+    computations separated by full synchronisations, bit for bit, on every repetition."""
+    cfg = CONFIGS["bert_large_512"].with_(batch=4)
+    q, k, v, _ = make_fmha_inputs(cfg)
+    qd, kd, vd = q.to(DEV), k.to(DEV), v.to(DEV)
+    # reference: one launch at a time
+    o1_ref = fm.fmha_fwd(qd, kd, vd, scale=cfg.scale)
+    torch.cuda.synchronize()
+    o2_ref = fm.fmha_fwd(o1_ref.clone(), kd, vd, scale=cfg.scale)
+    torch.cuda.synchronize()
+    o3_ref = fm.fmha_fwd(vd, qd, kd, scale=cfg.scale)
+    torch.cuda.synchronize()
+    for _ in range(20):
+        o1 = torch.empty_like(qd)
+        fm.fmha_fwd(qd, kd, vd, scale=cfg.scale, out=o1)          # writes o1
+        o2 = fm.fmha_fwd(o1, kd, vd, scale=cfg.scale)             # RAW on o1
+        fm.fmha_fwd(vd, qd, kd, scale=cfg.scale, out=o1)          # WAR on o1 (read by the previous launch)
+        torch.cuda.synchronize()
+        assert torch.equal(o2, o2_ref)
+        assert torch.equal(o1, o3_ref)
+
+
+@pytest.mark.timeout(240)
+def test_pdl_gemm_feeds_fmha():
+    """GEMM (PDL) -> FMHA (PDL) -> GEMM (PDL) on one stream: the FMHA's Q is the GEMM output and
+    the last GEMM reads the FMHA output; equal to the same chain with a sync after every launch."""
+    g = torch.Generator().manual_seed(7)
+    b, h, s, d = 2, 4, 256, 64
+    a = (torch.randn(b * h * s, 64, generator=g) * 0.5).half().to(DEV)
+    w = (torch.randn(64, 64, generator=g) * 0.125).half().to(DEV)
+    k = torch.randn(b, h, s, d, generator=g).half().to(DEV)
+    v = torch.rand(b, h, s, d, generator=g).half().to(DEV)
+
+    def chain(sync):
+        x = fm.gemm_bias_act(a, w)
+        if sync:
+            torch.cuda.synchronize()
+        o = fm.fmha_fwd(x.view(b, h, s, d), k, v, scale=0.125)
+        if sync:
+            torch.cuda.synchronize()
+        y = fm.gemm_bias_act(o.view(b * h * s, d), w, act="relu")
+        torch.cuda.synchronize()
+        return y
+
+    ref = chain(True)
+    for _ in range(10):
+        assert torch.equal(chain(False), ref)
