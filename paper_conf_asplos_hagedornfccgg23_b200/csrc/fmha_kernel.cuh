@@ -173,7 +173,7 @@ struct FmhaCfg {
   static constexpr int NUM_BARS = B_KV + 2 * NS;
   static constexpr int OFF_TMEMPTR = OFF_BAR + NUM_BARS * 8;
   static constexpr int OFF_SCHED = OFF_TMEMPTR + 16;  // SchedTable (sched mode 1 only)
-  static constexpr int SMEM_ALLOC = OFF_SCHED + 4 * (2 * (SCHED_MAX_LEVELS + 2) + SCHED_MAX_SEQS);
+  static constexpr int SMEM_ALLOC = OFF_SCHED + 4 * (3 * (SCHED_MAX_LEVELS + 2) + SCHED_MAX_SEQS);
   static constexpr int TMEM_COLS = 512;
   static constexpr int THREADS = 512;
   static constexpr int W_CORR = 8, W_MMA = 12, W_TMA = 14;  // first warp of each role
@@ -252,11 +252,11 @@ struct WorkItem {
   bool has1;     // tile 1 exists
   int tok0, tok1;  // varlen: first token of the sequence of tile 0 / 1; len = its length
   int len0, len1;
-  int head;        // varlen: h of unit bh0
+  int head, head1;  // varlen: h of unit bh0 / bh1
   int jb;          // split-KV: first KV tile of this item's range (0 otherwise)
   int split;       // split-KV: split index
   // TMA coordinates (c1, c2) of the 128-row block starting at row r of tile t (c0 = d)
-  __device__ __forceinline__ int c1(bool varlen, int t, int r) const { return varlen ? head : r; }
+  __device__ __forceinline__ int c1(bool varlen, int t, int r) const { return varlen ? (t ? head1 : head) : r; }
   __device__ __forceinline__ int c2(bool varlen, int t, int r) const { return varlen ? tok(t) + r : bh(t); }
   bool shared;
   __device__ __forceinline__ int n(int t) const { return t ? n1 : n0; }
@@ -319,7 +319,7 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
   w.has0 = true;
   w.kv0 = w.kv1 = p.seq_kv;
   w.tok0 = w.tok1 = 0;
-  w.head = 0;
+  w.head = w.head1 = 0;
   w.len0 = w.len1 = p.seq_q;
   if constexpr (VL) {  // varlen (pair_mode 0): both tiles belong to unit bh0 = b * H + h
     const int b = p.div_heads.div(w.bh0);
@@ -327,6 +327,7 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
     w.len0 = w.len1 = __ldg(p.cu_seqlens + b + 1) - w.tok0;
     w.kv0 = w.kv1 = w.len0;
     w.head = w.bh0 - b * p.heads;
+    w.head1 = w.head;
     w.has0 = w.r0 < w.len0;
     w.has1 = w.has1 && w.r1 < w.len0;
   }
@@ -358,13 +359,14 @@ struct SchedTable {
   int items_end[SCHED_MAX_LEVELS + 2];
   int seq_start[SCHED_MAX_LEVELS + 2];
   int seq_by_level[SCHED_MAX_SEQS];
+  int seq_count[SCHED_MAX_LEVELS + 2];  // sequences of level l
 };
 
 // Built by one full warp before the CTA's first __syncthreads.  Deterministic (no order-dependent
 // atomics), so every CTA derives the same order.
 __device__ __forceinline__ void build_sched(const FmhaParams& p, SchedTable* tb, int lane) {
   const int L = p.max_level;
-  for (int l = lane; l <= L + 1; l += 32) tb->items_end[l] = tb->seq_start[l] = 0;
+  for (int l = lane; l <= L + 1; l += 32) tb->items_end[l] = tb->seq_start[l] = tb->seq_count[l] = 0;
   __syncwarp();
   auto level_of = [&](int sq) {
     if (sq >= p.num_seqs) return -1;
@@ -380,9 +382,12 @@ __device__ __forceinline__ void build_sched(const FmhaParams& p, SchedTable* tb,
     int seqs = 0, items = 0;
     for (int l = L; l >= 1; --l) {
       const int c = tb->seq_start[l];
+      tb->seq_count[l] = c;
       tb->seq_start[l] = seqs;
       seqs += c;
-      items += c * p.heads * ((l + 1) >> 1);
+      // l >> 1 same-unit tile pairs per (sequence, head); for odd l the units' last tiles are
+      // paired across units (two different (sequence, head)), so no item runs half empty
+      items += c * p.heads * (l >> 1) + (l & 1) * ((c * p.heads + 1) >> 1);
       tb->items_end[l] = items;
     }
     tb->items_end[L + 1] = 0;
@@ -422,14 +427,68 @@ __device__ __forceinline__ int item_at(const FmhaParams& p, const SchedTable* tb
   } else {
     const long long pos = static_cast<long long>(k) * G + ((k & 1) ? G - 1 - c : c);
     if (pos >= tb->items_end[0]) return -1;
-    int l = p.max_level;
-    while (pos >= tb->items_end[l]) --l;  // items_end grows as l decreases
-    const int r = static_cast<int>(pos) - tb->items_end[l + 1];
-    const int pairs_l = (l + 1) >> 1, per = p.heads * pairs_l;
-    const int si = r / per, rem = r - si * per;
-    const int h = rem / pairs_l, pr = rem - h * pairs_l;
-    const int sq = tb->seq_by_level[tb->seq_start[l] + si];
-    return (sq * p.heads + h) * ((p.num_q_tiles + 1) >> 1) + pr;
+    return static_cast<int>(pos);  // decoded by sched_item
+  }
+}
+
+// Work item at schedule position pos (sched mode): level l = KV steps; positions of a level list
+// its same-unit pairs (sequence, head, pair) first, then the cross-unit pairs of the last tiles of
+// odd-level units (units in (sequence, head) order, two per item; the last may be alone).
+__device__ __forceinline__ WorkItem sched_item(const FmhaParams& p, const SchedTable* tb, int pos) {
+  int l = p.max_level;
+  while (pos >= tb->items_end[l]) --l;  // items_end grows as l decreases
+  const int r = pos - tb->items_end[l + 1];
+  const int H = p.heads, nl = tb->seq_count[l] * H, full = nl * (l >> 1);
+  WorkItem w;
+  w.jb = 0;
+  w.split = 0;
+  w.has0 = true;
+  int si0, h0, si1, h1;
+  if (r < full) {  // q-tiles 2 pr, 2 pr + 1 of one unit
+    const int pairs_l = l >> 1, per = H * pairs_l;
+    si0 = r / per;
+    const int rem = r - si0 * per;
+    h0 = rem / pairs_l;
+    const int pr = rem - h0 * pairs_l;
+    si1 = si0;
+    h1 = h0;
+    w.r0 = 2 * pr * 128;
+    w.r1 = w.r0 + 128;
+    w.has1 = true;
+    w.shared = true;
+  } else {  // the last q-tile (l - 1) of units 2 r2 and 2 r2 + 1 of this level
+    const int su0 = 2 * (r - full), su1 = su0 + 1;
+    si0 = su0 / H;
+    h0 = su0 - si0 * H;
+    w.has1 = su1 < nl;
+    si1 = w.has1 ? su1 / H : si0;
+    h1 = w.has1 ? su1 - si1 * H : h0;
+    w.r0 = w.r1 = (l - 1) * 128;
+    w.shared = false;
+  }
+  const int sq0 = tb->seq_by_level[tb->seq_start[l] + si0], sq1 = tb->seq_by_level[tb->seq_start[l] + si1];
+  w.tok0 = __ldg(p.cu_seqlens + sq0);
+  w.len0 = __ldg(p.cu_seqlens + sq0 + 1) - w.tok0;
+  w.tok1 = __ldg(p.cu_seqlens + sq1);
+  w.len1 = __ldg(p.cu_seqlens + sq1 + 1) - w.tok1;
+  w.head = h0;
+  w.head1 = h1;
+  w.bh0 = sq0 * H + h0;
+  w.bh1 = sq1 * H + h1;
+  w.kv0 = w.len0;
+  w.kv1 = w.len1;
+  w.n0 = (w.len0 + 127) / 128;
+  w.n1 = w.has1 ? (w.len1 + 127) / 128 : 0;
+  return w;
+}
+
+// decode_item, or sched_item in sched mode
+template <bool PAIRX, bool VL, bool SPLIT, bool SCHED>
+__device__ __forceinline__ WorkItem get_item(const FmhaParams& p, const SchedTable* tb, int idx) {
+  if constexpr (SCHED) {
+    return sched_item(p, tb, idx);
+  } else {
+    return decode_item<PAIRX, VL, SPLIT>(p, idx);
   }
 }
 
@@ -533,7 +592,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         }
       };
       for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
-        const WorkItem w = decode_item<PAIRX, VL, SPLIT>(p, idx);
+        const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED>(p, sched, idx);
         const int N = max(w.n0, w.n1);
 #pragma unroll
         for (int t = 0; t < 2; ++t) {
@@ -601,7 +660,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       auto seek = [&](Cursor& cu, int k, uint32_t base) {
         cu.valid = false;
         for (int idx; (idx = item_at<SCHED>(p, sched, k)) >= 0; ++k) {
-          const WorkItem w = decode_item<PAIRX, VL, SPLIT>(p, idx);
+          const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED>(p, sched, idx);
           const int N = max(w.n0, w.n1);
           if (N == 0) continue;
           cu.w.n0 = w.n0;
@@ -743,7 +802,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     // g = real steps this thread has done so far: the phase count of S_FULL and PV_DONE
     uint32_t g = 0, lc = 0;
     for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
-      const WorkItem w = decode_item<PAIRX, VL, SPLIT>(p, idx);
+      const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED>(p, sched, idx);
       const int n = w.n(t);
       const int N = C::TURNS ? max(w.n0, w.n1) : n;
       TRACE_EV(EV_ITEM, 1);
@@ -1033,7 +1092,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     // (which lived in local memory)
     uint32_t ofbits = 0, lbits = 0;
     for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
-      const WorkItem w = decode_item<PAIRX, VL, SPLIT>(p, idx);
+      const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED>(p, sched, idx);
       // ------------------------------------------------------------ epilogue per tile (a9)
 #pragma unroll 1
       for (int t = 0; t < 2; ++t) {
@@ -1105,7 +1164,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
               st_shared_v4(box + ((unit ^ (row & 7)) << 4), v0, v1, v2, v3);
             } else if (row < w.len(t) - w.row0(t)) {  // varlen partial tile: rows inside the sequence
               const size_t tokn = static_cast<size_t>(w.tok(t) + w.row0(t) + row);
-              st_global_v4(p.o_ptr + 2 * (tokn * p.o_row_elems + w.head * D + col0 + 8 * u), v0, v1, v2, v3);
+              st_global_v4(p.o_ptr + 2 * (tokn * p.o_row_elems + (t ? w.head1 : w.head) * D + col0 + 8 * u), v0, v1, v2, v3);
             }
           }
         }

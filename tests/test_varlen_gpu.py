@@ -38,6 +38,8 @@ LENGTHS = [
     [0, 77, 0, 300, 5],
     [384, 200, 31, 128, 129, 383],
     [513, 2, 640],
+    # odd levels 1, 3, 5 with several sequences each: last q-tiles paired across (sequence, head)
+    [1, 130, 260, 390, 5, 300, 129, 0, 384, 383, 600, 77, 520, 31],
 ]
 
 
