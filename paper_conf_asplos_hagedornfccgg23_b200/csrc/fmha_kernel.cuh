@@ -240,6 +240,25 @@ struct FmhaCfg {
   static_assert(SMEM_ALLOC <= 232448, "shared memory budget");
 };
 
+// Exponential-phase shape per kernel instance.  The cross-unit pair instance (BERT-large-384: each
+// tile streams its own K/V) measured best with every chunk inside the turn and 1 of 8 exp2 pairs
+// on the FMA pipe (+1.9% against the dense instance's 1 pre-turn chunk and 2 of 8, which is -2.4%
+// on the dense BERT-large-512 instance; profiles/r01_ab_pc0.txt).
+#ifndef FMHA_PAIRX_PRE_CHUNKS
+#define FMHA_PAIRX_PRE_CHUNKS 0
+#endif
+#ifndef FMHA_PAIRX_POLY_CNT
+#define FMHA_PAIRX_POLY_CNT 1
+#endif
+template <int D, bool PAIRX>
+struct ExpShape {
+  static constexpr bool ALT = PAIRX && D == 64 && FmhaCfg<D>::TURNS && !FmhaCfg<D>::POLY_MASK;
+  static constexpr int PRE_CHUNKS = ALT ? FMHA_PAIRX_PRE_CHUNKS : FmhaCfg<D>::PRE_CHUNKS;
+  static __host__ __device__ constexpr bool poly_pair(int q) {
+    return ALT ? (q % 8) < FMHA_PAIRX_POLY_CNT : FmhaCfg<D>::poly_pair(q);
+  }
+};
+
 // One work item = two 128-row query tiles t = 0, 1.  Every role decodes items identically.
 // shared: both tiles belong to one unit and share every K/V tile; otherwise (pair_mode 1) each tile
 // streams its own K/V through the ring (entries of tile 0 then tile 1 for every step j).
@@ -500,6 +519,7 @@ enum : int { MODE_DENSE = 0, MODE_PAIRX = 1, MODE_VARLEN = 2, MODE_VARLEN_SCHED 
 template <int D, bool BF16, int MODE>
 __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
   using C = FmhaCfg<D>;
+  using XS = ExpShape<D, MODE == MODE_PAIRX>;
   constexpr bool PAIRX = MODE == MODE_PAIRX, VL = MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
                  SCHED = MODE == MODE_VARLEN_SCHED, SPLIT = MODE == MODE_SPLIT, BIAS = MODE == MODE_BIAS;
   // Dynamic shared memory starts at the (1024-byte aligned) base of the CTA's shared window; the
@@ -955,7 +975,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           uint32_t pk_all[4][16];
 #pragma unroll
         for (int hh = 0; hh < 4; ++hh) {
-          if (hh == C::PRE_CHUNKS) {
+          if (hh == XS::PRE_CHUNKS) {
             // The exponentials are register-only work that ptxas would hoist above the barrier:
             // round-trip their input through shared memory, which bar.sync does order.
             const uint32_t slot = sbase + C::OFF_MC + (t * 128 + row) * 4;
@@ -965,8 +985,8 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             asm volatile("ld.volatile.shared.f32 %0, [%1];" : "=f"(mcv) : "r"(slot) : "memory");
           }
           uint32_t (&pk)[16] = pk_all[hh];
-          const bool defer = C::DEFER_ST != 0 && hh >= C::PRE_CHUNKS;
-          if (C::DEFER_ST == 2 && hh > C::PRE_CHUNKS) tmem_st_32x32b_x16(tP + 16 * (hh - 1), pk_all[hh - 1]);
+          const bool defer = C::DEFER_ST != 0 && hh >= XS::PRE_CHUNKS;
+          if (C::DEFER_ST == 2 && hh > XS::PRE_CHUNKS) tmem_st_32x32b_x16(tP + 16 * (hh - 1), pk_all[hh - 1]);
           if (SKIP && 32 * hh >= rem_w) {
 #pragma unroll
             for (int u = 0; u < 16; ++u) pk[u] = 0u;
@@ -983,7 +1003,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
               x0 = fadd2(x0, make_float2(1.f, 1.f));
             } else
 #endif
-            if (C::poly_pair(16 * hh + u)) {
+            if (XS::poly_pair(16 * hh + u)) {
               x0 = exp2_poly2(x0);
             } else {
               x0.x = ex2(x0.x);
@@ -994,7 +1014,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
               x1 = fadd2(x1, make_float2(1.f, 1.f));
             } else
 #endif
-            if (C::poly_pair(16 * hh + u + 1)) {
+            if (XS::poly_pair(16 * hh + u + 1)) {
               x1 = exp2_poly2(x1);
             } else {
               x1.x = ex2(x1.x);
@@ -1011,7 +1031,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         }
         if constexpr (C::DEFER_ST == 1) {
 #pragma unroll
-          for (int hh = C::PRE_CHUNKS; hh < 4; ++hh) tmem_st_32x32b_x16(tP + 16 * hh, pk_all[hh]);
+          for (int hh = XS::PRE_CHUNKS; hh < 4; ++hh) tmem_st_32x32b_x16(tP + 16 * hh, pk_all[hh]);
         } else if constexpr (C::DEFER_ST == 2) {
           tmem_st_32x32b_x16(tP + 16 * 3, pk_all[3]);
         }
