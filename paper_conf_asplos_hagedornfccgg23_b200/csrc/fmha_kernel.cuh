@@ -250,9 +250,12 @@ struct FmhaCfg {
 #ifndef FMHA_PAIRX_POLY_CNT
 #define FMHA_PAIRX_POLY_CNT 1
 #endif
-template <int D, bool PAIRX>
+#ifndef FMHA_VARLEN_ALT
+#define FMHA_VARLEN_ALT 0
+#endif
+template <int D, bool PAIRX, bool VL = false>
 struct ExpShape {
-  static constexpr bool ALT = PAIRX && D == 64 && FmhaCfg<D>::TURNS && !FmhaCfg<D>::POLY_MASK;
+  static constexpr bool ALT = (PAIRX || (VL && FMHA_VARLEN_ALT)) && D == 64 && FmhaCfg<D>::TURNS && !FmhaCfg<D>::POLY_MASK;
   static constexpr int PRE_CHUNKS = ALT ? FMHA_PAIRX_PRE_CHUNKS : FmhaCfg<D>::PRE_CHUNKS;
   static __host__ __device__ constexpr bool poly_pair(int q) {
     return ALT ? (q % 8) < FMHA_PAIRX_POLY_CNT : FmhaCfg<D>::poly_pair(q);
@@ -519,7 +522,7 @@ enum : int { MODE_DENSE = 0, MODE_PAIRX = 1, MODE_VARLEN = 2, MODE_VARLEN_SCHED 
 template <int D, bool BF16, int MODE>
 __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
   using C = FmhaCfg<D>;
-  using XS = ExpShape<D, MODE == MODE_PAIRX>;
+  using XS = ExpShape<D, MODE == MODE_PAIRX, MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED>;
   constexpr bool PAIRX = MODE == MODE_PAIRX, VL = MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
                  SCHED = MODE == MODE_VARLEN_SCHED, SPLIT = MODE == MODE_SPLIT, BIAS = MODE == MODE_BIAS;
   // Dynamic shared memory starts at the (1024-byte aligned) base of the CTA's shared window; the
