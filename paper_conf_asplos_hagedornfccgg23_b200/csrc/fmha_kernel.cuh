@@ -241,14 +241,15 @@ struct FmhaCfg {
 };
 
 // Exponential-phase shape per kernel instance.  The cross-unit pair instance (BERT-large-384: each
-// tile streams its own K/V) measured best with every chunk inside the turn and 1 of 8 exp2 pairs
-// on the FMA pipe (+1.9% against the dense instance's 1 pre-turn chunk and 2 of 8, which is -2.4%
-// on the dense BERT-large-512 instance; profiles/r01_ab_pc0.txt).
+// tile streams its own K/V) measured best with all exp2 on MUFU (no polynomial pairs), keeping the
+// one pre-turn chunk: 525 vs 517 TF/s for (0 pre-turn chunks, 1 of 8) and 509 for the dense
+// instance's (1, 2 of 8), which stays best on BERT-large-512 (profiles/r01_ab_pc0.txt,
+// r01_ab_pairx_expshape.txt, r01_ab_pairx_sweep.txt).
 #ifndef FMHA_PAIRX_PRE_CHUNKS
-#define FMHA_PAIRX_PRE_CHUNKS 0
+#define FMHA_PAIRX_PRE_CHUNKS 1
 #endif
 #ifndef FMHA_PAIRX_POLY_CNT
-#define FMHA_PAIRX_POLY_CNT 1
+#define FMHA_PAIRX_POLY_CNT 0
 #endif
 #ifndef FMHA_VARLEN_ALT
 #define FMHA_VARLEN_ALT 0
