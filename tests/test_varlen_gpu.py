@@ -67,16 +67,27 @@ def test_varlen_rows_outside_sequences_untouched_and_max_seqlen_slack():
     assert torch.equal(o1, o2)
 
 
-def test_varlen_equal_lengths_matches_dense_kernel():
-    """Equal lengths: the packed path and the dense [B,H,S,D] path compute the same per-row
-    arithmetic, so their outputs are bitwise equal."""
-    cfg = VarlenConfig("veq", 23, 3, 4, 384, 64)
-    x, cu = make_varlen_inputs(cfg, lengths=[384] * 3)
+@pytest.mark.parametrize("seq", [256, 512, 384])
+def test_varlen_equal_lengths_matches_dense_kernel(seq):
+    """Equal lengths: with an even q-tile count the dense [B,H,S,D] path runs the dense instance,
+    whose exponential-phase shape (ExpShape) is the varlen one, so the per-row arithmetic and the
+    outputs are bitwise equal.  An odd count (384 = 3 tiles) runs the cross-unit pair instance,
+    which takes every exp2 on MUFU instead of 2 of 8 pairs on the FMA-pipe polynomial: there both
+    sides are held to the oracle tolerance and to each other within fp16 rounding."""
+    cfg = VarlenConfig("veq", 23, 3, 4, seq, 64)
+    x, cu = make_varlen_inputs(cfg, lengths=[seq] * 3)
     o = run(cfg, x, cu)
-    xs = x.view(3, 384, 3, 4, 64).permute(2, 0, 3, 1, 4).contiguous().to(DEV)  # [3,B,H,S,D]
+    xs = x.view(3, seq, 3, 4, 64).permute(2, 0, 3, 1, 4).contiguous().to(DEV)  # [3,B,H,S,D]
     od = fm.fmha_fwd(xs[0], xs[1], xs[2], scale=cfg.scale)
     torch.cuda.synchronize()
-    assert torch.equal(o, od.permute(0, 2, 1, 3).reshape(3 * 384, 4, 64))
+    od = od.permute(0, 2, 1, 3).reshape(3 * seq, 4, 64)
+    if seq % 256 == 0:
+        assert torch.equal(o, od)
+    else:
+        ref = attention_varlen_fp64(x, cu, cfg.scale)
+        check(o, ref, "fp16", "varlen")
+        check(od, ref, "fp16", "dense pair instance")
+        assert (o.float() - od.float()).abs().max().item() <= 2e-3
 
 
 def test_varlen_bert_large_full_size():
