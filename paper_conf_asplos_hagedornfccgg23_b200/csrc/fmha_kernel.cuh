@@ -211,6 +211,13 @@ struct FmhaCfg {
 #define FMHA_BIAS_PF4 0
 #endif
   static constexpr bool BIAS_PF4 = FMHA_BIAS_PF4;
+  // Key bias: unpredicated loads with the column clamped into the row (stride >= seq_kv, a multiple
+  // of 4, so every valid column is unchanged; the clamped ones are past seq_kv and masked) instead
+  // of predicated loads with zero fill (A/B knob)
+#ifndef FMHA_BIAS_CLAMP
+#define FMHA_BIAS_CLAMP 1
+#endif
+  static constexpr bool BIAS_CLAMP = FMHA_BIAS_CLAMP;
   // The first PRE_CHUNKS of the four 32-column chunks of a row are exponentiated before the turn
   // (overlapping the other tile's turn), the rest inside it.
 #ifndef FMHA_PRE_CHUNKS
@@ -926,13 +933,19 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           } else if (key0 + 128 < p.seq_kv) {
             asm volatile("prefetch.global.L1 [%0];" ::"l"(brow + key0 + 128));
           }
+          // (clamp: last float4 of the row, >= 0 since key0 < seq_kv <= stride, all multiples of 4)
+          const unsigned cap4 = static_cast<unsigned>(p.key_bias_stride - 4 - key0) >> 2;
+          const float4* bk0 = reinterpret_cast<const float4*>(brow + key0);
 #pragma unroll
           for (int q = 0; q < 4; ++q) {
             float4 bq[8];
 #pragma unroll
             for (int u = 0; u < 8; ++u) {
               const int col = key0 + 32 * q + 4 * u;
-              bq[u] = col < p.seq_kv ? __ldg(reinterpret_cast<const float4*>(brow + col)) : make_float4(0.f, 0.f, 0.f, 0.f);
+              if constexpr (C::BIAS_CLAMP)  // keys >= seq_kv are set to -inf below, whatever they load
+                bq[u] = __ldg(bk0 + min(static_cast<unsigned>(8 * q + u), cap4));
+              else
+                bq[u] = col < p.seq_kv ? __ldg(reinterpret_cast<const float4*>(brow + col)) : make_float4(0.f, 0.f, 0.f, 0.f);
             }
 #pragma unroll
             for (int u = 0; u < 8; ++u) {
