@@ -94,3 +94,16 @@ def test_key_bias_errors():
         fm.fmha_fwd(qd, kd, vd, key_bias=torch.zeros(1, 28, device=DEV))
     with pytest.raises(fm.FmhaError):  # scale 0 (the bias is added as bias / scale)
         fm.fmha_fwd(qd, kd, vd, scale=0.0, key_bias=torch.zeros(1, 32, device=DEV))
+
+
+@pytest.mark.parametrize("skv,extra", [(260, 0), (200, 60), (129, 380), (512, 4)])
+def test_key_bias_row_stride_and_clamped_tail(skv, extra):
+    """Bias rows longer than seq_kv (stride = seq_kv rounded to 4 + extra, NaN past seq_kv): the
+    kernel's bias loads are clamped to the row's last float4 (FMHA_BIAS_CLAMP) and every column past
+    seq_kv is masked before the row max, so neither the stride nor the padding reaches a result."""
+    cfg = FmhaConfig("keybias_stride", 20, 3, 2, 150, skv, 64, "fp16")
+    q, k, v, _ = make_fmha_inputs(cfg)
+    kb = make_bias(3, skv, "random", seed=skv + extra, stride=(skv + 3) // 4 * 4 + extra)
+    o = fm.fmha_fwd(q.to(DEV), k.to(DEV), v.to(DEV), scale=cfg.scale, key_bias=torch.from_numpy(kb).to(DEV))
+    torch.cuda.synchronize()
+    check(o, attention_fp64(q, k, v, cfg.scale, key_bias=kb[:, :skv]), "fp16", f"skv={skv} extra={extra}")
