@@ -21,6 +21,10 @@ for d in (64, 128):
         q3 = r(2, 2, 384, d, dt=dt)
         fm.fmha_fwd(q3, q3, q3)  # pair_mode 1 (odd q-tile count)
         fm.fmha_fwd_splitkv(q[:, :, :16].contiguous(), k, v, num_splits=3)
+        # key bias (MODE_BIAS) with stride == seq_kv = 300: the clamped bias loads of the ragged last
+        # KV tile must stay inside the row (run with PYTORCH_NO_CUDA_MEMORY_CACHING=1 so the bias
+        # allocation ends exactly at the last row)
+        fm.fmha_fwd(q, k, v, key_bias=torch.randn(1, 300, generator=g).to(dev))
 qkv = r(300, 3, 4, 64)
 cu = torch.tensor([0, 100, 100, 300], dtype=torch.int32, device=dev)
 fm.fmha_fwd_varlen(qkv, cu, 200)
