@@ -267,12 +267,23 @@ struct FmhaCfg {
 #ifndef FMHA_VARLEN_ALT
 #define FMHA_VARLEN_ALT 0
 #endif
-template <int D, bool PAIRX, bool VL = false>
+// The key-bias instance has its own pair (FMHA_BIAS_PRE_CHUNKS, FMHA_BIAS_POLY_CNT): the bias add
+// lengthens the S -> max part of its step, which moves the best split of the exponential phase.
+// Sweep of 8 shapes (profiles/r01_ab_bias_shape.txt): (0 pre-turn chunks, all exp2 on MUFU) is
+// best, -4.9% at BERT-large-384 and -2.7% at 512 against the dense instance's (1, 2 of 8).
+#ifndef FMHA_BIAS_PRE_CHUNKS
+#define FMHA_BIAS_PRE_CHUNKS 0
+#endif
+#ifndef FMHA_BIAS_POLY_CNT
+#define FMHA_BIAS_POLY_CNT 0
+#endif
+template <int D, bool PAIRX, bool VL = false, bool BIAS = false>
 struct ExpShape {
   static constexpr bool ALT = (PAIRX || (VL && FMHA_VARLEN_ALT)) && D == 64 && FmhaCfg<D>::TURNS && !FmhaCfg<D>::POLY_MASK;
-  static constexpr int PRE_CHUNKS = ALT ? FMHA_PAIRX_PRE_CHUNKS : FmhaCfg<D>::PRE_CHUNKS;
+  static constexpr bool BSH = BIAS && D == 64 && FmhaCfg<D>::TURNS && !FmhaCfg<D>::POLY_MASK;
+  static constexpr int PRE_CHUNKS = ALT ? FMHA_PAIRX_PRE_CHUNKS : BSH ? FMHA_BIAS_PRE_CHUNKS : FmhaCfg<D>::PRE_CHUNKS;
   static __host__ __device__ constexpr bool poly_pair(int q) {
-    return ALT ? (q % 8) < FMHA_PAIRX_POLY_CNT : FmhaCfg<D>::poly_pair(q);
+    return ALT ? (q % 8) < FMHA_PAIRX_POLY_CNT : BSH ? (q % 8) < FMHA_BIAS_POLY_CNT : FmhaCfg<D>::poly_pair(q);
   }
 };
 
@@ -536,7 +547,7 @@ enum : int { MODE_DENSE = 0, MODE_PAIRX = 1, MODE_VARLEN = 2, MODE_VARLEN_SCHED 
 template <int D, bool BF16, int MODE>
 __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
   using C = FmhaCfg<D>;
-  using XS = ExpShape<D, MODE == MODE_PAIRX, MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED>;
+  using XS = ExpShape<D, MODE == MODE_PAIRX, MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED, MODE == MODE_BIAS>;
   constexpr bool PAIRX = MODE == MODE_PAIRX, VL = MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
                  SCHED = MODE == MODE_VARLEN_SCHED, SPLIT = MODE == MODE_SPLIT, BIAS = MODE == MODE_BIAS;
   // Dynamic shared memory starts at the (1024-byte aligned) base of the CTA's shared window; the
