@@ -277,13 +277,25 @@ struct FmhaCfg {
 #ifndef FMHA_BIAS_POLY_CNT
 #define FMHA_BIAS_POLY_CNT 0
 #endif
+// Varlen instances: (FMHA_VARLEN_PRE_CHUNKS, FMHA_VARLEN_POLY_CNT), -1 = the dense instance's shape.
+// Sweep of 8 shapes on bert_large_varlen (profiles/r01_ab_varlen_shape.txt): two pre-turn chunks
+// with the dense instance's 2 of 8 polynomial pairs is best, 172.0 vs 168.6 TF/s (+2%).
+#ifndef FMHA_VARLEN_PRE_CHUNKS
+#define FMHA_VARLEN_PRE_CHUNKS 2
+#endif
+#ifndef FMHA_VARLEN_POLY_CNT
+#define FMHA_VARLEN_POLY_CNT -1
+#endif
 template <int D, bool PAIRX, bool VL = false, bool BIAS = false>
 struct ExpShape {
   static constexpr bool ALT = (PAIRX || (VL && FMHA_VARLEN_ALT)) && D == 64 && FmhaCfg<D>::TURNS && !FmhaCfg<D>::POLY_MASK;
   static constexpr bool BSH = BIAS && D == 64 && FmhaCfg<D>::TURNS && !FmhaCfg<D>::POLY_MASK;
-  static constexpr int PRE_CHUNKS = ALT ? FMHA_PAIRX_PRE_CHUNKS : BSH ? FMHA_BIAS_PRE_CHUNKS : FmhaCfg<D>::PRE_CHUNKS;
+  static constexpr bool VSH = VL && !ALT && D == 64 && FmhaCfg<D>::TURNS && !FmhaCfg<D>::POLY_MASK;
+  static constexpr int PRE_CHUNKS = ALT ? FMHA_PAIRX_PRE_CHUNKS : BSH ? FMHA_BIAS_PRE_CHUNKS
+                                  : (VSH && FMHA_VARLEN_PRE_CHUNKS >= 0) ? FMHA_VARLEN_PRE_CHUNKS : FmhaCfg<D>::PRE_CHUNKS;
   static __host__ __device__ constexpr bool poly_pair(int q) {
-    return ALT ? (q % 8) < FMHA_PAIRX_POLY_CNT : BSH ? (q % 8) < FMHA_BIAS_POLY_CNT : FmhaCfg<D>::poly_pair(q);
+    return ALT ? (q % 8) < FMHA_PAIRX_POLY_CNT : BSH ? (q % 8) < FMHA_BIAS_POLY_CNT
+         : (VSH && FMHA_VARLEN_POLY_CNT >= 0) ? (q % 8) < FMHA_VARLEN_POLY_CNT : FmhaCfg<D>::poly_pair(q);
   }
 };
 
