@@ -278,13 +278,14 @@ struct FmhaCfg {
 #define FMHA_BIAS_POLY_CNT 0
 #endif
 // Varlen instances: (FMHA_VARLEN_PRE_CHUNKS, FMHA_VARLEN_POLY_CNT), -1 = the dense instance's shape.
-// Sweep of 8 shapes on bert_large_varlen (profiles/r01_ab_varlen_shape.txt): two pre-turn chunks
-// with the dense instance's 2 of 8 polynomial pairs is best, 172.0 vs 168.6 TF/s (+2%).
+// Sweeps of 13 shapes on bert_large_varlen (profiles/r01_ab_varlen_shape.txt, _shape2.txt): two
+// pre-turn chunks with every exp2 on MUFU is best, 173.7 vs 171.1 TF/s for (2, 2 of 8) and 168.6
+// for the dense instance's (1, 2 of 8).  (Same exp2 arithmetic as the pair instance.)
 #ifndef FMHA_VARLEN_PRE_CHUNKS
 #define FMHA_VARLEN_PRE_CHUNKS 2
 #endif
 #ifndef FMHA_VARLEN_POLY_CNT
-#define FMHA_VARLEN_POLY_CNT -1
+#define FMHA_VARLEN_POLY_CNT 0
 #endif
 template <int D, bool PAIRX, bool VL = false, bool BIAS = false>
 struct ExpShape {
