@@ -38,6 +38,25 @@ def _stream_ptr(dev: torch.device) -> int:
     return torch.cuda.current_stream(dev).cuda_stream
 
 
+def _check_out(out: torch.Tensor, shape, dtype, like: torch.Tensor, what: str) -> None:
+    """A caller-supplied output must be exactly what the kernel writes: shape, dtype, dense
+    row-major layout and the inputs' device (the kernels write every element through raw pointers)."""
+    if tuple(out.shape) != tuple(shape) or out.dtype != dtype or not out.is_contiguous() or out.device != like.device:
+        raise ValueError(f"{what}: out must be a contiguous {dtype} tensor of shape {tuple(shape)} on {like.device}, "
+                         f"got {out.dtype} {tuple(out.shape)} on {out.device}")
+
+
+def _check_bias(bias: torch.Tensor | None, shape, like: torch.Tensor, what: str) -> torch.Tensor | None:
+    """Bias vectors are read for every output column: exact shape, fp16, on the inputs' device; the
+    contiguous copy is returned so the caller keeps it alive across the launch."""
+    if bias is None:
+        return None
+    if tuple(bias.shape) != tuple(shape) or bias.dtype != torch.float16 or bias.device != like.device:
+        raise ValueError(f"{what}: bias must be fp16 {tuple(shape)} on {like.device}, got {bias.dtype} "
+                         f"{tuple(bias.shape)} on {bias.device}")
+    return bias.contiguous()
+
+
 def _mask(kv_len, causal: bool):
     if kv_len is not None and causal:
         raise ValueError("key padding and causal masks are mutually exclusive in this ABI")
@@ -73,6 +92,8 @@ def fmha_fwd(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, kv_len: torch.Te
         kv_len = kv_len.contiguous()
     if out is None:
         out = torch.empty_like(q)
+    else:
+        _check_out(out, q.shape, q.dtype, q, "fmha_fwd")
     scale = 1.0 / math.sqrt(d) if scale is None else float(scale)
     if key_bias is not None:
         if kv_len is not None or causal:
@@ -114,6 +135,8 @@ def fmha_fwd_splitkv(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, kv_len: 
         kv_len = kv_len.contiguous()
     if out is None:
         out = torch.empty_like(q)
+    else:
+        _check_out(out, q.shape, q.dtype, q, "fmha_fwd_splitkv")
     splits = num_splits if num_splits > 0 else lib.fmha_splitkv_default_splits(b, h, sq, skv)
     need = lib.fmha_splitkv_workspace_bytes(b, h, sq, d, splits)
     if workspace is None or workspace.numel() < need:
@@ -166,8 +189,21 @@ def fmha_fwd_from_host(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, out: t
     D2H copy are ordered after ``stream``'s queued work and joined back into it by ``fmha_fwd_from_host`` of the C ABI (async; the
     caller synchronises before reading ``out``)."""
     lib = _lib.load()
+    if q.dtype not in (torch.float16, torch.bfloat16) or k.dtype != q.dtype or v.dtype != q.dtype or out.dtype != q.dtype:
+        raise TypeError("q, k, v, out must share dtype fp16 or bf16")
+    if any(t.is_cuda for t in (q, k, v, out)):
+        raise TypeError("fmha_fwd_from_host takes HOST q, k, v, out (use fmha_fwd for device tensors)")
+    if not all(t.is_contiguous() for t in (q, k, v, out)):
+        raise ValueError("q, k, v, out must be contiguous [B,H,S,D]")
+    if not workspace.is_cuda:
+        raise TypeError("workspace must be a CUDA tensor")
     b, h, sq, d = q.shape
     skv = k.shape[2]
+    if k.shape != (b, h, skv, d) or v.shape != k.shape or out.shape != q.shape:
+        raise ValueError(f"shape mismatch q{tuple(q.shape)} k{tuple(k.shape)} v{tuple(v.shape)} out{tuple(out.shape)}")
+    if kv_len is not None and (kv_len.is_cuda or kv_len.dtype != torch.int32 or kv_len.numel() != b
+                               or not kv_len.is_contiguous()):
+        raise ValueError("kv_len must be a contiguous HOST int32 tensor of length batch for fmha_fwd_from_host")
     dt = {torch.float16: 0, torch.bfloat16: 1}[q.dtype]
     m = FmhaMask(MASK_NONE, None)
     if kv_len is not None:
@@ -196,9 +232,12 @@ def gemm_bias_act(a: torch.Tensor, w: torch.Tensor, bias: torch.Tensor | None = 
     n_ = w.shape[0]
     if w.shape[1] != k_:
         raise ValueError("K mismatch")
+    bias = _check_bias(bias, (n_,), a, "gemm_bias_act")
     if out is None:
         out = torch.empty((m_, n_), dtype=torch.float16, device=a.device)
-    st = lib.gemm_bias_act(a.data_ptr(), w.data_ptr(), None if bias is None else bias.contiguous().data_ptr(),
+    else:
+        _check_out(out, (m_, n_), torch.float16, a, "gemm_bias_act")
+    st = lib.gemm_bias_act(a.data_ptr(), w.data_ptr(), None if bias is None else bias.data_ptr(),
                            out.data_ptr(), m_, n_, k_, ACTS[act], _stream_ptr(a.device))
     _lib.check(st, "gemm_bias_act")
     return out
@@ -255,10 +294,13 @@ def dual_gemm_bias_act(a1: torch.Tensor, w1: torch.Tensor, a2: torch.Tensor, w2:
     n_, k2 = w1.shape[0], a2.shape[1]
     if w1.shape[1] != k1 or a2.shape[0] != m_ or w2.shape != (n_, k2):
         raise ValueError("shape mismatch")
+    bias = _check_bias(bias, (n_,), a1, "dual_gemm_bias_act")
     if out is None:
         out = torch.empty((m_, n_), dtype=torch.float16, device=a1.device)
+    else:
+        _check_out(out, (m_, n_), torch.float16, a1, "dual_gemm_bias_act")
     st = lib.dual_gemm_bias_act(a1.data_ptr(), w1.data_ptr(), a2.data_ptr(), w2.data_ptr(),
-                                None if bias is None else bias.contiguous().data_ptr(), out.data_ptr(),
+                                None if bias is None else bias.data_ptr(), out.data_ptr(),
                                 m_, n_, k1, k2, ACTS[act], _stream_ptr(a1.device))
     _lib.check(st, "dual_gemm_bias_act")
     return out
@@ -277,9 +319,12 @@ def mlp_fused(x: torch.Tensor, w: torch.Tensor, bias: torch.Tensor | None = None
     layers = w.shape[0]
     if w.shape != (layers, n_, n_) or (bias is not None and bias.shape != (layers, n_)):
         raise ValueError("shape mismatch")
+    bias = _check_bias(bias, (layers, n_), x, "mlp_fused")
     if out is None:
         out = torch.empty((m_, n_), dtype=torch.float16, device=x.device)
-    st = lib.mlp_fused_fwd(x.data_ptr(), w.data_ptr(), None if bias is None else bias.contiguous().data_ptr(),
+    else:
+        _check_out(out, (m_, n_), torch.float16, x, "mlp_fused")
+    st = lib.mlp_fused_fwd(x.data_ptr(), w.data_ptr(), None if bias is None else bias.data_ptr(),
                            out.data_ptr(), m_, n_, layers, ACTS[act], _stream_ptr(x.device))
     _lib.check(st, "mlp_fused_fwd")
     return out

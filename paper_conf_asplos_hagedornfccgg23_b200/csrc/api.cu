@@ -173,7 +173,7 @@ size_t splitkv_ws_bytes(long long units, int seq_q, int head_dim, int splits) {
 // s with the least rounds x (tiles + 2), at least one KV tile per split.  1 when the dense schedule
 // already fills the SMs.
 int splitkv_default(long long units, int seq_q, int seq_kv, int sms) {
-  const long long items = units * ((seq_q + 127) / 128 + 1) / 2;
+  const long long items = units * (((seq_q + 127) / 128 + 1) / 2);  // (unit, q-tile pair) items
   const int nkv = (seq_kv + 127) / 128;
   if (items <= 0 || items >= sms || nkv <= 1) return 1;
   int best_s = 1;
@@ -191,10 +191,11 @@ int splitkv_default(long long units, int seq_q, int seq_kv, int sms) {
   return best_s;
 }
 
-int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask,
-                int batch, int heads, int seq_q, int seq_kv, int head_dim, float scale, cudaStream_t stream,
-                int splits = 1, void* workspace = nullptr, size_t workspace_bytes = 0) {
-  g_last_cuda_error[0] = 0;
+// The argument checks of fmha_common that need no pointers to be valid device memory: shapes, scale,
+// head_dim, mask kind.  FMHA_OK with *empty = true means there is nothing to launch.
+int validate_shape(int batch, int heads, int seq_q, int seq_kv, int head_dim, float scale, const fmha_mask_t* mask,
+                   int splits, bool* empty) {
+  *empty = false;
   if (batch < 0 || heads < 0 || seq_q < 0 || seq_kv < 0) return FMHA_ERR_INVALID_ARG;
   if (!std::isfinite(scale)) return FMHA_ERR_INVALID_ARG;
   if (head_dim != 64 && head_dim != 128) return FMHA_ERR_UNSUPPORTED;
@@ -208,15 +209,30 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
     if (mask->key_bias_stride < seq_kv || (mask->key_bias_stride % 4) != 0) return FMHA_ERR_INVALID_ARG;
   }
   const long long units = static_cast<long long>(batch) * heads;
-  if (units == 0 || seq_q == 0) return FMHA_OK;
+  if (units == 0 || seq_q == 0) {
+    *empty = true;
+    return FMHA_OK;
+  }
   if (seq_kv == 0) return FMHA_ERR_INVALID_ARG;
-  if (!Q || !K || !V || !O) return FMHA_ERR_INVALID_ARG;
   if (kind == FMHA_MASK_KEY_PADDING && !mask->kv_len) return FMHA_ERR_INVALID_ARG;
+  if (units > 2147483647LL || static_cast<long long>(seq_q) * head_dim * units * 2 > (1LL << 40))
+    return FMHA_ERR_INVALID_ARG;
+  return FMHA_OK;
+}
+
+int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask,
+                int batch, int heads, int seq_q, int seq_kv, int head_dim, float scale, cudaStream_t stream,
+                int splits = 1, void* workspace = nullptr, size_t workspace_bytes = 0) {
+  g_last_cuda_error[0] = 0;
+  bool empty = false;
+  if (int vs = validate_shape(batch, heads, seq_q, seq_kv, head_dim, scale, mask, splits, &empty); vs != FMHA_OK || empty)
+    return vs;
+  const int kind = mask ? mask->kind : FMHA_MASK_NONE;
+  const long long units = static_cast<long long>(batch) * heads;
+  if (!Q || !K || !V || !O) return FMHA_ERR_INVALID_ARG;
   if (kind == FMHA_MASK_KEY_BIAS && !mask->key_bias) return FMHA_ERR_INVALID_ARG;
   if (kind == FMHA_MASK_KEY_BIAS && !aligned16(mask->key_bias)) return FMHA_ERR_MISALIGNED;
   if (!aligned16(Q) || !aligned16(K) || !aligned16(V) || !aligned16(O)) return FMHA_ERR_MISALIGNED;
-  if (units > 2147483647LL || static_cast<long long>(seq_q) * head_dim * units * 2 > (1LL << 40))
-    return FMHA_ERR_INVALID_ARG;
   int sm_count = 0;
   int st = check_device(&sm_count);
   if (st != FMHA_OK) return st;
@@ -247,7 +263,7 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   if (kind == FMHA_MASK_KEY_BIAS) {
     prm.key_bias = mask->key_bias;
     prm.key_bias_stride = mask->key_bias_stride;
-    prm.inv_scale = 1.f / scale;
+    prm.inv_scale = 1.4426950408889634f / prm.scale_log2;  // c * inv_scale = log2(e) exactly as used
     prm.mask_kind = FMHA_MASK_NONE;  // no key bound beyond seq_kv; the bias does the masking
   }
   long long items = prm.pair_mode ? (units * prm.num_q_tiles + 1) / 2 : units * ((prm.num_q_tiles + 1) / 2);
@@ -442,9 +458,12 @@ int fmha_fwd_from_host(int dtype, const void* hQ, const void* hK, const void* hV
   g_last_cuda_error[0] = 0;
   cudaStream_t stream = reinterpret_cast<cudaStream_t>(stream_);
   if (dtype != 0 && dtype != 1) return FMHA_ERR_UNSUPPORTED;
-  if (batch < 0 || heads < 0 || seq_q < 0 || seq_kv < 0) return FMHA_ERR_INVALID_ARG;
+  // every argument check happens before anything is enqueued (include/fmha.h)
+  if (mask && mask->kind == FMHA_MASK_KEY_BIAS) return FMHA_ERR_UNSUPPORTED;  // (fmha_fwd only)
+  bool empty = false;
+  if (int vs = validate_shape(batch, heads, seq_q, seq_kv, head_dim, scale, mask, 1, &empty); vs != FMHA_OK || empty)
+    return vs;
   const size_t u = static_cast<size_t>(batch) * heads;
-  if (u == 0 || seq_q == 0) return FMHA_OK;
   if (!hQ || !hK || !hV || !hO || !workspace) return FMHA_ERR_INVALID_ARG;
   if (workspace_bytes < fmha_workspace_bytes(batch, heads, seq_q, seq_kv, head_dim)) return FMHA_ERR_INVALID_ARG;
   if ((reinterpret_cast<uintptr_t>(workspace) & 255u) != 0) return FMHA_ERR_MISALIGNED;
@@ -456,7 +475,6 @@ int fmha_fwd_from_host(int dtype, const void* hQ, const void* hK, const void* hV
   uint8_t* dV = dK + round_up(kvb, 256);
   int32_t* dL = reinterpret_cast<int32_t*>(dV + round_up(kvb, 256));
   fmha_mask_t dmask = {FMHA_MASK_NONE, nullptr, nullptr, 0};
-  if (mask && mask->kind == FMHA_MASK_KEY_BIAS) return FMHA_ERR_UNSUPPORTED;  // (fmha_fwd only)
   if (mask) {
     dmask.kind = mask->kind;
     if (mask->kind == FMHA_MASK_KEY_PADDING) {

@@ -12,7 +12,7 @@ import pytest
 import torch
 
 import paper_conf_asplos_hagedornfccgg23_b200 as fm
-from oracle import attention_fp64, attention_rows_fp64
+from oracle import attention_fp64
 from workloads import (CONFIGS, MASK_CAUSAL, MASK_KEY_PADDING, MASK_NONE, FmhaConfig, make_fmha_inputs)
 
 pytestmark = pytest.mark.gpu
@@ -125,23 +125,23 @@ def test_determinism_and_shard_consistency():
     assert torch.equal(o1[2:], o3)
 
 
-# ------------------------------------------------------------------ BASELINE sizes, sampled rows
+# ------------------------------------------------------------------ BASELINE sizes, full tensors
 FULL = ["bert_base_pad", "bert_large_384", "bert_large_512", "gpt_causal"]
 
 
+@pytest.mark.timeout(600)
 @pytest.mark.parametrize("name", FULL)
-def test_full_size_sampled(name):
+def test_full_size_full_oracle(name):
+    """Every BASELINE config at full size, in the launch configuration bench.py times (the same
+    fmha_fwd call: persistent grid, its item schedule incl. BERT-large-384's single-tile tail items),
+    compared with the full fp64 oracle on every element (BL5: 16.8M outputs, ~3 s of oracle; GPT
+    causal: 67M outputs, ~40 s)."""
     cfg = CONFIGS[name]
     q, k, v, kl = make_fmha_inputs(cfg)
     o = run(cfg, q, k, v, kl)
-    r = np.random.default_rng(7)
-    units = [(int(r.integers(cfg.batch)), int(r.integers(cfg.heads)), int(r.integers(cfg.seq_q))) for _ in range(96)]
-    units += [(0, 0, 0), (cfg.batch - 1, cfg.heads - 1, cfg.seq_q - 1), (cfg.batch - 1, 0, min(127, cfg.seq_q - 1)),
-              (0, cfg.heads - 1, min(128, cfg.seq_q - 1))]
-    ref = attention_rows_fp64(q, k, v, cfg.scale, units, kl, causal=cfg.mask == MASK_CAUSAL)
-    got = np.stack([o[b, h, i].double().cpu().numpy() for (b, h, i) in units])
-    check(got, ref, cfg.dtype, name)
     assert torch.isfinite(o).all()
+    ref = attention_fp64(q, k, v, cfg.scale, kl, causal=cfg.mask == MASK_CAUSAL)
+    check(o, ref, cfg.dtype, name)
 
 
 def test_tiny_config_full_oracle():

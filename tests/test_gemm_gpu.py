@@ -1,5 +1,8 @@
-"""GPU parity for gemm_bias_act (C ABI) against the fp64 oracle (R15 tolerance:
-|err| <= 2e-3 + 2^-10 |ref| elementwise and rel-L2 <= 1e-3)."""
+"""GPU parity for gemm_bias_act (C ABI) against the fp64 oracle.  Tolerance: SURVEY.md §8(c) C15,
+|err| <= 1e-3 + 2^-10 |ref| elementwise and rel-L2 <= 1e-3 (R15): the fp16 output's own
+rounding is <= 2^-11 |ref|, and the fp32 accumulation of K <= 4096 products of size <= 1/sqrt(K)
+adds < 1e-5 absolute, so the 1e-3 floor covers the ulp of outputs near zero and the erf/tanh
+approximations of the GELU epilogue (|err| <= 4e-7)."""
 
 import numpy as np
 import pytest
@@ -17,7 +20,7 @@ ACTS = {"none": 0, "relu": 1, "gelu": 2, "gelu_tanh": 3}
 def check(c, ref, what):
     got = c.double().cpu().numpy()
     assert np.all(np.isfinite(got))
-    bad = np.abs(got - ref) > 2e-3 + 2 ** -10 * np.abs(ref)
+    bad = np.abs(got - ref) > 1e-3 + 2 ** -10 * np.abs(ref)
     rel = np.linalg.norm(got - ref) / max(np.linalg.norm(ref), 1e-30)
     assert not bad.any() and rel <= 1e-3, f"{what}: {bad.sum()} elems out of tol, rel-L2={rel:.3e}"
 

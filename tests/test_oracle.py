@@ -405,6 +405,23 @@ def test_mlp_brute_force_tiny(seed):
                                rtol=0, atol=1e-12)
 
 
+@pytest.mark.parametrize("seed", [3, 4])
+def test_mlp_rows_sampler_brute_force(seed):
+    """mlp_fused_rows_fp64 (the row-sampled checker of the GPU tests) against the pure-Python loops
+    on the selected rows only: rows in any order, duplicated, first and last."""
+    from oracle import mlp_fused_rows_fp64
+    rng = np.random.default_rng(seed)
+    m, n, L = 7, 6, 3
+    x = rng.uniform(-1, 1, (m, n)).astype(np.float16)
+    w = (rng.standard_normal((L, n, n)) * 0.6).astype(np.float16)
+    b = rng.uniform(-0.3, 0.3, (L, n)).astype(np.float16)
+    rows = [6, 0, 3, 3, 5]
+    got = mlp_fused_rows_fp64(x, w, b, rows, ACT_RELU)
+    want = _mlp_brute([x[r].tolist() for r in rows], w.tolist(), b.tolist())
+    assert got.shape == (len(rows), n)
+    np.testing.assert_allclose(got, want, rtol=0, atol=1e-12)
+
+
 def test_mlp_identity_weights_closed_form():
     """W_l = I, b_l = c >= 0, X >= 0 (ReLU): every layer adds c exactly, so Y = X + L c."""
     from oracle import mlp_fused_fp64

@@ -308,3 +308,28 @@ def make_fused_mlp_inputs(m: int, width: int, layers: int, seed: int = SEED, cfg
     w = (r(1).standard_normal((layers, width, width), dtype=np.float32) * np.sqrt(2.0 / width)).astype(np.float32)
     b = r(2).uniform(-0.1, 0.1, (layers, width)).astype(np.float32)
     return tuple(_round(a, torch.float16) for a in (x, w, b))
+
+
+# ------------------------------------------------------------------ score-ramp inputs (lazy rescale)
+def ramp_spikes(seq_kv: int, tile: int = 128):
+    """Positions of the 'spike' keys of the score-ramp inputs: one key per `tile`-key block t, at
+    128 t + (7 + 37 t) % 128 (t = 0 has none).  Returns a list of (t, key index)."""
+    return [(t, t * tile + (7 + 37 * t) % tile) for t in range(1, (seq_kv + tile - 1) // tile)
+            if t * tile + (7 + 37 * t) % tile < seq_kv]
+
+
+def add_score_ramp(q: torch.Tensor, k: torch.Tensor, scale: float, step_log2: float = 9.0):
+    """Score-ramp variant of [.., S, D] inputs (q, k CPU tensors, modified copies returned): feature 0
+    of every query row i gets a_i = (0, 0.5, 1, 2)[i % 4] and feature 0 of spike key t (see
+    ramp_spikes) gets t * step_log2 * ln(2) / scale, so row i's largest score grows by about
+    a_i * step_log2 (in log2 units) at every 128-key block: rows with a_i >= 1 move their max by
+    more than 8 (log2) from one KV tile to the next, a_i = 0.5 every second tile, a_i = 0 never.
+    Input construction only (no arithmetic of the method); feature 0 of the other keys is 0."""
+    q, k = q.clone(), k.clone()
+    sq, skv = q.shape[-2], k.shape[-2]
+    a = torch.tensor([0.0, 0.5, 1.0, 2.0], dtype=torch.float32)[torch.arange(sq) % 4]
+    q[..., :, 0] = a.to(q.dtype)
+    k[..., :, 0] = 0
+    for t, j in ramp_spikes(skv):
+        k[..., j, 0] = float(t * step_log2 * np.log(2.0) / scale)
+    return q, k
