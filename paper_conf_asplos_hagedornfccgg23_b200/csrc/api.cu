@@ -12,6 +12,7 @@
 
 #include "../../include/fmha.h"
 #include "fmha_kernel.cuh"
+#include "fmha_ks_kernel.cuh"
 #include "gemm_kernel.cuh"
 #include "mlp_kernel.cuh"
 #include "splitkv_kernel.cuh"
@@ -102,7 +103,7 @@ int make_map_3d(CUtensorMap* m, const void* base, bool bf16, uint64_t cols, uint
 // stride `tok_stride` elements, box {64, 1, 128}: one head's 128-token x 64-d block (the same
 // 128 rows x 128 B SWIZZLE_128B smem tile as the dense map).  Tokens >= T read as zero.
 int make_map_thd(CUtensorMap* m, const void* base, bool bf16, uint64_t d, uint64_t heads, uint64_t tokens,
-                 uint64_t tok_stride) {
+                 uint64_t tok_stride, uint32_t box_tokens = 128) {
   EncodeTiledFn enc = get_encode_fn();
   if (!enc) {
     snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "cuTensorMapEncodeTiled entry point unavailable");
@@ -110,7 +111,7 @@ int make_map_thd(CUtensorMap* m, const void* base, bool bf16, uint64_t d, uint64
   }
   cuuint64_t dims[3] = {d, heads, tokens};
   cuuint64_t strides[2] = {d * 2, tok_stride * 2};
-  cuuint32_t box[3] = {64, 1, 128};
+  cuuint32_t box[3] = {64, 1, box_tokens};
   cuuint32_t estr[3] = {1, 1, 1};
   CUresult r = enc(m, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 3,
                    const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
@@ -125,6 +126,42 @@ int make_map_thd(CUtensorMap* m, const void* base, bool bf16, uint64_t d, uint64
 
 bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
+// Key-split kernel (fmha_ks_kernel.cuh) for D = 64 in the dense, cross-unit pair and varlen modes.
+// B200_FMHA_KS=0 selects the two-tile kernel instead (A/B measurements only).
+bool ks_enabled() {
+  static const bool on = [] {
+    const char* v = std::getenv("B200_FMHA_KS");
+    return !(v && v[0] == '0');
+  }();
+  return on;
+}
+
+template <bool BF16>
+int launch_fmha_ks(const b200::FmhaParams& prm, int mode, int sm_count, cudaStream_t stream) {
+  using C = b200::FmhaKsCfg;
+  void (*kern)(b200::FmhaParams) = mode == b200::MODE_DENSE    ? b200::fmha_fwd_ks_sm100<BF16, b200::MODE_DENSE>
+                                   : mode == b200::MODE_PAIRX  ? b200::fmha_fwd_ks_sm100<BF16, b200::MODE_PAIRX>
+                                   : mode == b200::MODE_VARLEN ? b200::fmha_fwd_ks_sm100<BF16, b200::MODE_VARLEN>
+                                                               : b200::fmha_fwd_ks_sm100<BF16, b200::MODE_VARLEN_SCHED>;
+  static bool attr_done[64][4];
+  static std::mutex mu;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    if (dev >= 64 || !attr_done[dev][mode]) {
+      cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_ALLOC);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(fmha_ks)");
+      if (dev < 64) attr_done[dev][mode] = true;
+    }
+  }
+  dim3 grid(static_cast<unsigned>(std::min(prm.num_items, sm_count)), 1, 1);
+  const bool pdl = mode != b200::MODE_VARLEN && mode != b200::MODE_VARLEN_SCHED;
+  cudaError_t e = b200::launch_pdl(pdl, kern, grid, dim3(C::THREADS), C::SMEM_ALLOC, stream, prm);
+  if (e != cudaSuccess) return cuda_fail(e, "fmha_fwd_ks_kernel launch");
+  return FMHA_OK;
+}
+
 template <int D, bool BF16>
 int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) {
   using C = b200::FmhaCfg<D>;
@@ -138,6 +175,7 @@ int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) 
                                    : mode == b200::MODE_SPLIT  ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_SPLIT>
                                    : mode == b200::MODE_BIAS   ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_BIAS>
                                                                : b200::fmha_fwd_sm100<D, BF16, b200::MODE_VARLEN_SCHED>;
+  if (D == 64 && mode <= b200::MODE_VARLEN_SCHED && ks_enabled()) return launch_fmha_ks<BF16>(prm, mode, sm_count, stream);
   static bool attr_done[64][6];
   int dev = 0;
   cudaGetDevice(&dev);
@@ -243,6 +281,7 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   if ((st = make_map_3d(&prm.tmK, K, bf16, head_dim, seq_kv, units, 128)) != FMHA_OK) return st;
   if ((st = make_map_3d(&prm.tmV, V, bf16, head_dim, seq_kv, units, 128)) != FMHA_OK) return st;
   if ((st = make_map_3d(&prm.tmO, O, bf16, head_dim, seq_q, units, 128)) != FMHA_OK) return st;
+  if ((st = make_map_3d(&prm.tmO32, O, bf16, head_dim, seq_q, units, 32)) != FMHA_OK) return st;
   prm.kv_len = (kind == FMHA_MASK_KEY_PADDING) ? mask->kv_len : nullptr;
   prm.cu_seqlens = nullptr;
   prm.seq_q = seq_q;
@@ -340,6 +379,7 @@ int fmha_varlen_common(bool bf16, const void* QKV, void* O, const int32_t* cu_se
   if ((st = make_map_thd(&prm.tmK, base + 2 * hd, bf16, head_dim, heads, total_tokens, 3 * hd)) != FMHA_OK) return st;
   if ((st = make_map_thd(&prm.tmV, base + 4 * hd, bf16, head_dim, heads, total_tokens, 3 * hd)) != FMHA_OK) return st;
   if ((st = make_map_thd(&prm.tmO, O, bf16, head_dim, heads, total_tokens, hd)) != FMHA_OK) return st;
+  if ((st = make_map_thd(&prm.tmO32, O, bf16, head_dim, heads, total_tokens, hd, 32)) != FMHA_OK) return st;
   prm.kv_len = nullptr;
   prm.cu_seqlens = cu_seqlens;
   prm.o_ptr = static_cast<uint8_t*>(O);

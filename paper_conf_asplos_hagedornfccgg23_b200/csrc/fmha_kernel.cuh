@@ -100,6 +100,7 @@ struct FmhaParams {
   CUtensorMap tmK;  // 3-D {D, seq_kv, B*H}
   CUtensorMap tmV;
   CUtensorMap tmO;  // same geometry as Q
+  CUtensorMap tmO32;  // O with a 32-row box (key-split kernel: one store per (tile, lane quarter))
   const int32_t* kv_len;
   // Variable-length packed mode (fmha_fwd_varlen): sequence b of the batch is
   // tokens [cu_seqlens[b], cu_seqlens[b+1]) of QKV [T, 3, H, D] / O [T, H, D]; the tensor maps are
