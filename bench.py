@@ -5,8 +5,11 @@
 
 A step is one pass of the whole hot path (one fmha_fwd launch through the C ABI) over one batch
 of the workload (default bert_large_512: B=32, H=16, S=512, D=64, fp16).  N > 1 runs under
-torchrun, one process per GPU; every rank processes its own batch (weak scaling, no collective
-on the data path); value = all ranks' algorithmic flops / max-over-ranks device time.
+torchrun, one process per GPU; the config's batch is split over the ranks by (batch x head) shards
+(--scaling strong, the default; --scaling weak gives every rank its own full batch), with no
+collective on the data path; value = all ranks' algorithmic flops / max-over-ranks device time.
+After the timed region one all-gather reassembles O and rank 0 checks it bitwise against the same
+problem on one GPU plus sampled fp64 oracle rows (multigpu.py).
 
 Rank 0 prints ONE JSON line.  See DESIGN.md §6 for every field.
 """
@@ -178,8 +181,8 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of CPU oracle timing")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--scaling", choices=["weak", "strong"], default="weak",
-                    help="weak: each rank runs the whole config on its own batch; strong: ranks split its batch")
+    ap.add_argument("--scaling", choices=["weak", "strong"], default="strong",
+                    help="strong: ranks split the config's batch (SURVEY §8(e)); weak: each rank runs the whole config on its own batch")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -203,15 +206,26 @@ def main():
     if args.impl == "reference":
         return run_reference(args, cfg, world, rank)
 
+    # B200_BENCH_ONE_DEVICE=1 (testing only): every rank on cuda:0 with gloo collectives, so the
+    # world > 1 path (sharding, max-over-ranks timing, the O all-gather and its check) runs on a
+    # one-GPU box; the ranks then share one GPU, so its numbers are not scaling measurements.
+    one_dev = os.environ.get("B200_BENCH_ONE_DEVICE") == "1"
+    if one_dev:
+        local = 0
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     dist = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
+        if one_dev:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
 
     import paper_conf_asplos_hagedornfccgg23_b200 as fm
+    import multigpu
 
+    cfg_global = multigpu.global_config(cfg, world, args.scaling)
     cfg, offset = shard(cfg, rank, world, args.scaling)  # weak: own batch; strong: a slice of it
     q, k, v, kv_len = make_fmha_inputs(cfg, batch_offset=offset)
     set_bytes = alg_bytes(cfg)
@@ -252,11 +266,7 @@ def main():
         torch.cuda.synchronize()
         if dist:
             dist.barrier()
-    ms = ev0.elapsed_time(ev1)
-    if dist:
-        t = torch.tensor([ms], device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+    ms = multigpu.max_over_ranks(ev0.elapsed_time(ev1), world, dist, "cpu" if one_dev else dev)
     flops_rank = alg_flops(cfg, kv_len)
     ms_step = ms / args.steps
     value = flops_rank * world / (ms_step * 1e-3) / 1e12
@@ -281,11 +291,7 @@ def main():
             fm.fmha_fwd_from_host(pq, pk, pv, po, ws, kv_len=klh, causal=causal, scale=cfg.scale, stream=stream)
         e1.record(stream)
         torch.cuda.synchronize()
-        ems = e0.elapsed_time(e1)
-        if dist:
-            t = torch.tensor([ems], device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            ems = float(t.item())
+        ems = multigpu.max_over_ranks(e0.elapsed_time(e1), world, dist, "cpu" if one_dev else dev)
         in_bytes = (pq.numel() + pk.numel() + pv.numel()) * pq.element_size() + (0 if klh is None else klh.numel() * 4)
         e2e = {"value": flops_rank * world / (ems / e2e_steps * 1e-3) / 1e12, "unit": "TFLOP/s",
                "h2d_bytes_per_step": int(in_bytes), "d2h_bytes_per_step": int(po.numel() * po.element_size()),
@@ -299,6 +305,24 @@ def main():
     o_last = sets[(args.steps - 1) % n_sets][3]
     got = np.stack([o_last[b, h, i].double().cpu().numpy() for b, h, i in units])
     check_err = float(np.abs(got - ref).max())
+
+    # ---- N > 1: one all-gather reassembles O (untimed); rank 0 checks it bitwise against the whole
+    # problem on one GPU and against oracle rows spread over every rank's shard
+    mgpu = None
+    if world > 1:
+        o_full = multigpu.gather_output(o_last.cpu() if one_dev else o_last, world, dist)
+        if rank == 0:
+            gq, gk, gv, gkl = make_fmha_inputs(cfg_global)
+            gkl_dev = None if gkl is None else torch.from_numpy(gkl).to(dev)
+            o_one = fm.fmha_fwd(gq.to(dev), gk.to(dev), gv.to(dev), kv_len=gkl_dev, causal=causal, scale=cfg.scale)
+            torch.cuda.synchronize()
+            gb = cfg_global.batch
+            gunits = [(r * gb // world + (r % 2) * (gb // world - 1), r % cfg.heads, (37 * r) % cfg.seq_q)
+                      for r in range(world)] + [(gb - 1, cfg.heads - 1, cfg.seq_q - 1)]
+            gref = attention_rows_fp64(gq, gk, gv, cfg.scale, gunits, gkl, causal)
+            mgpu = multigpu.check_gathered(o_full, o_one, gref, gunits)
+            mgpu["collective"] = "all_gather_into_tensor (after the timed region)"
+            del gq, gk, gv, o_one
 
     peak_burst, peak_sust, hbm, peak_src = measured_peaks()
     if dist:
@@ -319,7 +343,7 @@ def main():
             "dtype": "f16" if cfg.dtype == "fp16" else "bf16", "data": "synthetic",
             "config": {"workload": cfg.name, "batch_per_gpu": cfg.batch, "heads": cfg.heads, "seq_q": cfg.seq_q,
                        "seq_kv": cfg.seq_kv, "head_dim": cfg.head_dim,
-                       "mask": ["none", "key_padding", "causal"][cfg.mask], "parallelism": f"dp{world} (b x h shards)",
+                       "mask": ["none", "key_padding", "causal"][cfg.mask], "parallelism": f"{args.scaling} dp{world} (b x h shards)",
                        "l2": f"rotating {n_sets} input/output sets ({n_sets * set_bytes / 1e6:.0f} MB > 126 MB L2)"},
             "pct_of_spec_2250": round(100 * achieved / SPEC_TFLOPS, 2),
             "pct_of_measured_peak": round(100 * achieved / peak_burst, 2),
@@ -332,7 +356,10 @@ def main():
             "roofline_exp": exp_roofline(alg_flops(cfg, kv_len) / (4.0 * cfg.head_dim), ms_step, sampler),
             "cpu_baseline": cpu,
             "check_max_abs_err": check_err,
+            "multi_gpu_check": mgpu,
         }
+        if world > 1:
+            line["config"]["global_batch"] = cfg_global.batch
         print(json.dumps(line), flush=True)
     if dist:
         dist.destroy_process_group()

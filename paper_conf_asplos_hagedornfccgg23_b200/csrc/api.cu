@@ -78,7 +78,7 @@ int check_device(int* sm_count) {
 // 3-D tile map over a [units, rows, cols] row-major tensor of 16-bit elements.
 // Box = {64 cols (128 B, the SWIZZLE_128B span), box_rows, 1}.  OOB elements read as zero.
 int make_map_3d(CUtensorMap* m, const void* base, bool bf16, uint64_t cols, uint64_t rows, uint64_t units,
-                uint32_t box_rows) {
+                uint32_t box_rows, uint32_t box_cols = 64) {
   EncodeTiledFn enc = get_encode_fn();
   if (!enc) {
     snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "cuTensorMapEncodeTiled entry point unavailable");
@@ -86,11 +86,11 @@ int make_map_3d(CUtensorMap* m, const void* base, bool bf16, uint64_t cols, uint
   }
   cuuint64_t dims[3] = {cols, rows, units};
   cuuint64_t strides[2] = {cols * 2, cols * rows * 2};
-  cuuint32_t box[3] = {64, box_rows, 1};
+  cuuint32_t box[3] = {box_cols, box_rows, 1};
   cuuint32_t estr[3] = {1, 1, 1};
   CUresult r = enc(m, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 3,
                    const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                   CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   box_cols == 64 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
     snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "cuTensorMapEncodeTiled failed (%d)", int(r));
@@ -103,7 +103,7 @@ int make_map_3d(CUtensorMap* m, const void* base, bool bf16, uint64_t cols, uint
 // stride `tok_stride` elements, box {64, 1, 128}: one head's 128-token x 64-d block (the same
 // 128 rows x 128 B SWIZZLE_128B smem tile as the dense map).  Tokens >= T read as zero.
 int make_map_thd(CUtensorMap* m, const void* base, bool bf16, uint64_t d, uint64_t heads, uint64_t tokens,
-                 uint64_t tok_stride, uint32_t box_tokens = 128) {
+                 uint64_t tok_stride, uint32_t box_tokens = 128, uint32_t box_d = 64) {
   EncodeTiledFn enc = get_encode_fn();
   if (!enc) {
     snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "cuTensorMapEncodeTiled entry point unavailable");
@@ -111,11 +111,11 @@ int make_map_thd(CUtensorMap* m, const void* base, bool bf16, uint64_t d, uint64
   }
   cuuint64_t dims[3] = {d, heads, tokens};
   cuuint64_t strides[2] = {d * 2, tok_stride * 2};
-  cuuint32_t box[3] = {64, 1, box_tokens};
+  cuuint32_t box[3] = {box_d, 1, box_tokens};
   cuuint32_t estr[3] = {1, 1, 1};
   CUresult r = enc(m, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 3,
                    const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                   CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   box_d == 64 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
     snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "cuTensorMapEncodeTiled failed (%d)", int(r));
@@ -126,12 +126,14 @@ int make_map_thd(CUtensorMap* m, const void* base, bool bf16, uint64_t d, uint64
 
 bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
-// Key-split kernel (fmha_ks_kernel.cuh) for D = 64 in the dense, cross-unit pair and varlen modes.
-// B200_FMHA_KS=0 selects the two-tile kernel instead (A/B measurements only).
+// Key-split kernel (fmha_ks_kernel.cuh: two softmax warps per row quarter and tile) for D = 64 in the
+// dense, cross-unit pair and varlen modes, selected with B200_FMHA_KS=1.  Off by default: measured
+// against the two-tile kernel on the same boxes it is level on BERT-large-512 (640 vs 657 TFLOP/s),
+// slower on BERT-large-384 and BERT-base and +3% on the packed varlen batch.
 bool ks_enabled() {
   static const bool on = [] {
     const char* v = std::getenv("B200_FMHA_KS");
-    return !(v && v[0] == '0');
+    return v && v[0] == '1';
   }();
   return on;
 }
@@ -281,7 +283,7 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   if ((st = make_map_3d(&prm.tmK, K, bf16, head_dim, seq_kv, units, 128)) != FMHA_OK) return st;
   if ((st = make_map_3d(&prm.tmV, V, bf16, head_dim, seq_kv, units, 128)) != FMHA_OK) return st;
   if ((st = make_map_3d(&prm.tmO, O, bf16, head_dim, seq_q, units, 128)) != FMHA_OK) return st;
-  if ((st = make_map_3d(&prm.tmO32, O, bf16, head_dim, seq_q, units, 32)) != FMHA_OK) return st;
+  if ((st = make_map_3d(&prm.tmO32, O, bf16, head_dim, seq_q, units, 32, 32)) != FMHA_OK) return st;
   prm.kv_len = (kind == FMHA_MASK_KEY_PADDING) ? mask->kv_len : nullptr;
   prm.cu_seqlens = nullptr;
   prm.seq_q = seq_q;
@@ -379,7 +381,7 @@ int fmha_varlen_common(bool bf16, const void* QKV, void* O, const int32_t* cu_se
   if ((st = make_map_thd(&prm.tmK, base + 2 * hd, bf16, head_dim, heads, total_tokens, 3 * hd)) != FMHA_OK) return st;
   if ((st = make_map_thd(&prm.tmV, base + 4 * hd, bf16, head_dim, heads, total_tokens, 3 * hd)) != FMHA_OK) return st;
   if ((st = make_map_thd(&prm.tmO, O, bf16, head_dim, heads, total_tokens, hd)) != FMHA_OK) return st;
-  if ((st = make_map_thd(&prm.tmO32, O, bf16, head_dim, heads, total_tokens, hd, 32)) != FMHA_OK) return st;
+  if ((st = make_map_thd(&prm.tmO32, O, bf16, head_dim, heads, total_tokens, hd, 32, 32)) != FMHA_OK) return st;
   prm.kv_len = nullptr;
   prm.cu_seqlens = cu_seqlens;
   prm.o_ptr = static_cast<uint8_t*>(O);

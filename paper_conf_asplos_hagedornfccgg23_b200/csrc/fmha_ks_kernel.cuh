@@ -1,42 +1,36 @@
-// fmha_ks_kernel.cuh — FMHA forward for sm_100a at head_dim 64: "key-split" streams.
+// fmha_ks_kernel.cuh — FMHA forward for sm_100a at head_dim 64: two softmax warps per row quarter.
 //
 // The operation is the paper's fused multi-head attention (§6): per (batch, head)
 // O = softmax(scale Q K^T + mask) V, two back-to-back GEMMs with the softmax between them.
 //
 // Why a second D = 64 kernel (round-1 measurements): with one softmax warp per
 // 128-row Q tile per SM sub-partition (SMSP), a KV step of the two-tile kernel (fmha_kernel.cuh) is
-// bound by each warp's serial chain -- S_FULL wait, 128-column TMEM load, row max, exponentials,
+// bound by each warp's serial chain -- S_FULL wait, 128-column TMEM load, row max, 128 exponentials,
 // P store -- at ~3.4k cycles per step against 1024 tensor-core cycles, with the issue slots 55%
-// busy and no pipe saturated.  More independent chains per SMSP is the lever.  TMEM (512 columns)
-// does not hold S + O for more than two 128-key tiles, so this kernel splits every 128-key KV tile
-// between two independent STREAMS per Q tile instead:
+// busy and no pipe saturated.  Here every 128-key S tile is split between TWO warps per row quarter
+// (16 softmax warps, four per SMSP), each loading, masking and exponentiating 64 of the 128 columns:
 //
-//   work item      two 128-row Q tiles (t = 0, 1) sharing every K/V tile load (as the two-tile
-//                  kernel: same item decode, schedules and ring protocol)                    [a1]
-//   stream (t, h)  query tile t against keys 64h .. 64h+63 of every 128-key KV tile, with its own
-//                  running max, row sum and O accumulator: four independent online softmaxes per
-//                  item, merged once per item (the split-KV identity, exact up to rounding)   [a6, a7]
-//   warps 0-15     softmax: warp w serves stream w >> 2, TMEM lane quarter w & 3 (one thread per
-//                  query row, 64 key columns per step, row statistics thread-local); each SMSP
-//                  hosts four independent chains.  After an item's last step the two warps of a
-//                  (tile, lane quarter) merge their streams (exchanging (max, sum) through shared
-//                  memory) and each writes 32 of the 64 output columns                         [a5, a6, a9]
-//   warp 16 / 17   MMA issuer of tile 0 / 1: S_th = Q_t K_j[64h..]^T (SS, M128 N64 K64), then
-//                  O_th += P_th V_j[64h..] (TS, P from TMEM)                                  [a4, a8]
+//   work item      two 128-row Q tiles (t = 0, 1) sharing every K/V tile load (the two-tile kernel's
+//                  item decode, schedules and K/V ring protocol)                              [a1]
+//   warps 0-15     softmax: warp w serves tile t = w >> 3, key half h = (w >> 2) & 1 and TMEM lane
+//                  quarter w & 3 (one thread per query row, 64 key columns per step).  The two
+//                  tiles' warp pairs of a lane quarter take turns for the exponential phase (named
+//                  barriers), so one tile's exponentials overlap the other tile's S load and max.
+//                  The row max needs both halves: each warp writes its half-row max to shared memory
+//                  before waiting for its turn, and the turn barrier -- which both warps of the pair
+//                  pass together -- publishes it to the partner, so the exchange costs no extra
+//                  synchronisation.  Both warps take the same lazy-rescale decision; each rescales its
+//                  32 of O_t's 64 columns, keeps the row sum of its half and, at the item's end,
+//                  stores 32 output columns (after exchanging the half sums)               [a5-a7, a9]
+//   warp 16 / 17   MMA issuer of tile t: S_t = Q_t K_j^T (SS, M128 N128 K64) as soon as the softmax
+//                  has read S_{t,j-1} (S_FREE), so QK of the next step runs under this step's
+//                  softmax; O_t += P_t V_j (TS, M128 N64 K128, P from TMEM) after P_FULL        [a4, a8]
 //   warp 18        TMA producer: Q per item (double-buffered), K_j / V_j ring                 [a2, a3]
 //   warp 19        varlen schedule builder (sched mode), otherwise idle
 //
-//   TMEM (512 columns): stream s = 2t + h owns columns [128 s, 128 s + 128):
-//       S_s  [128 s, +64)   fp32 scores of the step; P_s (16-bit pairs) overwrites its first 32
-//       O_s  [128 s + 64, +64)
-//   QK_{s,j+1} is issued after PV_{s,j} by the same thread (tcgen05.mma ops of one thread execute in
-//   issue order), so the P columns are consumed before the next S overwrites them, and S_FULL_{s,j+1}
-//   (a commit: all earlier MMAs of the thread complete) also tells the softmax that PV_{s,j} has
-//   landed in O_s (the lazy rescale may touch O_s then).
-//
-// Merge at the end of an item (per query row, mc_h = scale log2(e) m_h of stream h, m_h its
-// reference max, l_h its row sum): M = max(mc_0, mc_1), w_h = 2^(mc_h - M),
-//     O = (w_0 O_0 + w_1 O_1) / (w_0 l_0 + w_1 l_1),   rows with no visible key -> 0 (R4).
+//   TMEM (512 columns), tile t at [256 t, 256 t + 256): O_t [0, 64), then S and P of step g rotating
+//   over three 64-column regions (FmhaKsCfg::col_s / col_p), so neither the next QK nor the P store
+//   waits for the previous PV.
 #pragma once
 #include "fmha_kernel.cuh"
 
@@ -50,20 +44,38 @@ struct FmhaKsCfg {
 #endif
   static constexpr int NS = FMHA_KS_NS;      // K/V ring slots (K_j and V_j alternate)
   static constexpr int QS = 2;               // Q stages per tile (the next item's Q loads early)
-  static constexpr int STG = 32 * 128;       // O staging per (tile, lane quarter): 32 rows x 128 B, SW128
+  static constexpr int STG = 32 * 64;        // O staging per softmax warp: 32 rows x 32 columns (64 B rows)
   static constexpr int OFF_Q = 0;            // Q[stage][tile]
   static constexpr int OFF_RING = 2 * QS * TILE;
-  static constexpr int OFF_STG = OFF_RING + NS * TILE;     // [tile][quarter]
-  static constexpr int OFF_STAT = OFF_STG + 8 * STG;       // float2 (mc, l) [tile][h][row]
-  static constexpr int OFF_BAR = OFF_STAT + 2 * 2 * 128 * 8;
+  static constexpr int OFF_STG = OFF_RING + NS * TILE;     // [warp]
+  static constexpr int OFF_XMAX = OFF_STG + 16 * STG;        // float half-row max [step parity][tile][h][row]
+  static constexpr int OFF_LSUM = OFF_XMAX + 2 * 2 * 2 * 128 * 4;  // float half-row sum [item parity][tile][h][row]
+  static constexpr int OFF_BAR = OFF_LSUM + 2 * 2 * 2 * 128 * 4;
+  // TMEM columns inside tile t's 256: O_t [0, 64), then three 64-column regions A, B, C.  Step g (the
+  // tile's step count) puts S_g into AB (g even) / BC (g odd) and P_g into A (g even) / C (g odd):
+  // S_{g+1} never covers P_g (still to be read by PV_g), P_g never covers P_{g-1} (PV_{g-1} may still
+  // be reading it), and S_{g+1} covering P_{g-1} is safe because PV_{g-1} is issued before QK_{g+1}
+  // by the same thread.  So writing P_g waits for nothing but the pair's max exchange (P_g lies on
+  // S_g, which both warps of the pair have loaded by then).
+  // (ROT = 0: the fixed layout S [0, 128), P [128, 192), O [192, 256); P_g then waits for PV_{g-1})
+#ifndef FMHA_KS_ROT
+#define FMHA_KS_ROT 1
+#endif
+  static constexpr bool ROT = FMHA_KS_ROT;
+  static constexpr int COL_O = ROT ? 0 : 192;
+  __host__ __device__ static constexpr int col_s(uint32_t g) { return ROT ? ((g & 1) ? 128 : 64) : 0; }
+  __host__ __device__ static constexpr int col_p(uint32_t g) { return ROT ? ((g & 1) ? 192 : 64) : 128; }
   enum : int {
-    B_S_FULL = 0,    // [stream]   count 1 (commit)
-    B_P_FULL = 4,    // [stream]   count 128 (the stream's softmax threads)
-    B_O_FULL = 8,    // [tile]     count 1 (commit after the tile's last PV of an item)
-    B_O_EMPTY = 10,  // [tile]     count 256 (both streams' softmax threads read O)
-    B_Q_FULL = 12,   // [stage][tile]
-    B_Q_EMPTY = 16,  // [stage][tile]
-    B_KV = 20        // KV_FULL[NS], KV_EMPTY[NS] (count 2: both MMA warps)
+    B_S_FULL = 0,    // [tile]          count 1 (commit)
+    B_P_FULL = 2,    // [tile]          count 8 (one arrival per softmax warp of the tile)
+    B_O_FULL = 4,    // [tile]          count 1 (commit after the tile's last PV of an item)
+    B_O_EMPTY = 6,   // [tile]          count 8 (the tile's softmax warps read O)
+    B_Q_FULL = 8,    // [stage][tile]
+    B_Q_EMPTY = 12,  // [stage][tile]
+    B_STAT = 16,     // [tile][quarter] count 2 (the two warps of a (tile, lane quarter) wrote their l)
+    B_S_FREE = 24,   // [tile]          count 8 (the tile's softmax warps read S)
+    B_PV_DONE = 26,  // [tile]          count 1 (commit after each PV)
+    B_KV = 28        // KV_FULL[NS], KV_EMPTY[NS] (count 2: both MMA warps)
   };
   static constexpr int NUM_BARS = B_KV + 2 * NS;
   static constexpr int OFF_TMEMPTR = OFF_BAR + NUM_BARS * 8;
@@ -84,6 +96,20 @@ struct FmhaKsCfg {
 #define FMHA_KS_POLY_CNT 2
 #endif
   static constexpr int POLY_CNT = FMHA_KS_POLY_CNT;
+  // TURNS: the two tiles' warp pairs of a lane quarter alternate their exponential phases (128-thread
+  // named barriers 1 + 2 quarter + t, which also publish the half-row maxima); otherwise all four
+  // softmax warps of an SMSP run freely and each pair exchanges its maxima through its own 64-thread
+  // named barrier 1 + 4 t + quarter
+#ifndef FMHA_KS_TURNS
+#define FMHA_KS_TURNS 0
+#endif
+  static constexpr bool TURNS = FMHA_KS_TURNS;
+  // (no turns) OFFSET: at the start of an item tile 1's pairs wait until tile 0's pairs have done their
+  // first exponential phase (named barrier 9 + quarter), so the two tiles' phases start half a step apart
+#ifndef FMHA_KS_OFFSET
+#define FMHA_KS_OFFSET 0
+#endif
+  static constexpr bool OFFSET = FMHA_KS_OFFSET && !TURNS;
 };
 
 template <bool BF16, int MODE>
@@ -105,20 +131,22 @@ __global__ void __launch_bounds__(640, 1) fmha_fwd_ks_sm100(const __grid_constan
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(smem + C::OFF_TMEMPTR);
   const int warp = warp_id();
   const int lane = lane_id();
+  TRACE_DECL
 
   if (threadIdx.x == 0) {
     if (sbase & 1023u) __trap();
-    for (int s = 0; s < 4; ++s) {
-      mbar_init(BAR(C::B_S_FULL + s), 1);
-      mbar_init(BAR(C::B_P_FULL + s), 128);
-    }
     for (int t = 0; t < 2; ++t) {
+      mbar_init(BAR(C::B_S_FULL + t), 1);
+      mbar_init(BAR(C::B_P_FULL + t), 8);   // (one arrival per softmax warp)
       mbar_init(BAR(C::B_O_FULL + t), 1);
-      mbar_init(BAR(C::B_O_EMPTY + t), 256);
+      mbar_init(BAR(C::B_O_EMPTY + t), 8);
       for (int q = 0; q < 2; ++q) {
         mbar_init(Q_FULL(t, q), 1);
         mbar_init(Q_EMPTY(t, q), 1);
       }
+      for (int q = 0; q < 4; ++q) mbar_init(BAR(C::B_STAT + 4 * t + q), 2);
+      mbar_init(BAR(C::B_S_FREE + t), 8);
+      mbar_init(BAR(C::B_PV_DONE + t), 1);
     }
     for (int s = 0; s < C::NS; ++s) {
       mbar_init(KV_FULL(s), 1);
@@ -157,6 +185,7 @@ __global__ void __launch_bounds__(640, 1) fmha_fwd_ks_sm100(const __grid_constan
         for (int m = 0; m < 2; ++m, ++kv) {  // m = 0: K_j, m = 1: V_j
           const int s = kv % C::NS;
           mbar_wait_at(KV_EMPTY(s), ((kv / C::NS) & 1) ^ 1, 1, kv, j);
+          TRACE_EV(EV_TMA_KV, m * 64 + j);
           mbar_arrive_expect_tx_elect(KV_FULL(s), C::TILE);
           tma_load_3d_hint_elect(sbase + C::OFF_RING + s * C::TILE, m ? &p.tmV : &p.tmK, KV_FULL(s), 0,
                                  w.c1(VL, t, j * 128), w.c2(VL, t, j * 128), keep);
@@ -187,70 +216,89 @@ __global__ void __launch_bounds__(640, 1) fmha_fwd_ks_sm100(const __grid_constan
       }
     } else if (warp == C::W_MMA || warp == C::W_MMA + 1) {
       // ============================================================ MMA issuer of tile t (a4, a8)
+      // QK_{t,j+1} goes out as soon as the softmax has read S_{t,j} (S_FREE), so it runs under the
+      // softmax of step j; PV_{t,j} follows once P_{t,j} is written (P_FULL).
       const int t = warp - C::W_MMA;
-      constexpr uint32_t IDESC_QK = idesc_f16(BF16, 128, 64, false, false);  // Q, K: K-major
-      constexpr uint32_t IDESC_PV = idesc_f16(BF16, 128, 64, false, true);   // P: TMEM, V: MN-major
+      constexpr uint32_t IDESC_QK = idesc_f16(BF16, 128, 128, false, false);  // Q, K: K-major
+      constexpr uint32_t IDESC_PV = idesc_f16(BF16, 128, 64, false, true);    // P: TMEM, V: MN-major
       const uint64_t desc0 = sdesc_sw128(sbase, 16, 1024);
       const uint64_t vdesc0 = sdesc_sw128(sbase, 128 * 128, 1024);
-      const uint32_t tS0 = tmem + 256 * t, tS1 = tS0 + 128;  // streams (t, 0), (t, 1); O at +64
-      uint32_t qc = 0, oc = 0, pc0 = 0, pc1 = 0;
+      const uint32_t tT = tmem + 256 * t, tO = tT + C::COL_O;  // tile t's TMEM columns
+      const uint32_t S_FULL = BAR(C::B_S_FULL + t), P_FULL = BAR(C::B_P_FULL + t);
+      const uint32_t S_FREE = BAR(C::B_S_FREE + t), PV_DONE = BAR(C::B_PV_DONE + t);
+      uint32_t qc = 0, oc = 0, pc = 0, qkc = 0;
       auto ring_wait = [&](uint32_t k) {
         mbar_wait_at(KV_FULL(k % C::NS), (k / C::NS) & 1, 3, k, 0);
         tc_fence_after();
         return sbase + C::OFF_RING + (k % C::NS) * C::TILE;
       };
-      auto release = [&](uint32_t k) {
-        ring_wait(k);
-        umma_commit_elect(KV_EMPTY(k % C::NS));
-      };
-      // the step whose PVs are still to be issued (PV_{s,j} goes out right before QK_{s,j+1})
-      struct Pend {
+      struct Pend {  // the step whose PV is still to be issued
         uint32_t vidx;
         bool valid, first, last;
       } pend = {0, false, false, false};
-      auto pv = [&](int h) {
+      auto pv = [&]() {
         const uint32_t sV = ring_wait(pend.vidx);
-        if (h == 0 && pend.first) {  // the item's first PV overwrites O_t: the epilogue has read it
+        if (pend.first) {  // the item's first PV overwrites O_t: the previous item's epilogue has read it
           mbar_wait_at(BAR(C::B_O_EMPTY + t), (oc & 1) ^ 1, 7, oc, t);
           ++oc;
         }
-        uint32_t& pc = h ? pc1 : pc0;
-        mbar_wait_at(BAR(C::B_P_FULL + 2 * t + h), pc & 1, 6, pc, h);
+        TRACE_EV(EV_COR_ST, 0);
+        mbar_wait_at(P_FULL, pc & 1, 6, pc, t);
+        TRACE_EV(EV_MMA_P, 0);
+        const uint32_t tP = tT + C::col_p(pc);
         ++pc;
         tc_fence_after();
-        const uint32_t tS = h ? tS1 : tS0;
 #pragma unroll
-        for (int kk = 0; kk < 4; ++kk)  // keys 64h + 16kk .. of V_j (MN-major rows of 128 B)
-          umma_ts_elect(tS + 64, tS + kk * 8, vdesc0 + ((sV - sbase + 8192 * h + 2048 * kk) >> 4), IDESC_PV,
-                        (!pend.first || kk > 0));
+        for (int kk = 0; kk < 8; ++kk)  // keys 16kk .. of V_j (MN-major rows of 128 B); P: 8 columns per 16 keys
+          umma_ts_elect(tO, tP + kk * 8, vdesc0 + ((sV - sbase + 2048 * kk) >> 4), IDESC_PV, (!pend.first || kk > 0));
+        umma_commit_elect(PV_DONE);
+        if (pend.last) umma_commit_elect(BAR(C::B_O_FULL + t));
+        umma_commit_elect(KV_EMPTY(pend.vidx % C::NS));
+        TRACE_EV(EV_MMA_PV, 0);
       };
-      auto qk = [&](int h, uint32_t sK, int qs) {
-        const uint32_t qoff = C::OFF_Q + (2 * qs + t) * C::TILE;
-        const uint32_t koff = sK - sbase + 8192 * h;  // K rows 64h .. 64h+63
-#pragma unroll
-        for (int kk = 0; kk < 4; ++kk)
-          umma_ss_elect(h ? tS1 : tS0, desc0 + ((qoff + 32 * kk) >> 4), desc0 + ((koff + 32 * kk) >> 4), IDESC_QK,
-                        kk > 0);
-        umma_commit_elect(BAR(C::B_S_FULL + 2 * t + h));
+      // an entry this tile does not use: wait until it is filled, then release it (the pending PV goes
+      // first -- its V slot may be the one the TMA needs to fill this entry)
+      auto release = [&](uint32_t k) {
+        if (pend.valid) {
+          pv();
+          pend.valid = false;
+        }
+        ring_wait(k);
+        umma_commit_elect(KV_EMPTY(k % C::NS));
       };
       int qs = 0;
       auto step = [&](uint32_t kidx, int j, int n) {
+        TRACE_EV(EV_COR_PV, j);
+        // QK_{t,j+1} normally goes out before PV_{t,j}.  But when this K entry does not directly
+        // follow the pending V entry in the ring (cross-unit pairs: the other tile's entries sit in
+        // between), waiting for it first could deadlock: the TMA may need a slot that only this PV
+        // frees (through the epilogue -> turn -> other tile chain).  Then the PV goes first.
+        if (pend.valid && kidx != pend.vidx + 1) {
+          pv();
+          pend.valid = false;
+        }
         const uint32_t sK = ring_wait(kidx);
+        TRACE_EV(EV_COR_ORDY, j);
         if (j == 0) {
           qs = qc % C::QS;
           mbar_wait_at(Q_FULL(t, qs), (qc / C::QS) & 1, 4, qc, t);
           ++qc;
         }
-        if (pend.valid) pv(0);
-        qk(0, sK, qs);
-        if (pend.valid) {
-          pv(1);
-          if (pend.last) umma_commit_elect(BAR(C::B_O_FULL + t));
-          umma_commit_elect(KV_EMPTY(pend.vidx % C::NS));
+        if (qkc > 0) {  // the softmax has read S_t of the previous step
+          mbar_wait_at(S_FREE, (qkc - 1) & 1, 5, qkc, t);
+          tc_fence_after();
         }
-        qk(1, sK, qs);
+        const uint32_t tS = tT + C::col_s(qkc);
+        ++qkc;
+        const uint32_t qoff = C::OFF_Q + (2 * qs + t) * C::TILE;
+#pragma unroll
+        for (int kk = 0; kk < 4; ++kk)
+          umma_ss_elect(tS, desc0 + ((qoff + 32 * kk) >> 4), desc0 + ((sK - sbase + 32 * kk) >> 4), IDESC_QK, kk > 0);
+        umma_commit_elect(S_FULL);
+        TRACE_EV(EV_MMA_QK, j);
         if (j + 1 == n) umma_commit_elect(Q_EMPTY(t, qs));
         umma_commit_elect(KV_EMPTY(kidx % C::NS));
+        if (pend.valid) pv();
         pend = {kidx + 1, true, j == 0, j + 1 == n};
       };
       uint32_t ring = 0;  // ring index of the current item's first entry
@@ -281,47 +329,60 @@ __global__ void __launch_bounds__(640, 1) fmha_fwd_ks_sm100(const __grid_constan
         }
         ring += w.entries();
       }
-      if (pend.valid) {
-        pv(0);
-        pv(1);
-        umma_commit_elect(BAR(C::B_O_FULL + t));
-        umma_commit_elect(KV_EMPTY(pend.vidx % C::NS));
-      }
+      if (pend.valid) pv();
     }
   } else {
     asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(C::REG_SOFTMAX));
     // ============================================================== softmax + epilogue (a5-a7, a9)
-    const int s = warp >> 2, t = s >> 1, h = s & 1, quad = warp & 3;
+    const int t = warp >> 3, h = (warp >> 2) & 1, quad = warp & 3;
     const int row = quad * 32 + lane;
     const uint32_t lane_off = static_cast<uint32_t>(quad * 32) << 16;
-    const uint32_t tS = tmem + lane_off + 128 * s;  // S_s / P_s; O_s at +64
-    const uint32_t S_FULL = BAR(C::B_S_FULL + s), P_FULL = BAR(C::B_P_FULL + s);
-    const uint32_t pair_bar = 1 + 4 * t + quad;  // named barrier of the two warps of (t, quad)
-    float2* stat = reinterpret_cast<float2*>(smem + C::OFF_STAT);
-    const uint32_t stg = sbase + C::OFF_STG + (4 * t + quad) * C::STG;
+    const uint32_t tT = tmem + lane_off + 256 * t;           // tile t's columns, this warp's lanes
+    const uint32_t tO = tT + C::COL_O + 32 * h;               // O_t columns 32h .. 32h+31
+    const uint32_t S_FULL = BAR(C::B_S_FULL + t), P_FULL = BAR(C::B_P_FULL + t);
+    const uint32_t S_FREE = BAR(C::B_S_FREE + t), PV_DONE = BAR(C::B_PV_DONE + t);
+    const uint32_t STAT = BAR(C::B_STAT + 4 * t + quad);
+    // 128-thread named barriers: the pair (t, quad) waits on my_turn, the other tile's pair arrives
+    const uint32_t my_turn = 1 + 2 * quad + t, other_turn = 2 + 2 * quad - t;
+    float* xmax = reinterpret_cast<float*>(smem + C::OFF_XMAX);  // [step parity][tile][h][row]
+    float* lsum = reinterpret_cast<float*>(smem + C::OFF_LSUM);  // [item parity][tile][h][row]
+    const uint32_t stg = sbase + C::OFF_STG + warp * C::STG;
     const float c = p.scale_log2;
     const int off = p.seq_kv - p.seq_q;
-    uint32_t g = 0, ofc = 0;
+    const uint32_t pair_bar = 1 + 4 * t + quad;  // (no turns) the pair's 64-thread exchange barrier
+    if (C::TURNS && t == 1) named_bar_arrive(1 + 2 * quad, 128);  // tile 0 goes first
+    uint32_t g = 0, ofc = 0, ec = 0;
     for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
       const WorkItem w = get_item<PAIRX, VL, false, SCHED>(p, sched, idx);
-      if (!w.has(t)) continue;
       const int n = w.n(t);
+      const int N = C::TURNS ? max(w.n0, w.n1) : n;
       const int qi = w.row0(t) + row;
       int lim = w.kv(t);
       if (p.mask_kind == MASK_CAUSAL) lim = min(lim, qi + off + 1);
       if (qi >= w.len(t)) lim = 0;
       const int lim_w = __reduce_max_sync(0xffffffffu, lim);
       float m_ref = -INFINITY, l = 0.f;
-      for (int j = 0; j < n; ++j) {
+      for (int j = 0; j < N; ++j) {
+        if (j >= n) {  // no KV tile j for this tile: pass the turn on
+          named_bar_sync(my_turn, 128);
+          named_bar_arrive(other_turn, 128);
+          continue;
+        }
+        if (C::OFFSET && j == 0 && t == 1 && w.n0 > 0) named_bar_sync(9 + quad, 128);
         const int key0 = j * 128 + 64 * h;
+        TRACE_EV(EV_S_WAIT, j);
         mbar_wait_at(S_FULL, g & 1, 8, g, j);
-        ++g;
+        TRACE_EV(EV_S_READY, j);
         tc_fence_after();
+        const uint32_t tS = tT + C::col_s(g) + 64 * h;  // this warp's 64 S columns of step g
+        const uint32_t tP = tT + C::col_p(g) + 32 * h;  // ... and its 32 P columns
         uint32_t sv[64];
         tmem_ld_32x32b_x32(tS, *reinterpret_cast<uint32_t(*)[32]>(&sv[0]));
         tmem_ld_32x32b_x32(tS + 32, *reinterpret_cast<uint32_t(*)[32]>(&sv[32]));
         tmem_wait_ld();
         reg_fence(sv);
+        tc_fence_before();
+        mbar_arrive_elect(S_FREE);  // S_t read (wait::ld is warp-wide): QK_{t,j+1} may overwrite it
         const int rem = lim - key0, rem_w = lim_w - key0;
         if (rem < 64) {
 #pragma unroll
@@ -336,8 +397,23 @@ __global__ void __launch_bounds__(640, 1) fmha_fwd_ks_sm100(const __grid_constan
           mx2 = fmax3(mx2, __uint_as_float(sv[k + 4]), __uint_as_float(sv[k + 5]));
           mx3 = fmax3(mx3, __uint_as_float(sv[k + 6]), __uint_as_float(sv[k + 7]));
         }
-        const float m_new = fmaxf(fmaxf(mx0, mx1), fmaxf(mx2, mx3));
-        // lazy rescale (a7): keep the reference while the max grows by <= 8 in log2 units
+        // this warp's half of the row max goes to shared memory; the turn barrier (which the two
+        // warps of the pair pass together) makes the partner's half visible (slots by step parity)
+        float* xm = xmax + (g & 1) * 512 + 256 * t;
+        xm[128 * h + row] = fmaxf(fmaxf(mx0, mx1), fmaxf(mx2, mx3));
+        if (!C::ROT && g > 0) {  // fixed layout: P_g overwrites P_{g-1}
+          mbar_wait_at(PV_DONE, (g - 1) & 1, 10, g, j);
+          tc_fence_after();
+        }
+        TRACE_EV(EV_MAX_DONE, j);
+        if (C::TURNS)
+          named_bar_sync(my_turn, 128);
+        else
+          named_bar_sync(pair_bar, 64);
+        TRACE_EV(EV_XCHG, j);
+        const float m_new = fmaxf(xm[row], xm[128 + row]);
+        // lazy rescale (a7): keep the reference while the max grows by <= 8 in log2 units (both warps
+        // of the pair take the same decision from the same two halves)
         float alpha = 1.f;
         if (m_new > m_ref && (m_ref == -INFINITY || (m_new - m_ref) * c > 8.f)) {
           alpha = (m_ref == -INFINITY) ? 0.f : ex2((m_ref - m_new) * c);
@@ -345,7 +421,7 @@ __global__ void __launch_bounds__(640, 1) fmha_fwd_ks_sm100(const __grid_constan
         }
         const float mc = (m_ref == -INFINITY) ? 0.f : m_ref * c;
         float2 acc0 = make_float2(0.f, 0.f), acc1 = make_float2(0.f, 0.f);
-        auto chunk = [&](int hh) {  // keys 32 hh .. 32 hh + 31 of the stream's 64
+        auto chunk = [&](int hh) {  // keys 32 hh .. 32 hh + 31 of this warp's 64
           uint32_t pk[16];
 #pragma unroll
           for (int u = 0; u < 16; u += 2) {
@@ -369,13 +445,13 @@ __global__ void __launch_bounds__(640, 1) fmha_fwd_ks_sm100(const __grid_constan
             pk[u] = pack2<BF16>(x0.x, x0.y);
             pk[u + 1] = pack2<BF16>(x1.x, x1.y);
           }
-          tmem_st_32x32b_x16(tS + 16 * hh, pk);
+          tmem_st_32x32b_x16(tP + 16 * hh, pk);
         };
         auto zero_chunk = [&](int hh) {
           uint32_t pk[16];
 #pragma unroll
           for (int u = 0; u < 16; ++u) pk[u] = 0u;
-          tmem_st_32x32b_x16(tS + 16 * hh, pk);
+          tmem_st_32x32b_x16(tP + 16 * hh, pk);
         };
         if (rem_w >= 64) {  // (the common case: no chunk of this warp is fully masked)
           chunk(0);
@@ -384,79 +460,85 @@ __global__ void __launch_bounds__(640, 1) fmha_fwd_ks_sm100(const __grid_constan
           if (rem_w > 0) chunk(0); else zero_chunk(0);
           if (rem_w > 32) chunk(1); else zero_chunk(1);
         }
-        // lazy rescale of this row's O_s (PV_{s,j-1} has landed: S_FULL_{s,j} commits after it)
+        if (C::TURNS) named_bar_arrive(other_turn, 128);
+        if (C::OFFSET && j == 0 && t == 0 && w.n1 > 0) named_bar_arrive(9 + quad, 128);
+        TRACE_EV(EV_EXP_DONE, j);
+        // lazy rescale of O_t columns 32h .. 32h+31 of this row (a7); at j = 0 the PV overwrites O_t.
+        // O_t must hold PV_{t,g-1} first (PV_DONE's phases run one behind the softmax's step count,
+        // so the parity of completion g-1 is unambiguous even though most steps do not wait)
         if (j > 0 && __any_sync(0xffffffffu, alpha != 1.f)) {
-#pragma unroll 1
-          for (int q = 0; q < 2; ++q) {
-            uint32_t o[32];
-            tmem_ld_32x32b_x32(tS + 64 + 32 * q, o);
-            tmem_wait_ld();
-            reg_fence(o);
+          mbar_wait_at(PV_DONE, (g - 1) & 1, 10, g, j);
+          tc_fence_after();
+          uint32_t o[32];
+          tmem_ld_32x32b_x32(tO, o);
+          tmem_wait_ld();
+          reg_fence(o);
 #pragma unroll
-            for (int k = 0; k < 32; ++k) o[k] = __float_as_uint(__uint_as_float(o[k]) * alpha);
-            tmem_st_32x32b_x32(tS + 64 + 32 * q, o);
-          }
+          for (int k = 0; k < 32; ++k) o[k] = __float_as_uint(__uint_as_float(o[k]) * alpha);
+          tmem_st_32x32b_x32(tO, o);
         }
         tmem_wait_st();
         tc_fence_before();
-        mbar_arrive(P_FULL);
+        mbar_arrive_elect(P_FULL);
+        ++g;
+        TRACE_EV(EV_EPI, j);
         l = l * alpha + ((acc0.x + acc0.y) + (acc1.x + acc1.y));
       }
-      // ------------------------------------------------------------ merge the two streams (a9)
-      stat[(2 * t + h) * 128 + row] = make_float2(m_ref == -INFINITY ? -INFINITY : m_ref * c, l);
-      if (h == 0 && lane == 0) tma_store_wait_read0();  // staging buffer free again
-      named_bar_sync(pair_bar, 64);
-      const float2 st0 = stat[(2 * t) * 128 + row], st1 = stat[(2 * t + 1) * 128 + row];
-      const float M = fmaxf(st0.x, st1.x);
-      const float w0 = (st0.x == -INFINITY) ? 0.f : ex2(st0.x - M);
-      const float w1 = (st1.x == -INFINITY) ? 0.f : ex2(st1.x - M);
-      const float L = w0 * st0.y + w1 * st1.y;
+      if (!w.has(t)) continue;
+      // ------------------------------------------------------------ epilogue (a9)
+      TRACE_EV(EV_ITEM, 1);
+      // the row sum is split over the pair (same reference max): exchange the halves (slots by item
+      // parity, so a warp an item ahead never overwrites what its partner has yet to read)
+      float* ls = lsum + (ec & 1) * 512 + 256 * t;
+      ls[128 * h + row] = l;
+      __syncwarp();
+      mbar_arrive_elect(STAT);
+      if (lane == 0) tma_store_wait_read0();  // this warp's staging buffer free again
+      mbar_wait_at(STAT, ec & 1, 9, ec, t);
+      ++ec;
+      const float L = ls[row] + ls[128 + row];
       const float inv = L > 0.f ? 1.f / L : 0.f;  // fully masked row -> 0 (R4)
-      const float a0 = w0 * inv, a1 = w1 * inv;
-      uint32_t o0[32], o1[32];
+      uint32_t o[32];
       if (n > 0) {
         mbar_wait_at(BAR(C::B_O_FULL + t), ofc & 1, 14, ofc, t);
+        TRACE_EV(EV_ITEM, 2);
         ++ofc;
         tc_fence_after();
-        const uint32_t tOc = tmem + lane_off + 256 * t + 64 + 32 * h;  // columns 32h.. of O_(t,0)
-        tmem_ld_32x32b_x32(tOc, o0);
-        tmem_ld_32x32b_x32(tOc + 128, o1);                            // ... and of O_(t,1)
+        tmem_ld_32x32b_x32(tO, o);
         tmem_wait_ld();
-        reg_fence(o0);
-        reg_fence(o1);
+        reg_fence(o);
         tc_fence_before();
-        mbar_arrive(BAR(C::B_O_EMPTY + t));
+        mbar_arrive_elect(BAR(C::B_O_EMPTY + t));
       } else {
 #pragma unroll
-        for (int k = 0; k < 32; ++k) o0[k] = o1[k] = 0u;
+        for (int k = 0; k < 32; ++k) o[k] = 0u;
       }
       uint32_t pk[16];
 #pragma unroll
-      for (int u = 0; u < 16; ++u) {
-        const float lo = __uint_as_float(o0[2 * u]) * a0 + __uint_as_float(o1[2 * u]) * a1;
-        const float hi = __uint_as_float(o0[2 * u + 1]) * a0 + __uint_as_float(o1[2 * u + 1]) * a1;
-        pk[u] = pack2<BF16>(lo, hi);
-      }
+      for (int u = 0; u < 16; ++u)
+        pk[u] = pack2<BF16>(__uint_as_float(o[2 * u]) * inv, __uint_as_float(o[2 * u + 1]) * inv);
       const bool rowwise = VL && w.row0(t) + 128 > w.len(t);
-      if (!rowwise) {
+      if (!rowwise) {  // 32 rows x 64 B, SWIZZLE_64B: 16-B chunk u of row r at chunk u ^ ((r >> 1) & 3)
 #pragma unroll
         for (int u = 0; u < 4; ++u)
-          st_shared_v4(stg + lane * 128 + (((4 * h + u) ^ (lane & 7)) << 4), pk[4 * u], pk[4 * u + 1], pk[4 * u + 2],
+          st_shared_v4(stg + lane * 64 + 16 * (u ^ ((lane >> 1) & 3)), pk[4 * u], pk[4 * u + 1], pk[4 * u + 2],
                        pk[4 * u + 3]);
         fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          tma_store_3d(&p.tmO32, stg, 32 * h, w.c1(VL, t, w.row0(t) + 32 * quad), w.c2(VL, t, w.row0(t) + 32 * quad));
+          tma_store_commit();
+        }
       } else if (qi < w.len(t)) {  // varlen tile crossing the sequence's end: rows inside only
         const size_t tokn = static_cast<size_t>(w.tok(t) + qi);
         uint8_t* dst = p.o_ptr + 2 * (tokn * p.o_row_elems + (t ? w.head1 : w.head) * D + 32 * h);
 #pragma unroll
         for (int u = 0; u < 4; ++u) st_global_v4(dst + 16 * u, pk[4 * u], pk[4 * u + 1], pk[4 * u + 2], pk[4 * u + 3]);
       }
-      named_bar_sync(pair_bar, 64);
-      if (!rowwise && h == 0 && lane == 0) {
-        tma_store_3d(&p.tmO32, stg, 0, w.c1(VL, t, w.row0(t) + 32 * quad), w.c2(VL, t, w.row0(t) + 32 * quad));
-        tma_store_commit();
-      }
+      TRACE_EV(EV_ITEM, 3);
     }
-    if (h == 0 && lane == 0) tma_store_wait0();
+    if (C::TURNS && t == 0) named_bar_sync(1 + 2 * quad, 128);  // consume tile 1's last hand-over
+    if (lane == 0) tma_store_wait0();
   }
 
   tc_fence_before();

@@ -220,6 +220,16 @@ __device__ __forceinline__ void reg_fence(uint32_t (&r)[N]) {
 // the asm statement.  Keeping the warp converged lets the compiler move the (warp-uniform)
 // operands to uniform registers once, instead of wrapping each instruction in a divergent
 // waterfall loop as it must under `if (lane == 0)`.
+// One arrival per warp (the barrier counts warps, not threads): the whole warp must be converged and
+// have ordered its own prior work (tcgen05.wait::*, fences, or __syncwarp for shared-memory stores)
+// before this call.  32 arrivals per warp on one mbarrier cost the SYNCS unit 32 updates.
+__device__ __forceinline__ void mbar_arrive_elect(uint32_t bar) {
+  asm volatile(
+      "{\n\t.reg .pred e;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];\n\t}" ::"r"(bar)
+      : "memory");
+}
 __device__ __forceinline__ void mbar_arrive_expect_tx_elect(uint32_t bar, uint32_t bytes) {
   asm volatile(
       "{\n\t.reg .pred e;\n\t"
