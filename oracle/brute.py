@@ -13,9 +13,10 @@ from __future__ import annotations
 import math
 
 
-def attention_brute(q, k, v, scale: float, kv_len=None, causal: bool = False, key_bias=None):
+def attention_brute(q, k, v, scale: float, kv_len=None, causal: bool = False, key_bias=None, attn_bias=None):
     """q: nested lists [B][H][Sq][D] of floats; k, v: [B][H][Skv][D]; key_bias None or
-    [B][Skv] additive bias (R20; -inf excludes the key).
+    [B][Skv] additive bias (R20; -inf excludes the key); attn_bias None or nested
+    lists [B][H][Sq][Skv] (R21; -inf excludes the pair).
     Returns nested lists [B][H][Sq][D]."""
     import struct
     scale = struct.unpack("f", struct.pack("f", scale))[0]  # fp32 value (DESIGN.md R1)
@@ -30,12 +31,14 @@ def attention_brute(q, k, v, scale: float, kv_len=None, causal: bool = False, ke
             for i in range(sq):
                 vis = [j for j in range(skv)
                        if j < limit and (not causal or j <= i + (skv - sq))
-                       and (key_bias is None or key_bias[b][j] != -math.inf)]
+                       and (key_bias is None or key_bias[b][j] != -math.inf)
+                       and (attn_bias is None or attn_bias[b][h][i][j] != -math.inf)]
                 if not vis:
                     oh.append([0.0] * d)
                     continue
                 s = {j: math.fsum(qb[i][t] * kb[j][t] for t in range(d)) * scale
-                     + (0.0 if key_bias is None else key_bias[b][j]) for j in vis}
+                     + (0.0 if key_bias is None else key_bias[b][j])
+                     + (0.0 if attn_bias is None else attn_bias[b][h][i][j]) for j in vis}
                 m = max(s.values())
                 e = {j: math.exp(s[j] - m) for j in vis}
                 l = math.fsum(e.values())

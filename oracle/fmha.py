@@ -33,6 +33,11 @@ Masking readings (the paper's FMHA has no mask; BASELINE.json configs add them):
       S = (Q @ K^T) * scale + bias[b, None, :], bias in natural-log units, shared by
       all heads and queries of batch b; bias = -inf excludes the key (R3), and a row
       whose every score is -inf yields O_i = 0 (R4).
+  R21 general additive (query x key) mask (SURVEY §8(f) f2 "arbitrary boolean/additive masks"; the
+      HF "extended attention mask" in its general [B, 1 or H, Sq, Skv] form): step 1 becomes
+      S = (Q @ K^T) * scale + attn_bias[b, h, i, j], attn_bias broadcastable to [B, H, Sq, Skv],
+      natural-log units; -inf excludes the pair (query i, key j) (R3); a row whose every score is
+      -inf yields O_i = 0 (R4).  A boolean mask M is the bias 0 where M, -inf elsewhere.
 """
 
 from __future__ import annotations
@@ -65,9 +70,10 @@ def visible_mask(sq: int, skv: int, kv_len: int | None, causal: bool) -> np.ndar
 
 
 def softmax_probs_fp64(q_bh, k_bh, scale: float, kv_len: int | None = None,
-                       causal: bool = False, key_bias=None) -> np.ndarray:
+                       causal: bool = False, key_bias=None, attn_bias=None) -> np.ndarray:
     """Steps 1-6 for one (b,h): the row-stochastic matrix P [Sq, Skv] (rows of zeros
-    where every key is masked, R4).  Exposed so tests can pin sum_j P[i,j] = 1."""
+    where every key is masked, R4).  Exposed so tests can pin sum_j P[i,j] = 1.
+    attn_bias: None or this (b, h)'s [Sq, Skv] additive bias (R21)."""
     q = _as_f64(q_bh)
     k = _as_f64(k_bh)
     sq, skv = q.shape[0], k.shape[0]
@@ -77,6 +83,10 @@ def softmax_probs_fp64(q_bh, k_bh, scale: float, kv_len: int | None = None,
         kb = np.asarray(key_bias, dtype=np.float64)[:skv]
         s = s + kb[None, :]
         vis = vis & (kb > -np.inf)[None, :]
+    if attn_bias is not None:                                # R21: general additive mask
+        ab = np.broadcast_to(np.asarray(attn_bias, dtype=np.float64), (sq, skv))
+        s = s + ab
+        vis = vis & (ab > -np.inf)
     s = np.where(vis, s, -np.inf)                            # step 2 (mask)
     any_vis = vis.any(axis=1)
     m = np.where(any_vis, s.max(axis=1, initial=-np.inf), 0.0)  # step 3 (max reduction)
@@ -86,12 +96,14 @@ def softmax_probs_fp64(q_bh, k_bh, scale: float, kv_len: int | None = None,
     return p
 
 
-def attention_fp64(q, k, v, scale: float, kv_len=None, causal: bool = False, key_bias=None) -> np.ndarray:
+def attention_fp64(q, k, v, scale: float, kv_len=None, causal: bool = False, key_bias=None,
+                   attn_bias=None) -> np.ndarray:
     """O = softmax(scale * Q K^T + mask) V for Q:[B,H,Sq,D], K,V:[B,H,Skv,D].
 
     ``kv_len`` is None or a length-B integer sequence (R5); ``key_bias`` None or
-    [B, >= Skv] additive bias (R20).  Returns float64
-    [B,H,Sq,D].  One (b,h) at a time, exactly steps 1-7 above.
+    [B, >= Skv] additive bias (R20); ``attn_bias`` None or an additive bias broadcastable
+    to [B, H, Sq, Skv] (R21).  Returns float64 [B,H,Sq,D].  One (b,h) at a time, exactly
+    steps 1-7 above.
     """
     q = _as_f64(q)
     k = _as_f64(k)
@@ -100,17 +112,18 @@ def attention_fp64(q, k, v, scale: float, kv_len=None, causal: bool = False, key
     skv = k.shape[2]
     assert k.shape == (b_, h_, skv, d) and v.shape == (b_, h_, skv, d)
     out = np.zeros((b_, h_, sq, d), dtype=np.float64)
+    ab = None if attn_bias is None else np.broadcast_to(_as_f64(attn_bias), (b_, h_, sq, skv))
     for b in range(b_):
         kl = None if kv_len is None else int(kv_len[b])
         for h in range(h_):
             kb = None if key_bias is None else np.asarray(key_bias, dtype=np.float64)[b]
-            p = softmax_probs_fp64(q[b, h], k[b, h], scale, kl, causal, kb)
+            p = softmax_probs_fp64(q[b, h], k[b, h], scale, kl, causal, kb, None if ab is None else ab[b, h])
             out[b, h] = p @ v[b, h]                          # step 7 (GEMM #2)
     return out
 
 
 def attention_rows_fp64(q, k, v, scale: float, units, kv_len=None,
-                        causal: bool = False, key_bias=None) -> np.ndarray:
+                        causal: bool = False, key_bias=None, attn_bias=None) -> np.ndarray:
     """Steps 1-7 for a sample of output rows only: ``units`` is a list of
     (b, h, i) triples; returns float64 [len(units), D].  Used for parity at full
     BASELINE sizes, where the whole oracle would take too long on the sampled
@@ -129,6 +142,10 @@ def attention_rows_fp64(q, k, v, scale: float, units, kv_len=None,
             bb = np.asarray(key_bias, dtype=np.float64)[b][:skv]
             s = s + bb
             vis = vis & (bb > -np.inf)
+        if attn_bias is not None:                            # R21
+            ab = np.broadcast_to(_as_f64(attn_bias), (q.shape[0], q.shape[1], sq, skv))[b, h, i]
+            s = s + ab
+            vis = vis & (ab > -np.inf)
         if not vis.any():
             res.append(np.zeros(vb.shape[1]))
             continue

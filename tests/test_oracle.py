@@ -566,3 +566,55 @@ def test_key_bias_rows_sampler_matches_full():
     units = [(0, 0, 0), (1, 1, 4), (0, 1, 2)]
     np.testing.assert_allclose(attention_rows_fp64(q, k, v, 0.25, units, key_bias=kb),
                                np.stack([full[b, h, i] for b, h, i in units]), rtol=0, atol=1e-13)
+
+
+# ---------------------------------------------------------------------------------------------
+# General additive (query x key) mask (R21): pins for attention_fp64(..., attn_bias=)
+
+
+@pytest.mark.parametrize("seed", [0, 1])
+def test_attn_bias_brute_force(seed):
+    q, k, v = _bias_case(seed, b=2, h=2, sq=5, skv=6)
+    rng = np.random.default_rng(200 + seed)
+    ab = rng.uniform(-3, 3, (2, 2, 5, 6))
+    ab[0, 1, 2, :4] = -np.inf
+    ab[1, 0, 4, :] = -np.inf  # a fully excluded row -> 0
+    got = attention_fp64(q, k, v, 0.5, attn_bias=ab)
+    want = np.array(attention_brute(q.astype(np.float64).tolist(), k.astype(np.float64).tolist(),
+                                    v.astype(np.float64).tolist(), 0.5, attn_bias=ab.tolist()))
+    np.testing.assert_allclose(got, want, rtol=0, atol=1e-12)
+    assert not got[1, 0, 4].any()
+
+
+def test_attn_bias_torch_sdpa_fp64():
+    """Library special case: torch SDPA with a float additive attn_mask [B, 1, Sq, Skv] (broadcast over
+    heads), in float64 on the CPU."""
+    b, h, sq, skv, d = 2, 3, 19, 23, 8
+    q, k, v = rnd((b, h, sq, d), 21), rnd((b, h, skv, d), 22), rnd((b, h, skv, d), 23)
+    ab = np.random.default_rng(24).uniform(-4, 2, (b, 1, sq, skv))
+    got = attention_fp64(q, k, v, 0.25, attn_bias=ab)
+    ref = torch.nn.functional.scaled_dot_product_attention(
+        torch.from_numpy(q), torch.from_numpy(k), torch.from_numpy(v), attn_mask=torch.from_numpy(ab),
+        scale=float(np.float32(0.25))).numpy()
+    np.testing.assert_allclose(got, ref, atol=1e-12, rtol=1e-10)
+
+
+def test_attn_bias_reduces_to_key_bias_causal_and_padding():
+    q, k, v = _bias_case(5, b=2, h=2, sq=6, skv=6)
+    kb = np.random.default_rng(25).uniform(-2, 2, (2, 6))
+    # a bias that does not depend on the query row is the key bias (R20)
+    np.testing.assert_array_equal(attention_fp64(q, k, v, 0.5, attn_bias=kb[:, None, None, :]),
+                                  attention_fp64(q, k, v, 0.5, key_bias=kb))
+    # -inf above the diagonal is the causal mask (R6, Sq = Skv); -inf past kv_len is key padding (R5)
+    tri = np.where(np.arange(6)[None, :] <= np.arange(6)[:, None], 0.0, -np.inf)
+    np.testing.assert_array_equal(attention_fp64(q, k, v, 0.5, attn_bias=tri), attention_fp64(q, k, v, 0.5, causal=True))
+    kl = np.array([6, 2])
+    pad = np.where(np.arange(6)[None, :] < kl[:, None], 0.0, -np.inf)[:, None, None, :]
+    np.testing.assert_array_equal(attention_fp64(q, k, v, 0.5, attn_bias=pad), attention_fp64(q, k, v, 0.5, kv_len=kl))
+    # sampled rows agree with the full oracle
+    ab = np.random.default_rng(26).uniform(-2, 2, (2, 2, 6, 6))
+    full = attention_fp64(q, k, v, 0.5, attn_bias=ab)
+    units = [(0, 1, 3), (1, 0, 5)]
+    rows = attention_rows_fp64(q, k, v, 0.5, units, attn_bias=ab)
+    for n, (bb, hh, ii) in enumerate(units):
+        np.testing.assert_allclose(rows[n], full[bb, hh, ii], rtol=0, atol=1e-14)
