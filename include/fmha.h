@@ -26,6 +26,11 @@
  *                          excludes the key.  key_bias: DEVICE fp32, 16-byte aligned;
  *                          key_bias_stride >= seq_kv and a multiple of 4; scale must be > 0.
  *                          fmha_fwd / fmha_fwd_bf16 only (other entry points: FMHA_ERR_UNSUPPORTED).
+ *   FMHA_MASK_ATTN_BIAS    general additive (query x key) mask (R21; the HF extended
+ *                          attention mask in its [B, 1 or H, Sq, Skv] form): S[i,j] = scale * <q_i,
+ *                          k_j> + attn_bias[b, h, i, j] (layout and strides in fmha_mask_t), natural-
+ *                          log units, -inf excludes the pair; scale must be > 0.  fmha_fwd,
+ *                          fmha_fwd_bf16 and fmha_fwd_strided only.
  * The kinds are exclusive.  A query row with no visible key produces O = 0 (never NaN).
  *
  * Ownership and errors: every tensor pointer is caller-owned; the library never allocates device
@@ -68,7 +73,8 @@ typedef enum {
   FMHA_MASK_NONE = 0,
   FMHA_MASK_KEY_PADDING = 1,
   FMHA_MASK_CAUSAL = 2,
-  FMHA_MASK_KEY_BIAS = 3
+  FMHA_MASK_KEY_BIAS = 3,
+  FMHA_MASK_ATTN_BIAS = 4
 } fmha_mask_kind_t;
 
 typedef struct {
@@ -76,7 +82,28 @@ typedef struct {
   const int32_t* kv_len;   /* DEVICE pointer, [batch]; required for KEY_PADDING, else ignored  */
   const float* key_bias;   /* DEVICE pointer, [batch, key_bias_stride]; KEY_BIAS only          */
   int32_t key_bias_stride; /* elements between batches of key_bias; KEY_BIAS only              */
+  /* ATTN_BIAS only: DEVICE pointer to the additive bias in the I/O type (fp16 for fmha_fwd, bf16
+   * for fmha_fwd_bf16 / dtype 1), element (b, h, i, j) at attn_bias[b * attn_bias_stride_b +
+   * h * attn_bias_stride_h + i * attn_bias_stride_q + j]; strides in elements, 0 broadcasts (e.g.
+   * attn_bias_stride_h = 0 for the HF [B, 1, Sq, Skv] mask); attn_bias_stride_q 0 (one row for every
+   * query; it must then hold seq_kv rounded up to 8 elements) or >= seq_kv and a multiple of 8; the
+   * pointer 16-byte aligned; columns j >= seq_kv of a row may be read, never used. */
+  const void* attn_bias;
+  int64_t attn_bias_stride_b;
+  int64_t attn_bias_stride_h;
+  int64_t attn_bias_stride_q;
 } fmha_mask_t;
+
+/* Element strides {batch, head, row} of Q, K, V and O for fmha_fwd_strided (head_dim is always
+ * contiguous).  Contiguous [B, H, S, D] is {H*S*D, S*D, D}; the HF / packed-projection layout
+ * [B, S, H, D] is {S*H*D, D, H*D}.  Every stride must be a multiple of 8 elements (16 bytes, the
+ * TMA requirement) and the row stride >= head_dim; overlapping outputs are not detected. */
+typedef struct {
+  int64_t q[3];
+  int64_t k[3];
+  int64_t v[3];
+  int64_t o[3];
+} fmha_strides_t;
 
 /* FMHA forward, fp16 in / fp16 out.
  *   Q, K, V, O : DEVICE pointers, 16-byte aligned, layouts above.
@@ -92,6 +119,15 @@ FMHA_API int fmha_fwd(const void* Q, const void* K, const void* V, void* O, cons
 /* Identical contract with bf16 tensors. */
 FMHA_API int fmha_fwd_bf16(const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask, int batch,
                   int heads, int seq_q, int seq_kv, int head_dim, float scale, fmha_stream_t stream);
+
+/* Strided layouts: the same operation as fmha_fwd with Q, K, V, O addressed
+ * through per-tensor {batch, head, row} element strides (fmha_strides_t, HOST pointer, read during the
+ * call), e.g. [B, S, H, D] tensors straight out of a QKV projection without a transpose.  dtype: 0 =
+ * fp16, 1 = bf16.  Masks, precision, ownership and errors as fmha_fwd; a stride TMA cannot address
+ * returns FMHA_ERR_INVALID_ARG before anything is launched.  strides == NULL means contiguous. */
+FMHA_API int fmha_fwd_strided(int dtype, const void* Q, const void* K, const void* V, void* O,
+                              const fmha_strides_t* strides, const fmha_mask_t* mask, int batch, int heads,
+                              int seq_q, int seq_kv, int head_dim, float scale, fmha_stream_t stream);
 
 /* Variable-length packed input: the MLPerf BERT inference format the paper's FMHA serves
  * (SURVEY.md §8(f) f2).  A batch of num_seqs sequences is stored back to back:

@@ -21,12 +21,12 @@ import math
 import torch
 
 from . import _lib
-from ._lib import FmhaError, FmhaMask
+from ._lib import FmhaError, FmhaMask, FmhaStrides
 
 __all__ = ["fmha_fwd", "fmha_fwd_splitkv", "fmha_fwd_varlen", "fmha_fwd_from_host", "gemm_bias_act", "dual_gemm_bias_act", "mlp_fused", "transformer_layer", "layer_workspace_bytes", "workspace_bytes", "FmhaError",
-           "MASK_NONE", "MASK_KEY_PADDING", "MASK_CAUSAL", "ACTS", "version"]
+           "MASK_NONE", "MASK_KEY_PADDING", "MASK_CAUSAL", "MASK_KEY_BIAS", "MASK_ATTN_BIAS", "ACTS", "version"]
 
-MASK_NONE, MASK_KEY_PADDING, MASK_CAUSAL, MASK_KEY_BIAS = 0, 1, 2, 3
+MASK_NONE, MASK_KEY_PADDING, MASK_CAUSAL, MASK_KEY_BIAS, MASK_ATTN_BIAS = 0, 1, 2, 3, 4
 ACTS = {"none": 0, "relu": 1, "gelu": 2, "gelu_erf": 2, "gelu_tanh": 3, "tanh": 4}
 
 
@@ -67,21 +67,37 @@ def _mask(kv_len, causal: bool):
     return FmhaMask(MASK_NONE, None)
 
 
+def _bhsd_strides(t: torch.Tensor, what: str):
+    """{batch, head, row} element strides of a [B, H, S, D] view whose last dimension is contiguous."""
+    if t.dim() != 4 or t.stride(3) != 1:
+        raise ValueError(f"{what} must be a 4-D [B,H,S,D] view with head_dim contiguous (stride 1)")
+    st = (t.stride(0), t.stride(1), t.stride(2))
+    # size-1 dimensions may carry any stride; give them a legal one for the tensor map
+    st = tuple(s if t.shape[i] > 1 else max(8, t.shape[3]) * max(1, t.shape[2]) for i, s in enumerate(st))
+    if any(s % 8 for s in st):
+        raise ValueError(f"{what}: strides must be multiples of 8 elements (16 bytes, TMA), got {st}")
+    return st
+
+
 def fmha_fwd(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, kv_len: torch.Tensor | None = None,
              causal: bool = False, scale: float | None = None, out: torch.Tensor | None = None,
-             key_bias: torch.Tensor | None = None) -> torch.Tensor:
-    """O = softmax(scale * Q K^T + mask) V.  q: [B,H,Sq,D], k/v: [B,H,Skv,D] contiguous CUDA
-    fp16/bf16 tensors; kv_len: CUDA int32 [B] (key padding) or None; causal: bottom-right mask;
-    key_bias: CUDA fp32 [B, stride >= Skv] additive per-key bias (stride % 4 == 0; -inf excludes a
-    key), exclusive with the other masks.  Calls ``fmha_fwd`` / ``fmha_fwd_bf16`` of the C ABI on
-    the current stream."""
+             key_bias: torch.Tensor | None = None, attn_bias: torch.Tensor | None = None) -> torch.Tensor:
+    """O = softmax(scale * Q K^T + mask) V.  q: [B,H,Sq,D], k/v: [B,H,Skv,D] CUDA fp16/bf16 tensors
+    (any strides with head_dim contiguous and the others multiples of 8 elements -- e.g. a [B,S,H,D]
+    tensor viewed with .transpose(1, 2); non-contiguous views go through ``fmha_fwd_strided``);
+    kv_len: CUDA int32 [B] (key padding) or None; causal: bottom-right mask; key_bias: CUDA fp32
+    [B, stride >= Skv] additive per-key bias (stride % 4 == 0; -inf excludes a key); attn_bias: a CUDA
+    tensor of q's dtype broadcastable to [B, H, Sq, Skv] (additive (query x key) mask, DESIGN.md R21;
+    its last dimension contiguous, row stride a multiple of 8 and >= Skv).  The mask kinds are
+    exclusive.  Calls ``fmha_fwd`` / ``fmha_fwd_bf16`` / ``fmha_fwd_strided`` of the C ABI on the
+    current stream."""
     lib = _lib.load()
     if q.dtype not in (torch.float16, torch.bfloat16) or k.dtype != q.dtype or v.dtype != q.dtype:
         raise TypeError("q, k, v must share dtype fp16 or bf16")
     if not (q.is_cuda and k.is_cuda and v.is_cuda):
         raise TypeError("q, k, v must be CUDA tensors (no CPU fallback)")
-    if not (q.is_contiguous() and k.is_contiguous() and v.is_contiguous()):
-        raise ValueError("q, k, v must be contiguous [B,H,S,D]")
+    if q.dim() != 4:
+        raise ValueError("q, k, v must be 4-D [B,H,S,D]")
     b, h, sq, d = q.shape
     skv = k.shape[2]
     if k.shape != (b, h, skv, d) or v.shape != k.shape:
@@ -91,24 +107,44 @@ def fmha_fwd(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, kv_len: torch.Te
             raise ValueError("kv_len must be a CUDA int32 tensor of length batch")
         kv_len = kv_len.contiguous()
     if out is None:
-        out = torch.empty_like(q)
-    else:
-        _check_out(out, q.shape, q.dtype, q, "fmha_fwd")
+        out = torch.empty((b, h, sq, d), dtype=q.dtype, device=q.device)
+    elif tuple(out.shape) != (b, h, sq, d) or out.dtype != q.dtype or out.device != q.device:
+        raise ValueError("out must be a [B,H,Sq,D] tensor of q's dtype on q's device")
     scale = 1.0 / math.sqrt(d) if scale is None else float(scale)
+    kinds = sum(x is not None and x is not False for x in (kv_len, causal or None, key_bias, attn_bias))
+    if kinds > 1:
+        raise ValueError("kv_len, causal, key_bias and attn_bias are exclusive")
     if key_bias is not None:
-        if kv_len is not None or causal:
-            raise ValueError("key_bias is exclusive with kv_len / causal")
         if key_bias.dtype != torch.float32 or not key_bias.is_cuda or key_bias.dim() != 2 or key_bias.shape[0] != b:
             raise ValueError("key_bias must be a CUDA float32 tensor [batch, stride]")
         if key_bias.stride(1) != 1:
             raise ValueError("key_bias rows must be contiguous")
         m = FmhaMask(MASK_KEY_BIAS, None, key_bias.data_ptr(), key_bias.stride(0))
+    elif attn_bias is not None:
+        if attn_bias.dtype != q.dtype or not attn_bias.is_cuda or attn_bias.device != q.device:
+            raise ValueError("attn_bias must be a CUDA tensor of q's dtype on q's device")
+        ab = attn_bias
+        while ab.dim() < 4:
+            ab = ab.unsqueeze(0)
+        ab = ab.expand(b, h, sq, skv)  # broadcast dimensions get stride 0
+        if ab.stride(3) != 1 or ab.stride(2) % 8 or 0 < ab.stride(2) < skv or (ab.stride(2) == 0 and skv % 8):
+            raise ValueError("attn_bias rows must be contiguous with a row stride >= Skv and a multiple of 8 "
+                             "(or 0, broadcast over queries, with Skv a multiple of 8)")
+        m = FmhaMask(MASK_ATTN_BIAS, None, None, 0, ab.data_ptr(), ab.stride(0), ab.stride(1), ab.stride(2))
     else:
         m = _mask(kv_len, causal)
-    fn = lib.fmha_fwd if q.dtype == torch.float16 else lib.fmha_fwd_bf16
-    st = fn(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), ctypes.byref(m), b, h, sq, skv, d,
-            scale, _stream_ptr(q.device))
-    _lib.check(st, "fmha_fwd")
+    st = _stream_ptr(q.device)
+    if all(t.is_contiguous() for t in (q, k, v, out)):
+        fn = lib.fmha_fwd if q.dtype == torch.float16 else lib.fmha_fwd_bf16
+        status = fn(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), ctypes.byref(m), b, h, sq, skv, d,
+                    scale, st)
+        _lib.check(status, "fmha_fwd")
+        return out
+    strides = FmhaStrides((ctypes.c_int64 * 3)(*_bhsd_strides(q, "q")), (ctypes.c_int64 * 3)(*_bhsd_strides(k, "k")),
+                          (ctypes.c_int64 * 3)(*_bhsd_strides(v, "v")), (ctypes.c_int64 * 3)(*_bhsd_strides(out, "out")))
+    status = lib.fmha_fwd_strided(0 if q.dtype == torch.float16 else 1, q.data_ptr(), k.data_ptr(), v.data_ptr(),
+                                  out.data_ptr(), ctypes.byref(strides), ctypes.byref(m), b, h, sq, skv, d, scale, st)
+    _lib.check(status, "fmha_fwd_strided")
     return out
 
 

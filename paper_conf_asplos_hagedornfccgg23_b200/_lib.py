@@ -27,6 +27,7 @@ STATUS_NAMES = {
 EXPORTED_SYMBOLS = (
     "fmha_fwd",
     "fmha_fwd_bf16",
+    "fmha_fwd_strided",
     "fmha_fwd_varlen",
     "fmha_workspace_bytes",
     "fmha_fwd_from_host",
@@ -46,7 +47,15 @@ EXPORTED_SYMBOLS = (
 
 class FmhaMask(ctypes.Structure):
     _fields_ = [("kind", ctypes.c_int32), ("kv_len", ctypes.c_void_p), ("key_bias", ctypes.c_void_p),
-                ("key_bias_stride", ctypes.c_int32)]
+                ("key_bias_stride", ctypes.c_int32), ("attn_bias", ctypes.c_void_p),
+                ("attn_bias_stride_b", ctypes.c_int64), ("attn_bias_stride_h", ctypes.c_int64),
+                ("attn_bias_stride_q", ctypes.c_int64)]
+
+
+class FmhaStrides(ctypes.Structure):
+    """fmha_strides_t: element strides {batch, head, row} of Q, K, V, O."""
+    _fields_ = [("q", ctypes.c_int64 * 3), ("k", ctypes.c_int64 * 3), ("v", ctypes.c_int64 * 3),
+                ("o", ctypes.c_int64 * 3)]
 
 
 class FmhaError(RuntimeError):
@@ -75,6 +84,9 @@ def load() -> ctypes.CDLL:
         f = getattr(lib, name)
         f.argtypes = [vp, vp, vp, vp, mp, i32, i32, i32, i32, i32, f32, vp]
         f.restype = i32
+    lib.fmha_fwd_strided.argtypes = [i32, vp, vp, vp, vp, ctypes.POINTER(FmhaStrides), mp, i32, i32, i32, i32, i32,
+                                      f32, vp]
+    lib.fmha_fwd_strided.restype = i32
     if hasattr(lib, "fmha_fwd_varlen"):  # absent only in old tuning builds (B200FMHA_LIB A/B runs)
         lib.fmha_fwd_varlen.argtypes = [vp, vp, vp, i32, i32, i32, i32, i32, f32, i32, i32, vp]
         lib.fmha_fwd_varlen.restype = i32

@@ -99,27 +99,29 @@ int make_map_3d(CUtensorMap* m, const void* base, bool bf16, uint64_t cols, uint
   return FMHA_OK;
 }
 
-// 3-D tile map over token-major [T, (3,) H, D] data (varlen packed mode): dims {D, H, T}, token
-// stride `tok_stride` elements, box {64, 1, 128}: one head's 128-token x 64-d block (the same
-// 128 rows x 128 B SWIZZLE_128B smem tile as the dense map).  Tokens >= T read as zero.
-int make_map_thd(CUtensorMap* m, const void* base, bool bf16, uint64_t d, uint64_t heads, uint64_t tokens,
-                 uint64_t tok_stride, uint32_t box_tokens = 128, uint32_t box_d = 64) {
+// 4-D tile map over a 16-bit tensor with head_dim contiguous and arbitrary row / head / batch strides
+// (elements; multiples of 8, i.e. 16 bytes, as TMA requires): dims {D, rows, heads, batch}, box
+// {box_cols, box_rows, 1, 1}.  SWIZZLE_128B for 64-column boxes, SWIZZLE_64B for 32-column ones.
+// Rows >= `rows` read as zero and are clipped on stores.
+int make_map_4d(CUtensorMap* m, const void* base, bool bf16, uint64_t d, uint64_t rows, uint64_t heads,
+                uint64_t batch, uint64_t s_row, uint64_t s_head, uint64_t s_batch, uint32_t box_rows,
+                uint32_t box_cols = 64) {
   EncodeTiledFn enc = get_encode_fn();
   if (!enc) {
     snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "cuTensorMapEncodeTiled entry point unavailable");
     return FMHA_ERR_CUDA;
   }
-  cuuint64_t dims[3] = {d, heads, tokens};
-  cuuint64_t strides[2] = {d * 2, tok_stride * 2};
-  cuuint32_t box[3] = {box_d, 1, box_tokens};
-  cuuint32_t estr[3] = {1, 1, 1};
-  CUresult r = enc(m, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 3,
+  cuuint64_t dims[4] = {d, rows, heads, batch};
+  cuuint64_t strides[3] = {s_row * 2, s_head * 2, s_batch * 2};
+  cuuint32_t box[4] = {box_cols, box_rows, 1, 1};
+  cuuint32_t estr[4] = {1, 1, 1, 1};
+  CUresult r = enc(m, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4,
                    const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                   box_d == 64 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                   box_cols == 64 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
-    snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "cuTensorMapEncodeTiled failed (%d)", int(r));
-    return FMHA_ERR_CUDA;
+    snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "cuTensorMapEncodeTiled (4-D) failed (%d)", int(r));
+    return FMHA_ERR_INVALID_ARG;  // e.g. a stride that is not a multiple of 16 bytes
   }
   return FMHA_OK;
 }
@@ -168,6 +170,7 @@ template <int D, bool BF16>
 int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) {
   using C = b200::FmhaCfg<D>;
   const int mode = prm.num_splits > 1 ? b200::MODE_SPLIT
+                   : prm.attn_bias  ? b200::MODE_BIAS2D
                    : prm.key_bias   ? b200::MODE_BIAS
                    : prm.cu_seqlens ? (prm.sched ? b200::MODE_VARLEN_SCHED : b200::MODE_VARLEN)
                                     : (prm.pair_mode ? b200::MODE_PAIRX : b200::MODE_DENSE);
@@ -176,9 +179,12 @@ int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) 
                                    : mode == b200::MODE_VARLEN ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_VARLEN>
                                    : mode == b200::MODE_SPLIT  ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_SPLIT>
                                    : mode == b200::MODE_BIAS   ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_BIAS>
+                                   : mode == b200::MODE_BIAS2D ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_BIAS2D>
                                                                : b200::fmha_fwd_sm100<D, BF16, b200::MODE_VARLEN_SCHED>;
   if (D == 64 && mode <= b200::MODE_VARLEN_SCHED && ks_enabled()) return launch_fmha_ks<BF16>(prm, mode, sm_count, stream);
-  static bool attr_done[64][6];
+  static bool attr_done[64][7];
+  static std::mutex attr_mu;
+  std::lock_guard<std::mutex> attr_lock(attr_mu);
   int dev = 0;
   cudaGetDevice(&dev);
   if (dev >= 64 || !attr_done[dev][mode]) {
@@ -242,8 +248,15 @@ int validate_shape(int batch, int heads, int seq_q, int seq_kv, int head_dim, fl
   if (scale < 0.f) return FMHA_ERR_UNSUPPORTED;
   const int kind = mask ? mask->kind : FMHA_MASK_NONE;
   if (kind != FMHA_MASK_NONE && kind != FMHA_MASK_KEY_PADDING && kind != FMHA_MASK_CAUSAL &&
-      kind != FMHA_MASK_KEY_BIAS)
+      kind != FMHA_MASK_KEY_BIAS && kind != FMHA_MASK_ATTN_BIAS)
     return FMHA_ERR_UNSUPPORTED;
+  if (kind == FMHA_MASK_ATTN_BIAS) {  // (R21) fmha_fwd / fmha_fwd_bf16 / fmha_fwd_strided; added as bias / scale
+    if (splits != 1 || !(scale > 0.f)) return FMHA_ERR_UNSUPPORTED;
+    if ((mask->attn_bias_stride_q != 0 && mask->attn_bias_stride_q < seq_kv) || mask->attn_bias_stride_q < 0 ||
+        (mask->attn_bias_stride_q % 8) != 0 || mask->attn_bias_stride_b < 0 ||
+        mask->attn_bias_stride_h < 0 || (mask->attn_bias_stride_b % 8) != 0 || (mask->attn_bias_stride_h % 8) != 0)
+      return FMHA_ERR_INVALID_ARG;
+  }
   if (kind == FMHA_MASK_KEY_BIAS) {  // (R20) fmha_fwd / fmha_fwd_bf16 only; the bias is added as bias / scale
     if (splits != 1 || !(scale > 0.f)) return FMHA_ERR_UNSUPPORTED;
     if (mask->key_bias_stride < seq_kv || (mask->key_bias_stride % 4) != 0) return FMHA_ERR_INVALID_ARG;
@@ -262,7 +275,8 @@ int validate_shape(int batch, int heads, int seq_q, int seq_kv, int head_dim, fl
 
 int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask,
                 int batch, int heads, int seq_q, int seq_kv, int head_dim, float scale, cudaStream_t stream,
-                int splits = 1, void* workspace = nullptr, size_t workspace_bytes = 0) {
+                int splits = 1, void* workspace = nullptr, size_t workspace_bytes = 0,
+                const fmha_strides_t* strides = nullptr) {
   g_last_cuda_error[0] = 0;
   bool empty = false;
   if (int vs = validate_shape(batch, heads, seq_q, seq_kv, head_dim, scale, mask, splits, &empty); vs != FMHA_OK || empty)
@@ -272,6 +286,8 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   if (!Q || !K || !V || !O) return FMHA_ERR_INVALID_ARG;
   if (kind == FMHA_MASK_KEY_BIAS && !mask->key_bias) return FMHA_ERR_INVALID_ARG;
   if (kind == FMHA_MASK_KEY_BIAS && !aligned16(mask->key_bias)) return FMHA_ERR_MISALIGNED;
+  if (kind == FMHA_MASK_ATTN_BIAS && !mask->attn_bias) return FMHA_ERR_INVALID_ARG;
+  if (kind == FMHA_MASK_ATTN_BIAS && !aligned16(mask->attn_bias)) return FMHA_ERR_MISALIGNED;
   if (!aligned16(Q) || !aligned16(K) || !aligned16(V) || !aligned16(O)) return FMHA_ERR_MISALIGNED;
   int sm_count = 0;
   int st = check_device(&sm_count);
@@ -279,11 +295,27 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
 
   b200::FmhaParams prm;
   memset(&prm, 0, sizeof(prm));
-  if ((st = make_map_3d(&prm.tmQ, Q, bf16, head_dim, seq_q, units, 128)) != FMHA_OK) return st;
-  if ((st = make_map_3d(&prm.tmK, K, bf16, head_dim, seq_kv, units, 128)) != FMHA_OK) return st;
-  if ((st = make_map_3d(&prm.tmV, V, bf16, head_dim, seq_kv, units, 128)) != FMHA_OK) return st;
-  if ((st = make_map_3d(&prm.tmO, O, bf16, head_dim, seq_q, units, 128)) != FMHA_OK) return st;
-  if ((st = make_map_3d(&prm.tmO32, O, bf16, head_dim, seq_q, units, 32, 32)) != FMHA_OK) return st;
+  // element strides {row, head, batch} of Q, K, V, O (contiguous [B, H, S, D] unless given)
+  const uint64_t D_ = head_dim;
+  fmha_strides_t cs;
+  const uint64_t qsz = D_ * seq_q, ksz = D_ * seq_kv;
+  const int64_t cq[3] = {static_cast<int64_t>(qsz * heads), static_cast<int64_t>(qsz), static_cast<int64_t>(D_)};
+  const int64_t ck[3] = {static_cast<int64_t>(ksz * heads), static_cast<int64_t>(ksz), static_cast<int64_t>(D_)};
+  for (int i = 0; i < 3; ++i) {
+    cs.q[i] = strides ? strides->q[i] : cq[i];
+    cs.k[i] = strides ? strides->k[i] : ck[i];
+    cs.v[i] = strides ? strides->v[i] : ck[i];
+    cs.o[i] = strides ? strides->o[i] : cq[i];
+  }
+  auto map4 = [&](CUtensorMap* m, const void* base, const int64_t* st3, uint64_t rows, uint32_t box_rows,
+                  uint32_t box_cols) {
+    return make_map_4d(m, base, bf16, D_, rows, heads, batch, st3[2], st3[1], st3[0], box_rows, box_cols);
+  };
+  if ((st = map4(&prm.tmQ, Q, cs.q, seq_q, 128, 64)) != FMHA_OK) return st;
+  if ((st = map4(&prm.tmK, K, cs.k, seq_kv, 128, 64)) != FMHA_OK) return st;
+  if ((st = map4(&prm.tmV, V, cs.v, seq_kv, 128, 64)) != FMHA_OK) return st;
+  if ((st = map4(&prm.tmO, O, cs.o, seq_q, 128, 64)) != FMHA_OK) return st;
+  if ((st = map4(&prm.tmO32, O, cs.o, seq_q, 32, 32)) != FMHA_OK) return st;
   prm.kv_len = (kind == FMHA_MASK_KEY_PADDING) ? mask->kv_len : nullptr;
   prm.cu_seqlens = nullptr;
   prm.seq_q = seq_q;
@@ -299,13 +331,23 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   // odd q-tile counts >= 3 (non-causal): pair tiles across units so no item has an empty second
   // tile (BERT-large-384: +8%).  With a single q-tile per unit (short sequences) every item is one
   // latency-bound step and pairing across units measured slower, so those keep pair_mode 0.
-  prm.pair_mode = (kind != FMHA_MASK_CAUSAL && kind != FMHA_MASK_KEY_BIAS && (prm.num_q_tiles & 1) &&
-                   prm.num_q_tiles >= 3) ? 1 : 0;
+  prm.pair_mode = (kind != FMHA_MASK_CAUSAL && kind != FMHA_MASK_KEY_BIAS && kind != FMHA_MASK_ATTN_BIAS &&
+                   (prm.num_q_tiles & 1) && prm.num_q_tiles >= 3) ? 1 : 0;
   if (kind == FMHA_MASK_KEY_BIAS) {
     prm.key_bias = mask->key_bias;
     prm.key_bias_stride = mask->key_bias_stride;
     prm.inv_scale = 1.4426950408889634f / prm.scale_log2;  // c * inv_scale = log2(e) exactly as used
     prm.mask_kind = FMHA_MASK_NONE;  // no key bound beyond seq_kv; the bias does the masking
+  }
+  if (kind == FMHA_MASK_ATTN_BIAS) {
+    prm.attn_bias = static_cast<const uint16_t*>(mask->attn_bias);
+    prm.ab_sb = mask->attn_bias_stride_b;
+    prm.ab_sh = mask->attn_bias_stride_h;
+    prm.ab_sq = mask->attn_bias_stride_q;
+    const long long row8 = (seq_kv + 7) / 8 * 8;  // a broadcast row (stride 0) must hold row8 elements
+    prm.bias_cols8 = static_cast<int>((mask->attn_bias_stride_q == 0 ? row8 : std::min<long long>(mask->attn_bias_stride_q, row8)) / 8);
+    prm.inv_scale = 1.4426950408889634f / prm.scale_log2;  // c * inv_scale = log2(e) exactly as used
+    prm.mask_kind = FMHA_MASK_NONE;
   }
   long long items = prm.pair_mode ? (units * prm.num_q_tiles + 1) / 2 : units * ((prm.num_q_tiles + 1) / 2);
   prm.single_from = 0x7fffffff;
@@ -377,11 +419,30 @@ int fmha_varlen_common(bool bf16, const void* QKV, void* O, const int32_t* cu_se
   memset(&prm, 0, sizeof(prm));
   const uint64_t hd = static_cast<uint64_t>(heads) * head_dim;
   const uint8_t* base = static_cast<const uint8_t*>(QKV);
-  if ((st = make_map_thd(&prm.tmQ, base, bf16, head_dim, heads, total_tokens, 3 * hd)) != FMHA_OK) return st;
-  if ((st = make_map_thd(&prm.tmK, base + 2 * hd, bf16, head_dim, heads, total_tokens, 3 * hd)) != FMHA_OK) return st;
-  if ((st = make_map_thd(&prm.tmV, base + 4 * hd, bf16, head_dim, heads, total_tokens, 3 * hd)) != FMHA_OK) return st;
-  if ((st = make_map_thd(&prm.tmO, O, bf16, head_dim, heads, total_tokens, hd)) != FMHA_OK) return st;
-  if ((st = make_map_thd(&prm.tmO32, O, bf16, head_dim, heads, total_tokens, hd, 32, 32)) != FMHA_OK) return st;
+  // {D, H, T, 1}: a tile coordinate is (d, h, token, 0); box {64, 1, 128, 1} = one head's 128 tokens
+  auto mapv = [&](CUtensorMap* m, const void* b, uint64_t tok_stride, uint32_t box_tokens, uint32_t box_d) {
+    EncodeTiledFn enc = get_encode_fn();
+    if (!enc) return static_cast<int>(FMHA_ERR_CUDA);
+    cuuint64_t dims[4] = {static_cast<cuuint64_t>(head_dim), static_cast<cuuint64_t>(heads),
+                          static_cast<cuuint64_t>(total_tokens), 1};
+    cuuint64_t strd[3] = {static_cast<cuuint64_t>(head_dim) * 2, tok_stride * 2, tok_stride * 2 * total_tokens};
+    cuuint32_t box[4] = {box_d, 1, box_tokens, 1};
+    cuuint32_t estr[4] = {1, 1, 1, 1};
+    CUresult r = enc(m, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4, const_cast<void*>(b),
+                     dims, strd, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                     box_d == 64 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B,
+                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) {
+      snprintf(g_last_cuda_error, sizeof(g_last_cuda_error), "cuTensorMapEncodeTiled (varlen) failed (%d)", int(r));
+      return static_cast<int>(FMHA_ERR_CUDA);
+    }
+    return static_cast<int>(FMHA_OK);
+  };
+  if ((st = mapv(&prm.tmQ, base, 3 * hd, 128, 64)) != FMHA_OK) return st;
+  if ((st = mapv(&prm.tmK, base + 2 * hd, 3 * hd, 128, 64)) != FMHA_OK) return st;
+  if ((st = mapv(&prm.tmV, base + 4 * hd, 3 * hd, 128, 64)) != FMHA_OK) return st;
+  if ((st = mapv(&prm.tmO, O, hd, 128, 64)) != FMHA_OK) return st;
+  if ((st = mapv(&prm.tmO32, O, hd, 32, 32)) != FMHA_OK) return st;
   prm.kv_len = nullptr;
   prm.cu_seqlens = cu_seqlens;
   prm.o_ptr = static_cast<uint8_t*>(O);
@@ -439,6 +500,23 @@ int fmha_fwd_bf16(const void* Q, const void* K, const void* V, void* O, const fm
                   int heads, int seq_q, int seq_kv, int head_dim, float scale, fmha_stream_t stream) {
   return fmha_common(true, Q, K, V, O, mask, batch, heads, seq_q, seq_kv, head_dim, scale,
                      reinterpret_cast<cudaStream_t>(stream));
+}
+
+int fmha_fwd_strided(int dtype, const void* Q, const void* K, const void* V, void* O, const fmha_strides_t* strides,
+                     const fmha_mask_t* mask, int batch, int heads, int seq_q, int seq_kv, int head_dim, float scale,
+                     fmha_stream_t stream) {
+  g_last_cuda_error[0] = 0;
+  if (dtype != 0 && dtype != 1) return FMHA_ERR_UNSUPPORTED;
+  if (strides) {
+    const int64_t* all[4] = {strides->q, strides->k, strides->v, strides->o};
+    for (const int64_t* st3 : all) {
+      for (int i = 0; i < 3; ++i)
+        if (st3[i] <= 0 || (st3[i] % 8) != 0 || st3[i] > (int64_t(1) << 36)) return FMHA_ERR_INVALID_ARG;
+      if (st3[2] < head_dim) return FMHA_ERR_INVALID_ARG;
+    }
+  }
+  return fmha_common(dtype == 1, Q, K, V, O, mask, batch, heads, seq_q, seq_kv, head_dim, scale,
+                     reinterpret_cast<cudaStream_t>(stream), 1, nullptr, 0, strides);
 }
 
 int fmha_fwd_varlen(const void* QKV, void* O, const int32_t* cu_seqlens, int num_seqs, int max_seqlen,
@@ -501,7 +579,8 @@ int fmha_fwd_from_host(int dtype, const void* hQ, const void* hK, const void* hV
   cudaStream_t stream = reinterpret_cast<cudaStream_t>(stream_);
   if (dtype != 0 && dtype != 1) return FMHA_ERR_UNSUPPORTED;
   // every argument check happens before anything is enqueued (include/fmha.h)
-  if (mask && mask->kind == FMHA_MASK_KEY_BIAS) return FMHA_ERR_UNSUPPORTED;  // (fmha_fwd only)
+  if (mask && (mask->kind == FMHA_MASK_KEY_BIAS || mask->kind == FMHA_MASK_ATTN_BIAS))
+    return FMHA_ERR_UNSUPPORTED;  // (device-pointer masks: fmha_fwd / fmha_fwd_strided only)
   bool empty = false;
   if (int vs = validate_shape(batch, heads, seq_q, seq_kv, head_dim, scale, mask, 1, &empty); vs != FMHA_OK || empty)
     return vs;

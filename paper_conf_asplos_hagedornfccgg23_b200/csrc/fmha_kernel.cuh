@@ -96,8 +96,8 @@ constexpr int SCHED_MAX_LEVELS = 64, SCHED_MAX_SEQS = 1024;
 #endif
 
 struct FmhaParams {
-  CUtensorMap tmQ;  // 3-D {D, seq_q, B*H}, box {64, 128, 1}, SWIZZLE_128B
-  CUtensorMap tmK;  // 3-D {D, seq_kv, B*H}
+  CUtensorMap tmQ;  // 4-D {D, seq_q, H, B} (any row / head / batch strides), box {64, 128, 1, 1}, SWIZZLE_128B
+  CUtensorMap tmK;  // 4-D {D, seq_kv, H, B}; varlen maps: {D, H, T, 1}, box {64, 1, 128, 1}
   CUtensorMap tmV;
   CUtensorMap tmO;  // same geometry as Q
   CUtensorMap tmO32;  // O with a 32-row box (key-split kernel: one store per (tile, lane quarter))
@@ -139,6 +139,12 @@ struct FmhaParams {
   const float* key_bias;
   int key_bias_stride;
   float inv_scale;
+  // General additive (query x key) mask (MODE_BIAS2D; R21): raw scores get
+  // attn_bias[b, h, i, j] / scale added (16-bit, the I/O type), element strides below (0 broadcasts);
+  // bias_cols8 = min(row stride, seq_kv rounded up to 8) / 8 bounds the 16-byte loads of a row.
+  const uint16_t* attn_bias;
+  long long ab_sb, ab_sh, ab_sq;
+  int bias_cols8;
 };
 
 template <int D>
@@ -313,12 +319,15 @@ struct WorkItem {
   bool has1;     // tile 1 exists
   int tok0, tok1;  // varlen: first token of the sequence of tile 0 / 1; len = its length
   int len0, len1;
-  int head, head1;  // varlen: h of unit bh0 / bh1
+  int head, head1;  // h of unit bh0 / bh1
+  int bat0, bat1;   // dense: b of unit bh0 / bh1
   int jb;          // split-KV: first KV tile of this item's range (0 otherwise)
   int split;       // split-KV: split index
-  // TMA coordinates (c1, c2) of the 128-row block starting at row r of tile t (c0 = d)
+  // 4-D TMA coordinates (c1, c2, c3) of the block starting at row r of tile t (c0 = d):
+  // dense maps are {D, rows, heads, batch}, varlen maps {D, heads, tokens, 1}
   __device__ __forceinline__ int c1(bool varlen, int t, int r) const { return varlen ? (t ? head1 : head) : r; }
-  __device__ __forceinline__ int c2(bool varlen, int t, int r) const { return varlen ? tok(t) + r : bh(t); }
+  __device__ __forceinline__ int c2(bool varlen, int t, int r) const { return varlen ? tok(t) + r : (t ? head1 : head); }
+  __device__ __forceinline__ int c3(bool varlen, int t) const { return varlen ? 0 : (t ? bat1 : bat0); }
   bool shared;
   __device__ __forceinline__ int n(int t) const { return t ? n1 : n0; }
   __device__ __forceinline__ int bh(int t) const { return t ? bh1 : bh0; }
@@ -380,7 +389,10 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
   w.has0 = true;
   w.kv0 = w.kv1 = p.seq_kv;
   w.tok0 = w.tok1 = 0;
-  w.head = w.head1 = 0;
+  w.bat0 = p.div_heads.div(w.bh0);
+  w.bat1 = w.shared ? w.bat0 : p.div_heads.div(w.bh1);
+  w.head = w.bh0 - w.bat0 * p.heads;
+  w.head1 = w.bh1 - w.bat1 * p.heads;
   w.len0 = w.len1 = p.seq_q;
   if constexpr (VL) {  // varlen (pair_mode 0): both tiles belong to unit bh0 = b * H + h
     const int b = p.div_heads.div(w.bh0);
@@ -393,7 +405,7 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
     w.has1 = w.has1 && w.r1 < w.len0;
   }
   if (p.mask_kind == MASK_KEY_PADDING) {
-    w.kv0 = min(max(__ldg(p.kv_len + p.div_heads.div(w.bh0)), 0), p.seq_kv);
+    w.kv0 = min(max(__ldg(p.kv_len + w.bat0), 0), p.seq_kv);
     w.kv1 = w.shared ? w.kv0
                      : min(max(__ldg(p.kv_len + p.div_heads.div(min(w.bh1, p.num_units - 1))), 0), p.seq_kv);
   }
@@ -534,6 +546,7 @@ __device__ __forceinline__ WorkItem sched_item(const FmhaParams& p, const SchedT
   w.len1 = __ldg(p.cu_seqlens + sq1 + 1) - w.tok1;
   w.head = h0;
   w.head1 = h1;
+  w.bat0 = w.bat1 = 0;
   w.bh0 = sq0 * H + h0;
   w.bh1 = sq1 * H + h1;
   w.kv0 = w.len0;
@@ -556,14 +569,17 @@ __device__ __forceinline__ WorkItem get_item(const FmhaParams& p, const SchedTab
 // Kernel instances (MODE): dense [B,H,S,D]; dense with cross-unit tile pairing (pair_mode 1, see
 // FmhaParams::pair_mode); varlen packed; varlen packed with the cost-sorted schedule.  Separate
 // instances keep the varlen and scheduling code out of the dense kernels entirely.
-enum : int { MODE_DENSE = 0, MODE_PAIRX = 1, MODE_VARLEN = 2, MODE_VARLEN_SCHED = 3, MODE_SPLIT = 4, MODE_BIAS = 5 };
+enum : int { MODE_DENSE = 0, MODE_PAIRX = 1, MODE_VARLEN = 2, MODE_VARLEN_SCHED = 3, MODE_SPLIT = 4, MODE_BIAS = 5,
+             MODE_BIAS2D = 6 };
 
 template <int D, bool BF16, int MODE>
 __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
   using C = FmhaCfg<D>;
-  using XS = ExpShape<D, MODE == MODE_PAIRX, MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED, MODE == MODE_BIAS>;
+  using XS = ExpShape<D, MODE == MODE_PAIRX, MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
+                      MODE == MODE_BIAS || MODE == MODE_BIAS2D>;
   constexpr bool PAIRX = MODE == MODE_PAIRX, VL = MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
-                 SCHED = MODE == MODE_VARLEN_SCHED, SPLIT = MODE == MODE_SPLIT, BIAS = MODE == MODE_BIAS;
+                 SCHED = MODE == MODE_VARLEN_SCHED, SPLIT = MODE == MODE_SPLIT, BIAS = MODE == MODE_BIAS,
+                 BIAS2D = MODE == MODE_BIAS2D;
   // Dynamic shared memory starts at the (1024-byte aligned) base of the CTA's shared window; the
   // SWIZZLE_128B tiles need that alignment.  Using the base directly keeps smem addresses uniform.
   extern __shared__ __align__(1024) uint8_t smem[];
@@ -649,8 +665,8 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           const CUtensorMap* map = m ? &p.tmV : &p.tmK;
 #pragma unroll
           for (int c = 0; c < D / 64; ++c)
-            tma_load_3d_hint_elect(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64,
-                                   w.c1(vl, t, (w.jb + j) * 128), w.c2(vl, t, (w.jb + j) * 128), keep);
+            tma_load_4d_hint_elect(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64,
+                                   w.c1(vl, t, (w.jb + j) * 128), w.c2(vl, t, (w.jb + j) * 128), w.c3(vl, t), keep);
         }
       };
       for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
@@ -665,8 +681,8 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           mbar_arrive_expect_tx_elect(Q_FULL(t, qs), C::TILE);
 #pragma unroll
           for (int c = 0; c < D / 64; ++c)
-            tma_load_3d_hint_elect(sbase + C::OFF_Q + (2 * qs + t) * C::TILE + c * C::CHUNK, &p.tmQ, Q_FULL(t, qs),
-                                   c * 64, w.c1(vl, t, w.row0(t)), w.c2(vl, t, w.row0(t)), once);
+            tma_load_4d_hint_elect(sbase + C::OFF_Q + (2 * qs + t) * C::TILE + c * C::CHUNK, &p.tmQ, Q_FULL(t, qs),
+                                   c * 64, w.c1(vl, t, w.row0(t)), w.c2(vl, t, w.row0(t)), w.c3(vl, t), once);
           ++qc;
           TRACE_EV(EV_ITEM, 4 + t);
         }
@@ -987,6 +1003,37 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             }
           }
         }
+        if constexpr (BIAS2D) {  // s' = s + attn_bias[b, h, qi, key] / scale (R21): this row's 128 keys as
+                                 // 16 x 16-byte loads (clamped to the row; keys >= seq_kv are masked below)
+          const int bb = t ? w.bat1 : w.bat0, hh = t ? w.head1 : w.head;
+          const uint4* brow = reinterpret_cast<const uint4*>(
+              p.attn_bias + bb * p.ab_sb + hh * p.ab_sh + static_cast<long long>(min(qi, p.seq_q - 1)) * p.ab_sq);
+          const int c80 = (w.jb + j) * 16;  // first 8-key group of this step
+          const float2 is2 = make_float2(p.inv_scale, p.inv_scale);
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            uint4 bq[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) bq[u] = __ldg(brow + min(c80 + 4 * q + u, p.bias_cols8 - 1));
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+              const uint32_t hw[4] = {bq[u].x, bq[u].y, bq[u].z, bq[u].w};
+#pragma unroll
+              for (int e = 0; e < 4; ++e) {
+                const int k = 32 * q + 8 * u + 2 * e;
+                float2 bf;
+                if constexpr (BF16) {
+                  bf = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&hw[e]));
+                } else {
+                  bf = __half22float2(*reinterpret_cast<const __half2*>(&hw[e]));
+                }
+                const float2 r = ffma2(bf, is2, make_float2(__uint_as_float(s[k]), __uint_as_float(s[k + 1])));
+                s[k] = __float_as_uint(r.x);
+                s[k + 1] = __float_as_uint(r.y);
+              }
+            }
+          }
+        }
         if (rem < 128) {  // boundary tile for this row (a5)
 #pragma unroll
           for (int k = 0; k < 128; ++k)
@@ -1260,7 +1307,8 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             constexpr bool vl = VL;
 #pragma unroll
             for (int c2 = 0; c2 < D / 64; ++c2)
-              tma_store_3d(&p.tmO, stg + c2 * C::CHUNK, c2 * 64, w.c1(vl, t, w.row0(t)), w.c2(vl, t, w.row0(t)));
+              tma_store_4d(&p.tmO, stg + c2 * C::CHUNK, c2 * 64, w.c1(vl, t, w.row0(t)), w.c2(vl, t, w.row0(t)),
+                           w.c3(vl, t));
             tma_store_commit();
           }
         }

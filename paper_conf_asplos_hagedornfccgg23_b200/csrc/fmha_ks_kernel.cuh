@@ -187,8 +187,8 @@ __global__ void __launch_bounds__(640, 1) fmha_fwd_ks_sm100(const __grid_constan
           mbar_wait_at(KV_EMPTY(s), ((kv / C::NS) & 1) ^ 1, 1, kv, j);
           TRACE_EV(EV_TMA_KV, m * 64 + j);
           mbar_arrive_expect_tx_elect(KV_FULL(s), C::TILE);
-          tma_load_3d_hint_elect(sbase + C::OFF_RING + s * C::TILE, m ? &p.tmV : &p.tmK, KV_FULL(s), 0,
-                                 w.c1(VL, t, j * 128), w.c2(VL, t, j * 128), keep);
+          tma_load_4d_hint_elect(sbase + C::OFF_RING + s * C::TILE, m ? &p.tmV : &p.tmK, KV_FULL(s), 0,
+                                 w.c1(VL, t, j * 128), w.c2(VL, t, j * 128), w.c3(VL, t), keep);
         }
       };
       for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
@@ -201,8 +201,8 @@ __global__ void __launch_bounds__(640, 1) fmha_fwd_ks_sm100(const __grid_constan
           const int qs = qc % C::QS;
           mbar_wait_at(Q_EMPTY(t, qs), ((qc / C::QS) & 1) ^ 1, 2, qc, t);
           mbar_arrive_expect_tx_elect(Q_FULL(t, qs), C::TILE);
-          tma_load_3d_hint_elect(sbase + C::OFF_Q + (2 * qs + t) * C::TILE, &p.tmQ, Q_FULL(t, qs), 0,
-                                 w.c1(VL, t, w.row0(t)), w.c2(VL, t, w.row0(t)), once);
+          tma_load_4d_hint_elect(sbase + C::OFF_Q + (2 * qs + t) * C::TILE, &p.tmQ, Q_FULL(t, qs), 0,
+                                 w.c1(VL, t, w.row0(t)), w.c2(VL, t, w.row0(t)), w.c3(VL, t), once);
           ++qc;
         }
         for (int j = 0; j < N; ++j) {
@@ -526,7 +526,8 @@ __global__ void __launch_bounds__(640, 1) fmha_fwd_ks_sm100(const __grid_constan
         fence_proxy_async_smem();
         __syncwarp();
         if (lane == 0) {
-          tma_store_3d(&p.tmO32, stg, 32 * h, w.c1(VL, t, w.row0(t) + 32 * quad), w.c2(VL, t, w.row0(t) + 32 * quad));
+          tma_store_4d(&p.tmO32, stg, 32 * h, w.c1(VL, t, w.row0(t) + 32 * quad), w.c2(VL, t, w.row0(t) + 32 * quad),
+                       w.c3(VL, t));
           tma_store_commit();
         }
       } else if (qi < w.len(t)) {  // varlen tile crossing the sequence's end: rows inside only
