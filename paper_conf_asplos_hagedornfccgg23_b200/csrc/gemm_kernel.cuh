@@ -107,6 +107,28 @@ __device__ __forceinline__ float gelu_erf_fast(float x) {
   return x * (x < 0.f ? q : 1.f - q);
 }
 
+// The same GELU_erf on a pair with packed fp32x2 arithmetic (FFMA2 / FMUL2 / FADD2: two elements per
+// FMA-pipe instruction, half the issue slots of the scalar form -- the GELU GEMM's epilogue was
+// issue-bound).  The 0.5 of q is folded into the polynomial's coefficients (exact:
+// powers of two).  Identical formula, so identical error bound.
+__device__ __forceinline__ float2 gelu_erf_fast2(float2 x) {
+  const float2 z = make_float2(fabsf(x.x) * 0.70710678118654752f, fabsf(x.y) * 0.70710678118654752f);
+  const float2 d = ffma2(z, 0.3275911f, 1.f);
+  float2 t;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(t.x) : "f"(d.x));
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(t.y) : "f"(d.y));
+  float2 poly = ffma2(t, make_float2(0.5f * 1.061405429f, 0.5f * 1.061405429f),
+                      make_float2(0.5f * -1.453152027f, 0.5f * -1.453152027f));
+  poly = ffma2(t, poly, make_float2(0.5f * 1.421413741f, 0.5f * 1.421413741f));
+  poly = ffma2(t, poly, make_float2(0.5f * -0.284496736f, 0.5f * -0.284496736f));
+  poly = ffma2(t, poly, make_float2(0.5f * 0.254829592f, 0.5f * 0.254829592f));
+  poly = fmul2(poly, t);
+  const float2 arg = fmul2(fmul2(z, z), make_float2(-1.4426950408889634f, -1.4426950408889634f));
+  const float2 q = fmul2(poly, make_float2(ex2(arg.x), ex2(arg.y)));
+  const float2 omq = fadd2(make_float2(1.f, 1.f), make_float2(-q.x, -q.y));
+  return fmul2(x, make_float2(x.x < 0.f ? q.x : omq.x, x.y < 0.f ? q.y : omq.y));
+}
+
 template <int ACT>
 __device__ __forceinline__ float apply_act(float x) {
   if (ACT == 1) return fmaxf(x, 0.f);
@@ -115,6 +137,27 @@ __device__ __forceinline__ float apply_act(float x) {
   if (ACT == 4) return tanhf(x);
   return x;
 }
+
+// act on the 32 accumulator columns of a chunk: f = act(v + bias), packed pairs for GELU_erf
+#ifndef GEMM_GELU_PACKED
+#define GEMM_GELU_PACKED 1
+#endif
+template <int ACT>
+__device__ __forceinline__ void act_chunk(const uint32_t (&v)[32], const float (&bv)[32], float (&f)[32]) {
+  if constexpr (ACT == 2 && GEMM_GELU_PACKED) {
+#pragma unroll
+    for (int k = 0; k < 32; k += 2) {
+      const float2 y = gelu_erf_fast2(fadd2(make_float2(__uint_as_float(v[k]), __uint_as_float(v[k + 1])),
+                                           make_float2(bv[k], bv[k + 1])));
+      f[k] = y.x;
+      f[k + 1] = y.y;
+    }
+  } else {
+#pragma unroll
+    for (int k = 0; k < 32; ++k) f[k] = apply_act<ACT>(__uint_as_float(v[k]) + bv[k]);
+  }
+}
+
 
 template <int ACT>
 __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_constant__ GemmParams p) {
@@ -220,12 +263,23 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
       if (row == 0) tma_store_wait_read0();  // this half's staging boxes are free again
       named_bar_sync(bar_id, 128);
       const uint32_t tacc = tmem + lane_off + 256 * b + 128 * g;
-#pragma unroll 1
-      for (int q = 0; q < (active ? 4 : 0); ++q) {
-        uint32_t v[32];
-        tmem_ld_32x32b_x32(tacc + 32 * q, v);
+      // The four 32-column chunks are software-pipelined: chunk q+1's TMEM load is in flight while
+      // chunk q is computed, and the accumulator is released as soon as the last chunk is in
+      // registers (before its bias/activation/store), so the MMA can start the tile after next.
+      uint32_t va[32], vb[32];
+      if (active) tmem_ld_32x32b_x32(tacc, va);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        if (!active) break;
+        uint32_t(&v)[32] = (q & 1) ? vb : va;
         tmem_wait_ld();
         reg_fence(v);
+        if (q + 1 < 4) {
+          tmem_ld_32x32b_x32(tacc + 32 * (q + 1), (q & 1) ? va : vb);
+        } else {  // accumulator b fully read: the MMA warp may start the tile after next into it
+          tc_fence_before();
+          mbar_arrive(ACC_EMPTY(b));
+        }
         const int col0 = 128 * g + 32 * q;  // column within the tile
         // bias for these 32 columns: four 16-byte loads (N % 8 == 0, so a group is all in or all out)
         float bv[32];
@@ -243,8 +297,7 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
           }
         }
         float f[32];
-#pragma unroll
-        for (int k = 0; k < 32; ++k) f[k] = apply_act<ACT>(__uint_as_float(v[k]) + bv[k]);
+        act_chunk<ACT>(v, bv, f);
         const uint32_t box = sbase + C::OFF_STG + (col0 / 64) * C::C_BOX + row * 128;
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
@@ -254,9 +307,10 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
                        pack2<false>(f[8 * u + 6], f[8 * u + 7]));
         }
       }
-      // accumulator b fully read: the MMA warp may start the tile after next into it
-      tc_fence_before();
-      mbar_arrive(ACC_EMPTY(b));
+      if (!active) {  // (nothing read: release the accumulator at once)
+        tc_fence_before();
+        mbar_arrive(ACC_EMPTY(b));
+      }
       fence_proxy_async_smem();
       named_bar_sync(bar_id, 128);
       if (row == 0 && active) {
@@ -414,12 +468,22 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
       if (row == 0) tma_store_wait_read0();
       named_bar_sync(bar_id, 128);
       const uint32_t tacc = tmem + lane_off + 256 * b + 128 * g;
-#pragma unroll 1
-      for (int q = 0; q < (active ? 4 : 0); ++q) {
-        uint32_t v[32];
-        tmem_ld_32x32b_x32(tacc + 32 * q, v);
+      // software-pipelined chunks and early accumulator release, as in gemm_bias_act_kernel
+      uint32_t va[32], vb[32];
+      if (active) tmem_ld_32x32b_x32(tacc, va);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        if (!active) break;
+        uint32_t(&v)[32] = (q & 1) ? vb : va;
         tmem_wait_ld();
         reg_fence(v);
+        if (q + 1 < 4) {
+          tmem_ld_32x32b_x32(tacc + 32 * (q + 1), (q & 1) ? va : vb);
+        } else {  // this warp's accumulator reads are done: one arrival per warp on the leader's ACC_EMPTY
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive_cluster(mapa_shared(ACC_EMPTY(b), 0));
+        }
         const int col0 = 128 * g + 32 * q;
         float bv[32];
 #pragma unroll
@@ -436,8 +500,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
           }
         }
         float f[32];
-#pragma unroll
-        for (int k = 0; k < 32; ++k) f[k] = apply_act<ACT>(__uint_as_float(v[k]) + bv[k]);
+        act_chunk<ACT>(v, bv, f);
         const uint32_t box = sbase + C::OFF_STG + (col0 / 64) * C::C_BOX + row * 128;
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
@@ -447,10 +510,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
                        pack2<false>(f[8 * u + 6], f[8 * u + 7]));
         }
       }
-      // this warp's accumulator reads are done: one arrival per warp on the leader's ACC_EMPTY
-      tc_fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive_cluster(mapa_shared(ACC_EMPTY(b), 0));
+      if (!active) {  // (nothing read: release at once)
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive_cluster(mapa_shared(ACC_EMPTY(b), 0));
+      }
       fence_proxy_async_smem();
       named_bar_sync(bar_id, 128);
       if (row == 0 && active) {
