@@ -766,7 +766,7 @@ const char* fmha_status_string(int status) {
 
 const char* fmha_last_cuda_error(void) { return g_last_cuda_error; }
 
-#if FMHA_TRACE
+#if FMHA_TRACE || FMHA_PROF
 // Debug-build only (not part of include/fmha.h): point the timeline recorder at a device buffer
 // of 65536 uint64 records and reset its counter; fmha_trace_count() returns the record count.
 FMHA_API int fmha_trace_set(void* dev_buf) {

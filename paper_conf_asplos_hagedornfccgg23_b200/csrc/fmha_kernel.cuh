@@ -43,9 +43,14 @@
 
 namespace b200 {
 
-#if FMHA_TRACE
+#ifndef FMHA_PROF
+#define FMHA_PROF 0
+#endif
+#if FMHA_TRACE || FMHA_PROF
 __device__ unsigned long long* g_fmha_trace = nullptr;
 __device__ unsigned int g_fmha_trace_n = 0;
+#endif
+#if FMHA_TRACE
 #define TRACE_EV(ev, aux)                                                                                \
   do {                                                                                                   \
     if (blockIdx.x == 0 && (threadIdx.x & 31) == 0 && trace_buf && trace_i < 2048u) {                    \
@@ -63,6 +68,51 @@ __device__ unsigned int g_fmha_trace_n = 0;
   do {                    \
   } while (0)
 #define TRACE_DECL
+#endif
+// Timing-only ablations (WRONG RESULTS; never in the product build): FMHA_ABL bit 0 skips the S TMEM
+// load (registers zeroed), bit 1 the row max (fixed reference), bit 2 the P TMEM stores, bit 3 the
+// tensor-core instructions (commits still arrive), bit 4 the exponential phase (its turn kept), bit 5 the
+// epilogue's O TMEM loads, bit 6 makes every K/V load read the same (L2-resident) tile.  Used to locate what bounds a step.
+#ifndef FMHA_ABL
+#define FMHA_ABL 0
+#endif
+// FMHA_ELECT: the per-row hand-offs (S_FREE, P_FULL, L_FULL, L_EMPTY, O_EMPTY) arrive once per warp
+// (elect.sync, barrier count 4) instead of once per thread (count 128): 32x fewer mbarrier updates.
+#ifndef FMHA_ELECT
+#define FMHA_ELECT 0
+#endif
+#if FMHA_ELECT
+#define FMHA_ROW_ARRIVE(bar) mbar_arrive_elect(bar)
+#define FMHA_ROW_COUNT 4
+#else
+#define FMHA_ROW_ARRIVE(bar) mbar_arrive(bar)
+#define FMHA_ROW_COUNT 128
+#endif
+// Phase profile (build with -DFMHA_PROF=1; not the product build): every softmax thread accumulates
+// the cycles between consecutive marks into per-phase counters (two clock reads per mark, no memory
+// traffic until the end), and lane 0 of each softmax warp writes them to g_fmha_trace[block][warp][16].
+#ifndef FMHA_PROF
+#define FMHA_PROF 0
+#endif
+#if FMHA_PROF
+#define PROF_DECL                     \
+  uint32_t prof_acc[16] = {};         \
+  uint32_t prof_t = clock();
+#define PROF_MARK(k)                  \
+  do {                                \
+    const uint32_t prof_now = clock(); \
+    prof_acc[k] += prof_now - prof_t; \
+    prof_t = prof_now;                \
+  } while (0)
+#define PROF_COUNT(k) (++prof_acc[k])
+#else
+#define PROF_DECL
+#define PROF_MARK(k) \
+  do {               \
+  } while (0)
+#define PROF_COUNT(k) \
+  do {                \
+  } while (0)
 #endif
 enum : int { EV_S_WAIT = 1, EV_S_READY, EV_MAX_DONE, EV_XCHG, EV_EXP_DONE, EV_MMA_P, EV_MMA_O, EV_MMA_PV,
              EV_MMA_QK, EV_COR_ST, EV_COR_PV, EV_COR_ORDY, EV_EPI, EV_TMA_KV, EV_ITEM };
@@ -153,7 +203,10 @@ struct FmhaCfg {
   static constexpr int BN = 128;                // keys per KV tile
   static constexpr int CHUNK = 128 * 64 * 2;    // one SW128 TMA box: 128 rows x 64 16-bit elements
   static constexpr int TILE = BM * D * 2;       // bytes of one Q / K / V / O tile
-  static constexpr int NS = (D == 64) ? 6 : 3;  // K/V ring slots (K_j, V_j alternate)
+#ifndef FMHA_NS64
+#define FMHA_NS64 6
+#endif
+  static constexpr int NS = (D == 64) ? FMHA_NS64 : 3;  // K/V ring slots (K_j, V_j alternate)
   static constexpr int QS = (D == 64) ? 2 : 1;  // Q stages per tile: the next item's Q loads early
   static constexpr int NSTG = (D == 64) ? 2 : 1;  // O staging buffers (D=128: both tiles share one)
   static constexpr int OFF_Q = 0;               // Q[stage][tile]
@@ -177,7 +230,11 @@ struct FmhaCfg {
     B_S_FULL = 0, B_P_FULL = 2, B_O_FULL = 4, B_PV_DONE = 6, B_O_EMPTY = 8, B_L_FULL = 12,
     B_S_FREE = 14, B_Q_FULL = 16, B_Q_EMPTY = 20, B_L_EMPTY = 24, B_KV = 26
   };
-  static constexpr int NUM_BARS = B_KV + 2 * NS;
+  // B_P_FULL2 [tile]: P_FULL of odd steps (ROT).  Without the per-step PV_DONE wait the softmax can
+  // be two P hand-offs ahead of the MMA warp (S_FULL_g only implies PV_{g-2} was issued), which one
+  // barrier's phase parity cannot tell apart; two barriers by step parity can.
+  static constexpr int B_P_FULL2 = B_KV + 2 * NS;
+  static constexpr int NUM_BARS = B_P_FULL2 + 2;
   static constexpr int OFF_TMEMPTR = OFF_BAR + NUM_BARS * 8;
   static constexpr int OFF_SCHED = OFF_TMEMPTR + 16;  // SchedTable (sched mode 1 only)
   static constexpr int SMEM_ALLOC = OFF_SCHED + 4 * (3 * (SCHED_MAX_LEVELS + 2) + SCHED_MAX_SEQS);
@@ -186,6 +243,24 @@ struct FmhaCfg {
   static constexpr int W_CORR = 8, W_MMA = 12, W_TMA = 14;  // first warp of each role
   static constexpr bool SEP_P = (D == 64) && !LSUM_MMA;
   static constexpr int TMEM_P = 384;
+  // ROT (D = 64, separate P): tile t owns columns [256 t, 256 t + 256): O_t at +192 and three 64-column
+  // regions below it over which S and P rotate with the tile's step count g -- S_g in [0,128) (g even)
+  // or [64,192) (g odd), P_g in [0,64) or [128,192).  S_{g+1} never covers P_g (PV_g is issued after
+  // QK_{g+1}), P_g never covers P_{g-1} (PV_{g-1} may still be reading it), and S_{g+1} covering
+  // P_{g-1} is safe (PV_{g-1} is issued before QK_{g+1} by the same thread, and tcgen05.mma ops of one
+  // thread execute in order); P_g lies on S_g, which this warp has loaded.  So the softmax writes P_g
+  // without waiting for PV_{g-1} (PV_DONE is waited only before a lazy rescale of O).
+#ifndef FMHA_ROT
+#define FMHA_ROT 1
+#endif
+  static constexpr bool ROT = FMHA_ROT && SEP_P;
+  static __host__ __device__ constexpr uint32_t col_s(int t, uint32_t g) {
+    return ROT ? 256 * t + ((g & 1) ? 64 : 0) : 128 * t;
+  }
+  static __host__ __device__ constexpr uint32_t col_p(int t, uint32_t g) {
+    return ROT ? 256 * t + ((g & 1) ? 128 : 0) : (SEP_P ? TMEM_P + 64 * t : 128 * t);
+  }
+  static __host__ __device__ constexpr uint32_t col_o(int t) { return ROT ? 256 * t + 192 : 256 + t * OW; }
   // registers after setmaxnreg.  setmaxnreg.inc only draws on the CTA's launch allocation
   // (128 x 512 = 65536), so 8 x 32 x 192 + 4 x 32 x 56 + 4 x 32 x 72 = 65536 must not be exceeded
   // (56 / 72: the MMA and TMA warps spill at 48, and those spills cost 2-12%).
@@ -211,7 +286,7 @@ struct FmhaCfg {
 #ifndef FMHA_PREFETCH_S
 #define FMHA_PREFETCH_S 0
 #endif
-  static constexpr bool PREFETCH_S = FMHA_PREFETCH_S && SEP_P && !SPLIT_LD;
+  static constexpr bool PREFETCH_S = FMHA_PREFETCH_S && SEP_P && !SPLIT_LD && !FMHA_ROT;
   // Key bias: prefetch all four 128-B lines of this and the next step's bias into L1 (A/B knob;
   // measured -2% at BERT-large-384, +2% at 512: L1 misses are not the bias cost, left off)
 #ifndef FMHA_BIAS_PF4
@@ -601,13 +676,14 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     if (sbase & 1023u) __trap();  // the layout below assumes a 1024-byte aligned window
     for (int t = 0; t < 2; ++t) {
       mbar_init(BAR(C::B_S_FULL + t), 1);
-      mbar_init(BAR(C::B_P_FULL + t), 128);   // softmax threads of tile t (one per row)
+      mbar_init(BAR(C::B_P_FULL + t), FMHA_ROW_COUNT);   // softmax warps (threads) of tile t
+      mbar_init(BAR(C::B_P_FULL2 + t), FMHA_ROW_COUNT);
       mbar_init(BAR(C::B_O_FULL + t), 1);     // last PV of the tile committed
-      mbar_init(BAR(C::B_O_EMPTY + t), 128);  // epilogue threads have read O_t
+      mbar_init(BAR(C::B_O_EMPTY + t), FMHA_ROW_COUNT);  // epilogue warps (threads) have read O_t
       mbar_init(BAR(C::B_PV_DONE + t), 1);
-      mbar_init(BAR(C::B_L_FULL + t), 128);
-      mbar_init(BAR(C::B_L_EMPTY + t), 128);  // epilogue threads, after reading the row sums
-      mbar_init(BAR(C::B_S_FREE + t), 128);
+      mbar_init(BAR(C::B_L_FULL + t), FMHA_ROW_COUNT);
+      mbar_init(BAR(C::B_L_EMPTY + t), FMHA_ROW_COUNT);  // epilogue, after reading the row sums
+      mbar_init(BAR(C::B_S_FREE + t), FMHA_ROW_COUNT);
       for (int q = 0; q < 2; ++q) {
         mbar_init(Q_FULL(t, q), 1);
         mbar_init(Q_EMPTY(t, q), 1);
@@ -665,8 +741,12 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           const CUtensorMap* map = m ? &p.tmV : &p.tmK;
 #pragma unroll
           for (int c = 0; c < D / 64; ++c)
-            tma_load_4d_hint_elect(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64,
-                                   w.c1(vl, t, (w.jb + j) * 128), w.c2(vl, t, (w.jb + j) * 128), w.c3(vl, t), keep);
+            if (FMHA_ABL & 64)  // (timing ablation: every K/V load hits the same L2-resident tile)
+              tma_load_4d_hint_elect(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64, 0, 0, 0,
+                                     keep);
+            else
+              tma_load_4d_hint_elect(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64,
+                                     w.c1(vl, t, (w.jb + j) * 128), w.c2(vl, t, (w.jb + j) * 128), w.c3(vl, t), keep);
         }
       };
       for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
@@ -705,13 +785,12 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       // descriptors differ only in the start-address field: one base, plus (offset >> 4)
       const uint64_t desc0 = sdesc_sw128(sbase, 16, 1024);         // K-major Q / K tiles
       const uint64_t vdesc0 = sdesc_sw128(sbase, C::CHUNK, 1024);  // MN-major V tiles
-      const uint32_t tS = tmem + 128 * t;
-      const uint32_t tO = tmem + 256 + t * C::OW;
-      const uint32_t tP = tmem + (C::SEP_P ? C::TMEM_P + 64 * t : 128 * t);
-      const uint32_t S_FULL = BAR(C::B_S_FULL + t), P_FULL = BAR(C::B_P_FULL + t);
+      const uint32_t tO = tmem + C::col_o(t);
+      const uint32_t S_FULL = BAR(C::B_S_FULL + t), P_FULL = BAR(C::B_P_FULL + t), P_FULL2 = BAR(C::B_P_FULL2 + t);
       const uint32_t O_FULL = BAR(C::B_O_FULL + t), O_EMPTY = BAR(C::B_O_EMPTY + t);
       const uint32_t PV_DONE = BAR(C::B_PV_DONE + t), S_FREE = BAR(C::B_S_FREE + t);
       uint32_t qc = 0, pc = 0, oc = 0, qkc = 0;
+      PROF_DECL
       auto ring_wait = [&](uint32_t k) {
         mbar_wait_at(KV_FULL(k % C::NS), (k / C::NS) & 1, 3, k, 0);
         tc_fence_after();
@@ -770,39 +849,53 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       // S_t <- Q_t K_{t,j}^T (separate P: once the softmax warps have read the previous S_t)
       auto qk_entry = [&](Cursor& cu, uint32_t kidx) {
         const int n = cu.w.n(t);
+        PROF_MARK(8);  // (between MMA phases)
         const uint32_t sK = ring_wait(kidx);
+        PROF_MARK(0);  // K ring wait
         if (cu.j == 0) {  // first QK of this item's tile t: its Q tile must have landed
           cu.qs = qc % C::QS;
           mbar_wait_at(Q_FULL(t, cu.qs), (qc / C::QS) & 1, 4, qc, cu.idx);
           ++qc;
         }
+        PROF_MARK(1);  // Q wait
         if (C::SEP_P && qkc > 0) {
           mbar_wait_at(S_FREE, (qkc - 1) & 1, 5, qkc, cu.idx);
           tc_fence_after();
         }
+        PROF_MARK(2);  // S_FREE wait
+        const uint32_t tS = tmem + C::col_s(t, qkc);
         ++qkc;
         const uint32_t qoff = C::OFF_Q + (2 * cu.qs + t) * C::TILE;
         const uint32_t koff = sK - sbase;
 #pragma unroll
         for (int kk = 0; kk < D / 16; ++kk) {
           const uint32_t off = (kk / 4) * C::CHUNK + (kk % 4) * 32;
-          umma_ss_elect(tS, desc0 + ((qoff + off) >> 4), desc0 + ((koff + off) >> 4), IDESC_QK, kk > 0);
+          if (!(FMHA_ABL & 8)) umma_ss_elect(tS, desc0 + ((qoff + off) >> 4), desc0 + ((koff + off) >> 4), IDESC_QK, kk > 0);
         }
         umma_commit_elect(S_FULL);
         TRACE_EV(EV_MMA_QK, t * 64 + cu.j);
         if (cu.j + 1 == n) umma_commit_elect(Q_EMPTY(t, cu.qs));  // last QK of the tile: Q slot reusable
         umma_commit_elect(KV_EMPTY(kidx % C::NS));
+        PROF_MARK(3);  // QK issue
       };
       // O_t (+)= P_t V_{t,j} once the softmax wrote P_t (and rescaled its rows of O_t if needed);
       // the first PV of an item overwrites O_t, so it also waits until the epilogue has read O_t
       auto pv_entry = [&](Cursor& cu, uint32_t vidx) {
+        PROF_MARK(8);
         const uint32_t sV = ring_wait(vidx);
+        PROF_MARK(4);  // V ring wait
         if (cu.j == 0) {
           mbar_wait_at(O_EMPTY, (oc & 1) ^ 1, 7, oc, cu.idx);
           ++oc;
         }
-        mbar_wait_at(P_FULL, pc & 1, 6, pc, cu.idx);
+        PROF_MARK(5);  // O_EMPTY wait
+        if (C::ROT)
+          mbar_wait_at((pc & 1) ? P_FULL2 : P_FULL, (pc >> 1) & 1, 6, pc, cu.idx);
+        else
+          mbar_wait_at(P_FULL, pc & 1, 6, pc, cu.idx);
+        const uint32_t tP = tmem + C::col_p(t, pc);
         ++pc;
+        PROF_MARK(6);  // P_FULL wait
         TRACE_EV(EV_MMA_P, t * 64 + cu.j);
         tc_fence_after();
         // LSUM_MMA: the second 64-column N chunk of B (columns 64..79 used) is the ones atom, one
@@ -810,11 +903,12 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         const uint64_t vdesc = C::LSUM_MMA ? sdesc_sw128(sbase, C::OFF_ONES - (sV - sbase), 1024) : vdesc0;
 #pragma unroll
         for (int kk = 0; kk < 8; ++kk)
-          umma_ts_elect(tO, tP + kk * 8, vdesc + ((sV - sbase + kk * 2048) >> 4), IDESC_PV, (cu.j > 0 || kk > 0));
+          if (!(FMHA_ABL & 8)) umma_ts_elect(tO, tP + kk * 8, vdesc + ((sV - sbase + kk * 2048) >> 4), IDESC_PV, (cu.j > 0 || kk > 0));
         if (C::SEP_P) umma_commit_elect(PV_DONE);   // P_t may be overwritten
         if (cu.j + 1 == cu.w.n(t)) umma_commit_elect(O_FULL);  // O_t final: epilogue
         TRACE_EV(EV_MMA_PV, t * 64 + cu.j);
         umma_commit_elect(KV_EMPTY(vidx % C::NS));
+        PROF_MARK(7);  // PV issue
       };
       // walk the ring entries of step j in ring order: use this tile's, release the rest
       auto issue_qk = [&](Cursor& cu) {
@@ -860,6 +954,14 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         }
         started = true;
       }
+#if FMHA_PROF
+      PROF_MARK(9);
+      if (lane == 0 && g_fmha_trace) {
+        unsigned long long* dst = g_fmha_trace + (static_cast<size_t>(blockIdx.x) * 16 + warp) * 16;
+        for (int k = 0; k < 16; ++k) dst[k] = prof_acc[k];
+        dst[15] = qkc;
+      }
+#endif
     }
   } else if (warp < C::W_CORR) {
     asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(C::REG_SOFTMAX));
@@ -867,18 +969,18 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     const int t = warp >> 2, quad = warp & 3;
     const int row = quad * 32 + lane;
     const uint32_t lane_off = static_cast<uint32_t>(quad * 32) << 16;
-    const uint32_t tS = tmem + lane_off + 128 * t;  // this row's 128 S columns
-    const uint32_t tP = tmem + lane_off + (C::SEP_P ? C::TMEM_P + 64 * t : 128 * t);
-    const uint32_t S_FULL = BAR(C::B_S_FULL + t), P_FULL = BAR(C::B_P_FULL + t);
+    // this row's S (128 columns) and P (64) of step g: tmem + lane_off + col_s / col_p(t, g)
+    const uint32_t S_FULL = BAR(C::B_S_FULL + t), P_FULL = BAR(C::B_P_FULL + t), P_FULL2 = BAR(C::B_P_FULL2 + t);
     const uint32_t PV_DONE = BAR(C::B_PV_DONE + t), S_FREE = BAR(C::B_S_FREE + t);
     const uint32_t L_FULL = BAR(C::B_L_FULL + t), L_EMPTY = BAR(C::B_L_EMPTY + t);
-    const uint32_t tO = tmem + lane_off + 256 + t * C::OW;  // this row of O_t
+    const uint32_t tO = tmem + lane_off + C::col_o(t);  // this row of O_t
     const uint32_t my_turn = 2 + 2 * quad + t, other_turn = 3 + 2 * quad - t;  // 64-thread barriers
     if (C::TURNS && t == 1) named_bar_arrive(2 + 2 * quad, 64);  // tile 0 goes first
     const float c = p.scale_log2;
     const int off = p.seq_kv - p.seq_q;
     // g = real steps this thread has done so far: the phase count of S_FULL and PV_DONE
     uint32_t g = 0, lc = 0;
+    PROF_DECL
     for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
       const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED>(p, sched, idx);
       const int n = w.n(t);
@@ -900,6 +1002,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           named_bar_arrive(other_turn, 64);
           continue;
         }
+        const uint32_t tS = tmem + lane_off + C::col_s(t, g);  // this row's 128 S columns of step g
         if constexpr (BIAS && C::BIAS_PF4) {  // lanes 0-3: this step's four bias lines, 4-7: the next step's
           if (lane < 8) {
             const float* brow = p.key_bias + static_cast<size_t>(p.div_heads.div(w.bh(t))) * p.key_bias_stride;
@@ -907,9 +1010,12 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             if (pf < p.seq_kv) asm volatile("prefetch.global.L1 [%0];" ::"l"(brow + pf));
           }
         }
+        PROF_COUNT(15);
+        PROF_MARK(0);  // loop turnaround since the last P_FULL (or the item start)
         if (!pre) {
           TRACE_EV(EV_S_WAIT, j);
           mbar_wait_at(S_FULL, g & 1, 8, g, idx);
+          PROF_MARK(1);  // S_FULL wait
           TRACE_EV(EV_S_READY, j);
           tc_fence_after();
           if constexpr (C::PREFETCH_S) {
@@ -948,6 +1054,10 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           }
           tmem_wait_ld();
           reg_fence(*reinterpret_cast<uint32_t(*)[64]>(&s[64]));
+        } else if (FMHA_ABL & 1) {
+#pragma unroll
+          for (int k = 0; k < 128; ++k) s[k] = __float_as_uint(0.01f * (k & 7));
+          reg_fence(s);
         } else {
 #pragma unroll
           for (int q = 0; q < 4; ++q)
@@ -955,9 +1065,10 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           tmem_wait_ld();
           reg_fence(s);
         }
+        PROF_MARK(2);  // S TMEM load
         if (C::SEP_P) {  // S_t read: the tensor core may overwrite it with S_{t,j+1}
           tc_fence_before();
-          mbar_arrive(S_FREE);
+          FMHA_ROW_ARRIVE(S_FREE);
         }
         const int rem = lim - (w.jb + j) * 128;
         // 32-key chunks no row of this warp can see are skipped: their P is stored as zeros
@@ -1050,7 +1161,8 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           mx2 = fmax3(mx2, __uint_as_float(s[k + 4]), __uint_as_float(s[k + 5]));
           mx3 = fmax3(mx3, __uint_as_float(s[k + 6]), __uint_as_float(s[k + 7]));
         }
-        const float m_new = fmaxf(fmaxf(mx0, mx1), fmaxf(mx2, mx3));
+        const float m_new = (FMHA_ABL & 2) ? 1.f : fmaxf(fmaxf(mx0, mx1), fmaxf(mx2, mx3));
+        PROF_MARK(3);  // masks, bias, row max
         TRACE_EV(EV_MAX_DONE, j);
         // Lazy rescale: keep the old reference while the max grows by < 8 in the log2 domain (the
         // p's then stay <= 2^8, exact in fp32 and in fp16/bf16 range); l and O share the reference.
@@ -1063,11 +1175,15 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         TRACE_EV(EV_COR_ST, j);
         // PV_{t,j-1} must be done before P_t is overwritten (separate P) and before O_t is rescaled.
         // (With P over S, S_{t,j} was computed after PV_{t,j-1}: S_FULL already implies it.)
-        if (C::SEP_P && g > 0) {
+        // (ROT: P_g has its own region; PV_DONE is then waited only before a rescale, below)
+        if (C::SEP_P && !C::ROT && g > 0) {
           mbar_wait_at(PV_DONE, (g - 1) & 1, 10, g, idx);
           tc_fence_after();
         }
+        PROF_MARK(4);  // rescale decision + PV_DONE wait
         TRACE_EV(EV_COR_PV, j);  // after the PV_DONE wait
+        const uint32_t gs = g;  // this step's index (the rotation of S / P)
+        const uint32_t tP = tmem + lane_off + C::col_p(t, gs);
         ++g;
         // P = exp2(c*s - c*m_ref) (a6), rounded to the I/O type, stored to TMEM for the PV MMA
         float2 acc0 = make_float2(0.f, 0.f), acc1 = make_float2(0.f, 0.f);
@@ -1088,7 +1204,9 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             // round-trip their input through shared memory, which bar.sync does order.
             const uint32_t slot = sbase + C::OFF_MC + (t * 128 + row) * 4;
             asm volatile("st.shared.f32 [%0], %1;" ::"r"(slot), "f"(mc) : "memory");
+            PROF_MARK(5);  // pre-turn chunks
             named_bar_sync(my_turn, 64);
+            PROF_MARK(6);  // turn wait
             TRACE_EV(EV_XCHG, j);  // turn granted
             asm volatile("ld.volatile.shared.f32 %0, [%1];" : "=f"(mcv) : "r"(slot) : "memory");
           }
@@ -1135,7 +1253,8 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             pk[u] = pack2<BF16>(x0.x, x0.y);
             pk[u + 1] = pack2<BF16>(x1.x, x1.y);
           }
-          if (!defer) tmem_st_32x32b_x16(tP + 16 * hh, pk);
+          if (!defer && !(FMHA_ABL & 4)) tmem_st_32x32b_x16(tP + 16 * hh, pk);
+          if (FMHA_ABL & 4) reg_fence(pk);
         }
         if constexpr (C::DEFER_ST == 1) {
 #pragma unroll
@@ -1144,15 +1263,23 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           tmem_st_32x32b_x16(tP + 16 * 3, pk_all[3]);
         }
         };
-        if (rem_w >= 128)
+        if (FMHA_ABL & 16) {  // (timing ablation: no exponential phase, only its turn)
+          if (C::TURNS) named_bar_sync(my_turn, 64);
+        } else if (rem_w >= 128)
           exp_phase(std::false_type{});
         else
           exp_phase(std::true_type{});
         if (C::TURNS) named_bar_arrive(other_turn, 64);
+        PROF_MARK(7);  // exponentials inside the turn
         TRACE_EV(EV_EXP_DONE, j);
         // lazy rescale of this warp's rows of O_t (a7), after the exponentials so that S is no
         // longer live; at j = 0 PV overwrites O_t instead
         if (j > 0 && __any_sync(0xffffffffu, alpha != 1.f)) {
+          if (C::ROT) {  // O_t must hold PV_{t,gs-1}: PV_DONE's completions run one behind the step count,
+                         // so the parity of completion gs-1 is unambiguous although most steps skip it
+            mbar_wait_at(PV_DONE, (gs - 1) & 1, 10, gs, idx);
+            tc_fence_after();
+          }
 #pragma unroll 1
           for (int q = 0; q < D / 32; ++q) {
             uint32_t o[32];
@@ -1186,10 +1313,12 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           for (int q = 0; q < 4; ++q)
             tmem_ld_32x32b_x32(tS + 32 * q, *reinterpret_cast<uint32_t(*)[32]>(&s[32 * q]));
         }
+        PROF_MARK(8);  // rescale of O
         tmem_wait_st();
+        PROF_MARK(9);  // P store drain
         TRACE_EV(EV_EPI, j);  // P stores landed
         tc_fence_before();
-        mbar_arrive(P_FULL);
+        FMHA_ROW_ARRIVE((C::ROT && (gs & 1)) ? P_FULL2 : P_FULL);
         l = l * alpha + ((acc0.x + acc0.y) + (acc1.x + acc1.y));
       }
       if (!w.has(t)) continue;
@@ -1207,9 +1336,18 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           if constexpr (!C::LSUM_MMA) p.ws_l[o] = l;  // (LSUM_MMA: the epilogue reads l from TMEM)
         }
       }
-      mbar_arrive(L_FULL);
+      __syncwarp();
+      FMHA_ROW_ARRIVE(L_FULL);
+      PROF_MARK(10);  // item end: L_EMPTY wait, row sums
     }
     if (C::TURNS && t == 0) named_bar_sync(2 + 2 * quad, 64);  // consume tile 1's last hand-over
+#if FMHA_PROF
+    PROF_MARK(11);
+    if (lane == 0 && g_fmha_trace) {
+      unsigned long long* dst = g_fmha_trace + (static_cast<size_t>(blockIdx.x) * 16 + warp) * 16;
+      for (int k = 0; k < 16; ++k) dst[k] = prof_acc[k];
+    }
+#endif
   } else {
     asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(C::REG_CORR));
     // ================================================================ epilogue (a9)
@@ -1229,7 +1367,8 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         TRACE_EV(EV_EPI, 100 + t);
         lbits ^= 1u << t;
         float l = s_lsum[t * 128 + row];
-        mbar_arrive(BAR(C::B_L_EMPTY + t));
+        __syncwarp();
+        FMHA_ROW_ARRIVE(BAR(C::B_L_EMPTY + t));
         const int n = w.n(t);
         if (n > 0) {
           mbar_wait_at(BAR(C::B_O_FULL + t), (ofbits >> t) & 1, 14, t, idx);  // last PV of this tile
@@ -1241,7 +1380,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           l = 0.f;
           if (n > 0) {
             uint32_t lv[1];
-            tmem_ld_32x32b_x1(tmem + lane_off + 256 + t * C::OW + D, lv);
+            tmem_ld_32x32b_x1(tmem + lane_off + C::col_o(t) + D, lv);
             tmem_wait_ld();
             l = __uint_as_float(lv[0]);
           }
@@ -1257,11 +1396,11 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         const uint32_t stg = sbase + C::OFF_STG + (t % C::NSTG) * C::TILE;
         if (row == 0) tma_store_wait_read0();  // previous store out of this staging buffer done
         named_bar_sync(1, 128);
-        const uint32_t tO = tmem + lane_off + 256 + t * C::OW;
+        const uint32_t tO = tmem + lane_off + C::col_o(t);
 #pragma unroll 1
         for (int q = 0; q < D / 32; ++q) {
           uint32_t o[32];
-          if (n > 0) {
+          if (n > 0 && !(FMHA_ABL & 32)) {
             tmem_ld_32x32b_x32(tO + 32 * q, o);
             tmem_wait_ld();
             reg_fence(o);
@@ -1298,7 +1437,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         }
         if (n > 0) {  // O_t read: the next item's first PV may overwrite it
           tc_fence_before();
-          mbar_arrive(BAR(C::B_O_EMPTY + t));
+          FMHA_ROW_ARRIVE(BAR(C::B_O_EMPTY + t));
         }
         if (!rowwise && !SPLIT) {
           fence_proxy_async_smem();
