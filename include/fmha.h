@@ -38,8 +38,9 @@
  * valid until the kernel completes, stream-ordered).  `mask` is read on the host during the call.
  * Validation failures return a non-zero fmha_status_t before anything is launched; launch failures
  * return FMHA_ERR_CUDA.  Device faults surface at the caller's next synchronisation.  The library
- * is stateless and thread-safe (cached: the driver entry point for tensor-map encoding, per-device
- * kernel attributes).  There is no CPU fallback: without an sm_100 device every entry point that
+ * is thread-safe; its host state is a cache (the driver entry point for tensor-map encoding, per-device
+ * kernel attributes and device properties, all mutex-protected) plus fmha_fwd_from_host's per-thread
+ * copy streams.  There is no CPU fallback: without an sm_100 device every entry point that
  * launches returns FMHA_ERR_NO_DEVICE.
  */
 #ifndef B200FMHA_FMHA_H
@@ -151,8 +152,9 @@ FMHA_API int fmha_fwd_varlen(const void* QKV, void* O, const int32_t* cu_seqlens
 /* End-to-end variant: Q/K/V/O and kv_len are HOST buffers (pinned memory for asynchronous copies).
  * Copies Q, K, V (and kv_len) host->device into `workspace`, runs the same kernel, copies O
  * device->host.  The work is ordered after everything already queued on `stream` and pipelined over
- * up to 4 batch chunks on three streams created and released inside the call (the copy-in of chunk
- * c+1 and the copy-out of chunk c-1 overlap the kernel on chunk c); `stream` is made to wait for the
+ * up to 4 batch chunks on three internal streams (created on a thread's first call for a device and
+ * reused by that thread; the copy-in of chunk c+1 and the copy-out of chunk c-1 overlap the kernel on
+ * chunk c); `stream` is made to wait for the
  * last copy-out, so syncing `stream` (no synchronisation happens inside) makes O complete on the host.
  * Results are bitwise those of fmha_fwd (every (b, h) is independent of the batch it runs in).
  * dtype: 0 = fp16, 1 = bf16.  `workspace` is a DEVICE buffer of at least

@@ -55,6 +55,8 @@ int check_device(int* sm_count) {
   }
   static int cached_major[64], cached_sms[64];
   static bool cached[64];
+  static std::mutex mu;
+  std::lock_guard<std::mutex> lk(mu);
   if (dev < 64 && cached[dev]) {
     if (sm_count) *sm_count = cached_sms[dev];
     return cached_major[dev] == 10 ? FMHA_OK : FMHA_ERR_NO_DEVICE;
@@ -147,18 +149,8 @@ int launch_fmha_ks(const b200::FmhaParams& prm, int mode, int sm_count, cudaStre
                                    : mode == b200::MODE_PAIRX  ? b200::fmha_fwd_ks_sm100<BF16, b200::MODE_PAIRX>
                                    : mode == b200::MODE_VARLEN ? b200::fmha_fwd_ks_sm100<BF16, b200::MODE_VARLEN>
                                                                : b200::fmha_fwd_ks_sm100<BF16, b200::MODE_VARLEN_SCHED>;
-  static bool attr_done[64][4];
-  static std::mutex mu;
-  int dev = 0;
-  cudaGetDevice(&dev);
-  {
-    std::lock_guard<std::mutex> lk(mu);
-    if (dev >= 64 || !attr_done[dev][mode]) {
-      cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_ALLOC);
-      if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(fmha_ks)");
-      if (dev < 64) attr_done[dev][mode] = true;
-    }
-  }
+  if (cudaError_t e = b200::ensure_smem_attr(reinterpret_cast<const void*>(kern), C::SMEM_ALLOC); e != cudaSuccess)
+    return cuda_fail(e, "cudaFuncSetAttribute(fmha_ks)");
   dim3 grid(static_cast<unsigned>(std::min(prm.num_items, sm_count)), 1, 1);
   const bool pdl = mode != b200::MODE_VARLEN && mode != b200::MODE_VARLEN_SCHED;
   cudaError_t e = b200::launch_pdl(pdl, kern, grid, dim3(C::THREADS), C::SMEM_ALLOC, stream, prm);
@@ -182,16 +174,8 @@ int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) 
                                    : mode == b200::MODE_BIAS2D ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_BIAS2D>
                                                                : b200::fmha_fwd_sm100<D, BF16, b200::MODE_VARLEN_SCHED>;
   if (D == 64 && mode <= b200::MODE_VARLEN_SCHED && ks_enabled()) return launch_fmha_ks<BF16>(prm, mode, sm_count, stream);
-  static bool attr_done[64][7];
-  static std::mutex attr_mu;
-  std::lock_guard<std::mutex> attr_lock(attr_mu);
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (dev >= 64 || !attr_done[dev][mode]) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_ALLOC);
-    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(fmha)");
-    if (dev < 64) attr_done[dev][mode] = true;
-  }
+  if (cudaError_t e = b200::ensure_smem_attr(reinterpret_cast<const void*>(kern), C::SMEM_ALLOC); e != cudaSuccess)
+    return cuda_fail(e, "cudaFuncSetAttribute(fmha)");
   // persistent: one CTA per SM (or fewer when there is less work)
   dim3 grid(static_cast<unsigned>(std::min(prm.num_items, sm_count)), 1, 1);
   // PDL measured: +0.5% (BERT-large-512) to +4.5% (BERT-base, padded); -5% on the varlen schedule
@@ -605,43 +589,41 @@ int fmha_fwd_from_host(int dtype, const void* hQ, const void* hK, const void* hV
       dmask.kv_len = dL;
     }
   }
-  // Pipelined over batch chunks on three streams that live only for this call: the host->device
-  // copy of chunk c+1 and the device->host copy of chunk c-1 overlap the kernel on chunk c (PCIe is
-  // full duplex), ordered by events; `stream` waits for the last copy-out, so a caller that syncs
-  // `stream` sees O complete.  Each (b, h) is independent, so a chunk is just a smaller batch.
+  // Pipelined over batch chunks on three streams: the host->device copy of chunk c+1 and the
+  // device->host copy of chunk c-1 overlap the kernel on chunk c (PCIe is full duplex), ordered by
+  // events; `stream` waits for the last copy-out, so a caller that syncs `stream` sees O complete.
+  // Each (b, h) is independent, so a chunk is just a smaller batch.  The streams and events are
+  // created once per thread and device and reused (thread-local, so concurrent callers on other
+  // threads never share them).
   cudaError_t e;
   const int chunks = std::min(batch, 4);
   const size_t qb1 = qb / batch, kvb1 = kvb / batch;  // bytes per batch element
-  cudaStream_t sh = nullptr, sc = nullptr, sd = nullptr;
-  cudaEvent_t ev_start = nullptr, ev_h[8] = {}, ev_c[8] = {}, ev_d = nullptr;
-  auto cleanup = [&]() {
-    for (int c = 0; c < 8; ++c) {
-      if (ev_h[c]) cudaEventDestroy(ev_h[c]);
-      if (ev_c[c]) cudaEventDestroy(ev_c[c]);
-    }
-    if (ev_start) cudaEventDestroy(ev_start);
-    if (ev_d) cudaEventDestroy(ev_d);
-    if (sh) cudaStreamDestroy(sh);  // (returns at once; queued work still completes)
-    if (sc) cudaStreamDestroy(sc);
-    if (sd) cudaStreamDestroy(sd);
+  struct HostPipe {
+    cudaStream_t sh = nullptr, sc = nullptr, sd = nullptr;
+    cudaEvent_t start = nullptr, d = nullptr, h[4] = {}, c[4] = {};
+    bool ok = false;
   };
-  bool ok = cudaStreamCreateWithFlags(&sh, cudaStreamNonBlocking) == cudaSuccess &&
-            cudaStreamCreateWithFlags(&sc, cudaStreamNonBlocking) == cudaSuccess &&
-            cudaStreamCreateWithFlags(&sd, cudaStreamNonBlocking) == cudaSuccess &&
-            cudaEventCreateWithFlags(&ev_start, cudaEventDisableTiming) == cudaSuccess &&
-            cudaEventCreateWithFlags(&ev_d, cudaEventDisableTiming) == cudaSuccess;
-  for (int c = 0; ok && c < chunks; ++c)
-    ok = cudaEventCreateWithFlags(&ev_h[c], cudaEventDisableTiming) == cudaSuccess &&
-         cudaEventCreateWithFlags(&ev_c[c], cudaEventDisableTiming) == cudaSuccess;
-  if (!ok) {
-    e = cudaGetLastError();
-    cleanup();
-    return cuda_fail(e, "fmha_fwd_from_host streams/events");
+  thread_local HostPipe pipes[64];
+  int dev = 0;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess || dev >= 64) return cuda_fail(e, "fmha_fwd_from_host device");
+  HostPipe& hp = pipes[dev];
+  if (!hp.ok) {
+    bool ok = cudaStreamCreateWithFlags(&hp.sh, cudaStreamNonBlocking) == cudaSuccess &&
+              cudaStreamCreateWithFlags(&hp.sc, cudaStreamNonBlocking) == cudaSuccess &&
+              cudaStreamCreateWithFlags(&hp.sd, cudaStreamNonBlocking) == cudaSuccess &&
+              cudaEventCreateWithFlags(&hp.start, cudaEventDisableTiming) == cudaSuccess &&
+              cudaEventCreateWithFlags(&hp.d, cudaEventDisableTiming) == cudaSuccess;
+    for (int c = 0; ok && c < 4; ++c)
+      ok = cudaEventCreateWithFlags(&hp.h[c], cudaEventDisableTiming) == cudaSuccess &&
+           cudaEventCreateWithFlags(&hp.c[c], cudaEventDisableTiming) == cudaSuccess;
+    if (!ok) return cuda_fail(cudaGetLastError(), "fmha_fwd_from_host streams/events");
+    hp.ok = true;
   }
+  cudaStream_t sh = hp.sh, sc = hp.sc, sd = hp.sd;
+  cudaEvent_t ev_start = hp.start, ev_d = hp.d, *ev_h = hp.h, *ev_c = hp.c;
   // everything already queued on `stream` (incl. the kv_len copy) happens first
   if ((e = cudaEventRecord(ev_start, stream)) != cudaSuccess ||
       (e = cudaStreamWaitEvent(sh, ev_start, 0)) != cudaSuccess) {
-    cleanup();
     return cuda_fail(e, "fmha_fwd_from_host ordering");
   }
   int st = FMHA_OK;
@@ -675,7 +657,6 @@ int fmha_fwd_from_host(int dtype, const void* hQ, const void* hK, const void* hV
   // `stream` continues after the last copy-out (sd is in order, so it covers every chunk)
   if ((e = cudaEventRecord(ev_d, sd)) != cudaSuccess || (e = cudaStreamWaitEvent(stream, ev_d, 0)) != cudaSuccess)
     if (st == FMHA_OK) st = cuda_fail(e, "fmha_fwd_from_host join");
-  cleanup();
   return st;
 }
 

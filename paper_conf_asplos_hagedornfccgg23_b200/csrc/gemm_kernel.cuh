@@ -582,16 +582,9 @@ inline int launch_gemm_bias_act(const void* A, const void* W, const void* A2, co
                             : act == 3 ? gemm_bias_act_2sm_kernel<3>
                             : act == 4 ? gemm_bias_act_2sm_kernel<4>
                                        : gemm_bias_act_2sm_kernel<0>;
-    static bool attr2[64][5];
-    int dev2 = 0;
-    cudaGetDevice(&dev2);
-    if (dev2 >= 64 || !attr2[dev2][act]) {
-      cudaError_t e = cudaFuncSetAttribute(k2, cudaFuncAttributeMaxDynamicSharedMemorySize, Gemm2Cfg::SMEM_ALLOC);
-      if (e != cudaSuccess) {
-        snprintf(err, errlen, "cudaFuncSetAttribute(gemm2sm): %s", cudaGetErrorString(e));
-        return 4;
-      }
-      if (dev2 < 64) attr2[dev2][act] = true;
+    if (cudaError_t e = ensure_smem_attr(reinterpret_cast<const void*>(k2), Gemm2Cfg::SMEM_ALLOC); e != cudaSuccess) {
+      snprintf(err, errlen, "cudaFuncSetAttribute(gemm2sm): %s", cudaGetErrorString(e));
+      return 4;
     }
     const long long clusters = std::min<long long>(pair_tiles, sms / 2);
     cudaError_t e = launch_pdl(true, k2, dim3(static_cast<unsigned>(2 * clusters)), dim3(Gemm2Cfg::THREADS),
@@ -607,16 +600,9 @@ inline int launch_gemm_bias_act(const void* A, const void* W, const void* A2, co
                             : act == 3 ? gemm_bias_act_kernel<3>
                             : act == 4 ? gemm_bias_act_kernel<4>
                                        : gemm_bias_act_kernel<0>;
-  static bool attr_done[64][5];
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (dev >= 64 || !attr_done[dev][act]) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, GemmCfg::SMEM_ALLOC);
-    if (e != cudaSuccess) {
-      snprintf(err, errlen, "cudaFuncSetAttribute(gemm): %s", cudaGetErrorString(e));
-      return 4;
-    }
-    if (dev < 64) attr_done[dev][act] = true;
+  if (cudaError_t e = ensure_smem_attr(reinterpret_cast<const void*>(kern), GemmCfg::SMEM_ALLOC); e != cudaSuccess) {
+    snprintf(err, errlen, "cudaFuncSetAttribute(gemm): %s", cudaGetErrorString(e));
+    return 4;
   }
   const long long tiles = static_cast<long long>(prm.tiles_m) * prm.tiles_n;
   const long long r = tiles > sms ? tiles % sms : 0;  // big tiles in the last, partial wave

@@ -343,16 +343,9 @@ inline int launch_mlp_fused_w(MlpParams& prm, int act, int sms, cudaStream_t str
                             : act == 3 ? mlp_fused_kernel<NW, 3, TA>
                             : act == 4 ? mlp_fused_kernel<NW, 4, TA>
                                        : mlp_fused_kernel<NW, 0, TA>;
-  static bool attr_done[64][5];
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (dev >= 64 || !attr_done[dev][act]) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_ALLOC);
-    if (e != cudaSuccess) {
-      snprintf(err, errlen, "cudaFuncSetAttribute(mlp_fused): %s", cudaGetErrorString(e));
-      return 4;
-    }
-    if (dev < 64) attr_done[dev][act] = true;
+  if (cudaError_t e = ensure_smem_attr(reinterpret_cast<const void*>(kern), C::SMEM_ALLOC); e != cudaSuccess) {
+    snprintf(err, errlen, "cudaFuncSetAttribute(mlp_fused): %s", cudaGetErrorString(e));
+    return 4;
   }
   // Slots per group S.  One tile's layer is a serial chain: MMA (t) -> epilogue (E ~ e t, e ~ 3) ->
   // next MMA.  With S tiles in flight a group's layer takes about max(S t, t + E ceil(S / SG)) (an

@@ -13,6 +13,10 @@
 #include <cstdlib>
 #include <cuda_runtime.h>
 
+#include <mutex>
+#include <set>
+#include <utility>
+
 #include "tmem_ops.cuh"
 
 namespace b200 {
@@ -163,6 +167,22 @@ inline bool pdl_enabled() {
     return !(v && v[0] == '0');
   }();
   return on;
+}
+
+// Host: raise a kernel's dynamic shared-memory limit once per (device, kernel).  Thread-safe: the
+// library's only mutable host state besides the driver entry point (include/fmha.h promises
+// thread safety).
+inline cudaError_t ensure_smem_attr(const void* kern, int bytes) {
+  static std::mutex mu;
+  static std::set<std::pair<int, const void*>> done;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  std::lock_guard<std::mutex> lk(mu);
+  if (done.count({dev, kern})) return cudaSuccess;
+  e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+  if (e == cudaSuccess) done.insert({dev, kern});
+  return e;
 }
 
 template <typename... Args>
