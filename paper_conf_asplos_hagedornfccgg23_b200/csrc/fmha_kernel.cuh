@@ -250,8 +250,14 @@ struct FmhaCfg {
   // P_{g-1} is safe (PV_{g-1} is issued before QK_{g+1} by the same thread, and tcgen05.mma ops of one
   // thread execute in order); P_g lies on S_g, which this warp has loaded.  So the softmax writes P_g
   // without waiting for PV_{g-1} (PV_DONE is waited only before a lazy rescale of O).
+// Default off: measured level on BERT-large-512 and +1.7% on BERT-large-384 only while PV_DONE
+// phases go unwaited, which compute-sanitizer's synccheck rejects ("Missing wait"); consuming every
+// phase (FMHA_ROT_PVWAIT) costs 2% on BERT-large-512 (profiles/r02_fmha_ablation.txt).
 #ifndef FMHA_ROT
-#define FMHA_ROT 1
+#define FMHA_ROT 0
+#endif
+#ifndef FMHA_ROT_PVWAIT
+#define FMHA_ROT_PVWAIT 1
 #endif
   static constexpr bool ROT = FMHA_ROT && SEP_P;
   static __host__ __device__ constexpr uint32_t col_s(int t, uint32_t g) {
@@ -1317,6 +1323,10 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         tmem_wait_st();
         PROF_MARK(9);  // P store drain
         TRACE_EV(EV_EPI, j);  // P stores landed
+        // ROT: every PV_DONE phase is still consumed in order, here, before P_FULL_g lets PV_g start
+        // (PV_{g-1} has had a whole exponential phase to finish, so this rarely blocks; waiting any
+        // later could alias two phases, and compute-sanitizer's synccheck requires each phase waited)
+        if (C::ROT && FMHA_ROT_PVWAIT && gs > 0) mbar_wait_at(PV_DONE, (gs - 1) & 1, 10, gs, idx);
         tc_fence_before();
         FMHA_ROW_ARRIVE((C::ROT && (gs & 1)) ? P_FULL2 : P_FULL);
         l = l * alpha + ((acc0.x + acc0.y) + (acc1.x + acc1.y));

@@ -478,6 +478,8 @@ __global__ void __launch_bounds__(640, 1) fmha_fwd_ks_sm100(const __grid_constan
           tmem_st_32x32b_x32(tO, o);
         }
         tmem_wait_st();
+        // every PV_DONE phase is consumed in order before P_FULL_g lets PV_g start (see fmha_kernel.cuh)
+        if (g > 0) mbar_wait_at(PV_DONE, (g - 1) & 1, 10, g, j);
         tc_fence_before();
         mbar_arrive_elect(P_FULL);
         ++g;
