@@ -72,7 +72,7 @@ struct FmhaKsCfg {
     B_O_EMPTY = 6,   // [tile]          count 8 (the tile's softmax warps read O)
     B_Q_FULL = 8,    // [stage][tile]
     B_Q_EMPTY = 12,  // [stage][tile]
-    B_STAT = 16,     // [tile][quarter] count 2 (the two warps of a (tile, lane quarter) wrote their l)
+    B_STAT = 16,     // [tile][quarter] count 64 (the two warps' threads of a (tile, lane quarter) wrote their l)
     B_S_FREE = 24,   // [tile]          count 8 (the tile's softmax warps read S)
     B_PV_DONE = 26,  // [tile]          count 1 (commit after each PV)
     B_KV = 28        // KV_FULL[NS], KV_EMPTY[NS] (count 2: both MMA warps)
@@ -144,7 +144,7 @@ __global__ void __launch_bounds__(640, 1) fmha_fwd_ks_sm100(const __grid_constan
         mbar_init(Q_FULL(t, q), 1);
         mbar_init(Q_EMPTY(t, q), 1);
       }
-      for (int q = 0; q < 4; ++q) mbar_init(BAR(C::B_STAT + 4 * t + q), 2);
+      for (int q = 0; q < 4; ++q) mbar_init(BAR(C::B_STAT + 4 * t + q), 64);
       mbar_init(BAR(C::B_S_FREE + t), 8);
       mbar_init(BAR(C::B_PV_DONE + t), 1);
     }
@@ -493,8 +493,7 @@ __global__ void __launch_bounds__(640, 1) fmha_fwd_ks_sm100(const __grid_constan
       // parity, so a warp an item ahead never overwrites what its partner has yet to read)
       float* ls = lsum + (ec & 1) * 512 + 256 * t;
       ls[128 * h + row] = l;
-      __syncwarp();
-      mbar_arrive_elect(STAT);
+      mbar_arrive(STAT);  // (one arrival per thread: each publishes its own shared-memory write)
       if (lane == 0) tma_store_wait_read0();  // this warp's staging buffer free again
       mbar_wait_at(STAT, ec & 1, 9, ec, t);
       ++ec;

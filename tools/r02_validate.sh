@@ -13,3 +13,8 @@ for tool in memcheck racecheck synccheck; do
   done
 done
 tail -3 gpurun_out/r02_pytest_gpu.log; cat gpurun_out/r02_smoke.log | tail -2; cat gpurun_out/r02_sanitizer.txt
+# ncu: launch list of the default bench command and one --set full capture of the BERT-large-512 kernel
+ncu --metrics gpu__time_duration.sum --clock-control none -c 40 --csv --log-file gpurun_out/r02_bl5_launches.csv python bench.py --steps 5 --warmup 3 --no-cpu-baseline --no-e2e --sustained 0 > /dev/null 2>&1
+ncu --set full --clock-control none --import-source on -k regex:fmha_fwd_sm100 -s 2 -c 1 -o gpurun_out/r02_bl5_full python tools/fmha_prof.py bert_large_512 4 > /dev/null 2>&1
+timeout 300 python bench.py --steps 20 --warmup 5 > gpurun_out/r02_bench_default.json 2> gpurun_out/r02_bench_default.err
+tail -c 400 gpurun_out/r02_bench_default.json
