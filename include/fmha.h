@@ -185,6 +185,34 @@ FMHA_API int fmha_fwd_splitkv(int dtype, const void* Q, const void* K, const voi
                               float scale, int num_splits, void* workspace, size_t workspace_bytes,
                               fmha_stream_t stream);
 
+/* Stream-K tail FMHA: the same operation, layouts, masks and scale rules as
+ * fmha_fwd / fmha_fwd_bf16 (dtype 0 = fp16, 1 = bf16), in ONE launch of the persistent
+ * kernel whose last, partial round is split along the keys.  The full rounds run the fmha_fwd schedule;
+ * each of the last round's `tail_items` items is cut into s ranges of whole 128-key tiles
+ * (fmha_streamk_plan), every piece writes its online-softmax state (unnormalised fp32 O, the exp2
+ * reference scale*log2(e)*m and the row sum l) to `workspace` and counts itself in a per-item counter,
+ * and the piece that counts last merges O = sum_s 2^(m_s - M) O_s / sum_s 2^(m_s - M) l_s and stores
+ * it (one RNE rounding).  The last round then takes ~1/s of the time (BERT-large-384: 28 of 768
+ * items in the last round of 148 SMs, s = 3).  When the plan gives s = 1 (or the mask is a bias) this
+ * runs exactly fmha_fwd's kernel and schedule and does not touch `workspace`.
+ * `workspace`: DEVICE, 256-byte aligned, >= fmha_streamk_workspace_bytes(head_dim, 0) bytes, owned by
+ * the caller; it MUST be zero-filled before its first use, and every launch leaves it zero-filled
+ * again (the merging piece resets its counter), so one buffer serves any number of launches on one
+ * stream (not concurrent launches).  Results agree with fmha_fwd within the oracle tolerance, not
+ * bitwise (the tail rows are summed in another order).  Errors as fmha_fwd; too small a workspace ->
+ * FMHA_ERR_INVALID_ARG, misaligned -> FMHA_ERR_MISALIGNED. */
+FMHA_API int fmha_fwd_streamk(int dtype, const void* Q, const void* K, const void* V, void* O,
+                              const fmha_mask_t* mask, int batch, int heads, int seq_q, int seq_kv, int head_dim,
+                              float scale, void* workspace, size_t workspace_bytes, fmha_stream_t stream);
+/* Bytes of fmha_fwd_streamk's workspace for head_dim on a GPU with sm_count SMs (sm_count <= 0: the
+ * current device; 0 if there is none or head_dim is unsupported).  Host-only. */
+FMHA_API size_t fmha_streamk_workspace_bytes(int head_dim, int sm_count);
+/* The key-split count s of fmha_fwd_streamk's tail for this shape and mask kind on sm_count SMs
+ * (1 = no split), and *tail_items (may be NULL) = the items of the last, partial round.  Host-only,
+ * needs no device. */
+FMHA_API int fmha_streamk_plan(int batch, int heads, int seq_q, int seq_kv, int mask_kind, int sm_count,
+                               int* tail_items);
+
 /* GEMM + bias + activation, the MLP building block:
  *     C[m,n] = act( sum_k A[m,k] * W[n,k] + bias[n] )
  * A [M,K], W [N,K] (nn.Linear layout), bias [N] (or NULL), C [M,N]: fp16, row-major, DEVICE,

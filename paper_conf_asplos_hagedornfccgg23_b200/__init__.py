@@ -23,7 +23,7 @@ import torch
 from . import _lib
 from ._lib import FmhaError, FmhaMask, FmhaStrides
 
-__all__ = ["fmha_fwd", "fmha_fwd_splitkv", "fmha_fwd_varlen", "fmha_fwd_from_host", "gemm_bias_act", "dual_gemm_bias_act", "mlp_fused", "transformer_layer", "layer_workspace_bytes", "workspace_bytes", "FmhaError",
+__all__ = ["fmha_fwd", "fmha_fwd_splitkv", "fmha_fwd_streamk", "streamk_plan", "fmha_fwd_varlen", "fmha_fwd_from_host", "gemm_bias_act", "dual_gemm_bias_act", "mlp_fused", "transformer_layer", "layer_workspace_bytes", "workspace_bytes", "FmhaError",
            "MASK_NONE", "MASK_KEY_PADDING", "MASK_CAUSAL", "MASK_KEY_BIAS", "MASK_ATTN_BIAS", "ACTS", "version"]
 
 MASK_NONE, MASK_KEY_PADDING, MASK_CAUSAL, MASK_KEY_BIAS, MASK_ATTN_BIAS = 0, 1, 2, 3, 4
@@ -183,6 +183,73 @@ def fmha_fwd_splitkv(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, kv_len: 
                               out.data_ptr(), ctypes.byref(m), b, h, sq, skv, d, scale, splits,
                               workspace.data_ptr(), workspace.numel(), _stream_ptr(q.device))
     _lib.check(st, "fmha_fwd_splitkv")
+    return out
+
+
+_STREAMK_WS: dict = {}
+
+
+def streamk_workspace(device: torch.device, head_dim: int) -> torch.Tensor:
+    """The zero-filled workspace of fmha_fwd_streamk for `device` (cached: every launch leaves it
+    zero-filled again, so one buffer per device serves all launches on one stream)."""
+    lib = _lib.load()
+    device = torch.device(device)
+    key = (device.index if device.index is not None else torch.cuda.current_device(), head_dim)
+    ws = _STREAMK_WS.get(key)
+    if ws is None:
+        with torch.cuda.device(device):
+            need = lib.fmha_streamk_workspace_bytes(head_dim, 0)
+        if need == 0:
+            raise RuntimeError("fmha_streamk_workspace_bytes: no sm_100 device or unsupported head_dim")
+        ws = torch.zeros(need, dtype=torch.uint8, device=device)
+        _STREAMK_WS[key] = ws
+    return ws
+
+
+def streamk_plan(batch: int, heads: int, seq_q: int, seq_kv: int, sm_count: int,
+                 mask_kind: int = 0) -> tuple[int, int]:
+    """(key splits of each last-round item, items in the last round) of fmha_fwd_streamk's schedule
+    on a GPU with `sm_count` SMs (host-only; ``fmha_streamk_plan`` of the C ABI)."""
+    lib = _lib.load()
+    tail = ctypes.c_int(0)
+    s = lib.fmha_streamk_plan(batch, heads, seq_q, seq_kv, mask_kind, sm_count, ctypes.byref(tail))
+    return s, tail.value
+
+
+def fmha_fwd_streamk(q: torch.Tensor, k: torch.Tensor, v: torch.Tensor, kv_len: torch.Tensor | None = None,
+                     causal: bool = False, scale: float | None = None, out: torch.Tensor | None = None,
+                     workspace: torch.Tensor | None = None) -> torch.Tensor:
+    """fmha_fwd in one launch whose last, partial round of work items is split along the keys and
+    merged in the kernel by the piece that finishes last (stream-K tail).  q, k, v contiguous
+    [B,H,S,D] CUDA fp16/bf16.  `workspace` defaults to a cached zero-filled per-device buffer.  Calls
+    ``fmha_fwd_streamk`` of the C ABI."""
+    lib = _lib.load()
+    if q.dtype not in (torch.float16, torch.bfloat16) or k.dtype != q.dtype or v.dtype != q.dtype:
+        raise TypeError("q, k, v must share dtype fp16 or bf16")
+    if not (q.is_cuda and k.is_cuda and v.is_cuda):
+        raise TypeError("q, k, v must be CUDA tensors (no CPU fallback)")
+    if not (q.is_contiguous() and k.is_contiguous() and v.is_contiguous()):
+        raise ValueError("q, k, v must be contiguous [B,H,S,D]")
+    b, h, sq, d = q.shape
+    skv = k.shape[2]
+    if k.shape != (b, h, skv, d) or v.shape != k.shape:
+        raise ValueError(f"shape mismatch q{tuple(q.shape)} k{tuple(k.shape)} v{tuple(v.shape)}")
+    if kv_len is not None:
+        if kv_len.dtype != torch.int32 or not kv_len.is_cuda or kv_len.numel() != b:
+            raise ValueError("kv_len must be a CUDA int32 tensor of length batch")
+        kv_len = kv_len.contiguous()
+    if out is None:
+        out = torch.empty_like(q)
+    else:
+        _check_out(out, q.shape, q.dtype, q, "fmha_fwd_streamk")
+    if workspace is None:
+        workspace = streamk_workspace(q.device, d)
+    scale = 1.0 / math.sqrt(d) if scale is None else float(scale)
+    m = _mask(kv_len, causal)
+    st = lib.fmha_fwd_streamk(0 if q.dtype == torch.float16 else 1, q.data_ptr(), k.data_ptr(), v.data_ptr(),
+                              out.data_ptr(), ctypes.byref(m), b, h, sq, skv, d, scale, workspace.data_ptr(),
+                              workspace.numel(), _stream_ptr(q.device))
+    _lib.check(st, "fmha_fwd_streamk")
     return out
 
 

@@ -34,6 +34,9 @@ EXPORTED_SYMBOLS = (
     "fmha_splitkv_default_splits",
     "fmha_splitkv_workspace_bytes",
     "fmha_fwd_splitkv",
+    "fmha_fwd_streamk",
+    "fmha_streamk_workspace_bytes",
+    "fmha_streamk_plan",
     "gemm_bias_act",
     "dual_gemm_bias_act",
     "mlp_fused_fwd",
@@ -103,6 +106,13 @@ def load() -> ctypes.CDLL:
         lib.fmha_splitkv_workspace_bytes.restype = sz
         lib.fmha_fwd_splitkv.argtypes = [i32, vp, vp, vp, vp, mp, i32, i32, i32, i32, i32, f32, i32, vp, sz, vp]
         lib.fmha_fwd_splitkv.restype = i32
+    if hasattr(lib, "fmha_fwd_streamk"):  # absent only in old tuning builds
+        lib.fmha_fwd_streamk.argtypes = [i32, vp, vp, vp, vp, mp, i32, i32, i32, i32, i32, f32, vp, sz, vp]
+        lib.fmha_fwd_streamk.restype = i32
+        lib.fmha_streamk_workspace_bytes.argtypes = [i32, i32]
+        lib.fmha_streamk_workspace_bytes.restype = sz
+        lib.fmha_streamk_plan.argtypes = [i32, i32, i32, i32, i32, i32, ctypes.POINTER(i32)]
+        lib.fmha_streamk_plan.restype = i32
     if hasattr(lib, "mlp_fused_fwd"):
         lib.mlp_fused_fwd.argtypes = [vp, vp, vp, vp, i32, i32, i32, i32, vp]
         lib.mlp_fused_fwd.restype = i32

@@ -162,6 +162,7 @@ template <int D, bool BF16>
 int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) {
   using C = b200::FmhaCfg<D>;
   const int mode = prm.num_splits > 1 ? b200::MODE_SPLIT
+                   : prm.tail_splits > 1 ? (prm.pair_mode ? b200::MODE_PAIRX_TAIL : b200::MODE_DENSE_TAIL)
                    : prm.attn_bias  ? b200::MODE_BIAS2D
                    : prm.key_bias   ? b200::MODE_BIAS
                    : prm.cu_seqlens ? (prm.sched ? b200::MODE_VARLEN_SCHED : b200::MODE_VARLEN)
@@ -172,6 +173,8 @@ int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) 
                                    : mode == b200::MODE_SPLIT  ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_SPLIT>
                                    : mode == b200::MODE_BIAS   ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_BIAS>
                                    : mode == b200::MODE_BIAS2D ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_BIAS2D>
+                                   : mode == b200::MODE_DENSE_TAIL ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_DENSE_TAIL>
+                                   : mode == b200::MODE_PAIRX_TAIL ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_PAIRX_TAIL>
                                                                : b200::fmha_fwd_sm100<D, BF16, b200::MODE_VARLEN_SCHED>;
   if (D == 64 && mode <= b200::MODE_VARLEN_SCHED && ks_enabled()) return launch_fmha_ks<BF16>(prm, mode, sm_count, stream);
   if (cudaError_t e = b200::ensure_smem_attr(reinterpret_cast<const void*>(kern), C::SMEM_ALLOC); e != cudaSuccess)
@@ -221,6 +224,56 @@ int splitkv_default(long long units, int seq_q, int seq_kv, int sms) {
   return best_s;
 }
 
+// Work items of the dense schedule and its pairing mode: (unit, q-tile pair) items, or (pair_mode 1)
+// pairs of the flattened (unit, q-tile) list when a unit has an odd number (>= 3) of q-tiles and the
+// mask is not causal / a bias (BERT-large-384: no half-empty items, +8%).  With a single q-tile per
+// unit (short sequences) every item is one latency-bound step and pairing across units measured
+// slower, so those keep pair_mode 0.
+long long dense_items(long long units, int num_q_tiles, int kind, int* pair_mode) {
+  *pair_mode = (kind != FMHA_MASK_CAUSAL && kind != FMHA_MASK_KEY_BIAS && kind != FMHA_MASK_ATTN_BIAS &&
+                (num_q_tiles & 1) && num_q_tiles >= 3) ? 1 : 0;
+  return *pair_mode ? (units * num_q_tiles + 1) / 2 : units * ((num_q_tiles + 1) / 2);
+}
+
+// Stream-K tail plan (fmha_fwd_streamk): the persistent grid runs `items` two-tile items in rounds of
+// `sms`; the last, partial round's `rest` items are cut into s key ranges of whole 128-key tiles
+// (s <= nkv, rest * s <= sms: the pieces still fit one round, s <= MAX_TAIL_SPLITS), so that round
+// takes ceil(nkv / s) instead of nkv KV steps.  The merge (the last piece's stores, release / acquire
+// through L2, bulk loads of the other pieces' states, the combine) costs ~5 us on B200, about 2.5 KV
+// steps of a BERT-large item, and fmha_fwd already runs a cross-unit-paired last round as single
+// tiles (`singles`, ~0.65 of a pair step), so a split is planned only when the modelled
+// round time drops by >= 1.5 steps (profiles/r02_streamk_probe.txt: BERT-large-384 and
+// 8 x 14 x 384 x 1024 measured slower split, long key ranges 13-39% faster).  Returns s (1: no
+// split), *tail_items = rest.
+int streamk_plan(long long items, int nkv, int sms, bool singles, long long* tail_items) {
+  *tail_items = 0;
+  if (items <= 0 || sms <= 0 || nkv < 2) return 1;
+  const long long rest = items % sms;
+  if (rest == 0) return 1;
+  long long s = std::min<long long>(std::min<long long>(nkv, sms / rest), b200::MAX_TAIL_SPLITS);
+  if (s < 2) return 1;
+  const int per = static_cast<int>((nkv + s - 1) / s);
+  s = (nkv + per - 1) / per;  // every piece gets at least one key tile
+  const long long cost_fwd = (singles ? 65LL : 100LL) * nkv, cost_sk = 100LL * per + 250;
+  if (s < 2 || cost_fwd - cost_sk < 150) return 1;
+  *tail_items = rest;
+  return static_cast<int>(s);
+}
+
+// fmha_fwd's last round runs as single tiles (pair_mode 1 with at least one full round, and the
+// last round's tiles fit one round)
+bool singles_tail(long long items, long long tiles, int pair_mode, int sms) {
+  const long long full = items / sms * sms;
+  return pair_mode && full > 0 && tiles - 2 * full > 0 && tiles - 2 * full <= sms;
+}
+
+// Stream-K workspace: tail counters (one per tail item, < sms) then the pieces' states (< sms pieces
+// of two tiles x 128 rows x (D + 2) floats).
+size_t streamk_cnt_bytes(int sms) { return (static_cast<size_t>(sms) * 4 + 255) / 256 * 256; }
+size_t streamk_ws_bytes(int head_dim, int sms) {
+  return streamk_cnt_bytes(sms) + static_cast<size_t>(sms) * 2 * 128 * (head_dim + 2) * sizeof(float);
+}
+
 // The argument checks of fmha_common that need no pointers to be valid device memory: shapes, scale,
 // head_dim, mask kind.  FMHA_OK with *empty = true means there is nothing to launch.
 int validate_shape(int batch, int heads, int seq_q, int seq_kv, int head_dim, float scale, const fmha_mask_t* mask,
@@ -260,7 +313,7 @@ int validate_shape(int batch, int heads, int seq_q, int seq_kv, int head_dim, fl
 int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask,
                 int batch, int heads, int seq_q, int seq_kv, int head_dim, float scale, cudaStream_t stream,
                 int splits = 1, void* workspace = nullptr, size_t workspace_bytes = 0,
-                const fmha_strides_t* strides = nullptr) {
+                const fmha_strides_t* strides = nullptr, bool streamk = false) {
   g_last_cuda_error[0] = 0;
   bool empty = false;
   if (int vs = validate_shape(batch, heads, seq_q, seq_kv, head_dim, scale, mask, splits, &empty); vs != FMHA_OK || empty)
@@ -312,11 +365,7 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   // scores (-inf) still map to exp2(-inf) = 0 instead of -inf * 0 = NaN.  1e-30 perturbs visible
   // scores by < 1e-25 in the exponent.
   prm.scale_log2 = std::max(scale * 1.4426950408889634f, 1e-30f);
-  // odd q-tile counts >= 3 (non-causal): pair tiles across units so no item has an empty second
-  // tile (BERT-large-384: +8%).  With a single q-tile per unit (short sequences) every item is one
-  // latency-bound step and pairing across units measured slower, so those keep pair_mode 0.
-  prm.pair_mode = (kind != FMHA_MASK_CAUSAL && kind != FMHA_MASK_KEY_BIAS && kind != FMHA_MASK_ATTN_BIAS &&
-                   (prm.num_q_tiles & 1) && prm.num_q_tiles >= 3) ? 1 : 0;
+  long long items = dense_items(units, prm.num_q_tiles, kind, &prm.pair_mode);
   if (kind == FMHA_MASK_KEY_BIAS) {
     prm.key_bias = mask->key_bias;
     prm.key_bias_stride = mask->key_bias_stride;
@@ -333,9 +382,25 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
     prm.inv_scale = 1.4426950408889634f / prm.scale_log2;  // c * inv_scale = log2(e) exactly as used
     prm.mask_kind = FMHA_MASK_NONE;
   }
-  long long items = prm.pair_mode ? (units * prm.num_q_tiles + 1) / 2 : units * ((prm.num_q_tiles + 1) / 2);
   prm.single_from = 0x7fffffff;
-  if (prm.pair_mode) {  // a last, partial round of tile pairs runs as single tiles (half as long)
+  prm.tail_from = 0x7fffffff;
+  long long tail_items = 0;
+  const int tail_s = (streamk && splits == 1 && kind != FMHA_MASK_KEY_BIAS && kind != FMHA_MASK_ATTN_BIAS)
+                         ? streamk_plan(items, (seq_kv + 127) / 128, sm_count,
+                                        singles_tail(items, units * prm.num_q_tiles, prm.pair_mode, sm_count), &tail_items)
+                         : 1;
+  if (tail_s > 1) {  // stream-K tail: the last round's items as key-range pieces, merged in the kernel
+    if (!workspace || workspace_bytes < streamk_ws_bytes(head_dim, sm_count)) return FMHA_ERR_INVALID_ARG;
+    if (reinterpret_cast<uintptr_t>(workspace) % 256 != 0) return FMHA_ERR_MISALIGNED;
+    const int nkv = (seq_kv + 127) / 128;
+    prm.tail_from = static_cast<int>(items - tail_items);
+    prm.tail_splits = tail_s;
+    prm.tail_tiles = (nkv + tail_s - 1) / tail_s;
+    prm.div_tail.init(static_cast<uint32_t>(tail_s));
+    prm.tail_cnt = static_cast<unsigned int*>(workspace);
+    prm.ws_tail = reinterpret_cast<float*>(static_cast<uint8_t*>(workspace) + streamk_cnt_bytes(sm_count));
+    items = prm.tail_from + tail_items * tail_s;
+  } else if (prm.pair_mode) {  // a last, partial round of tile pairs runs as single tiles (half as long)
     const long long tiles = units * prm.num_q_tiles;
     const long long full = items / sm_count * sm_count;  // pair items in full rounds
     const long long rest = tiles - 2 * full;              // tiles left for the last round
@@ -714,6 +779,35 @@ int fmha_fwd_splitkv(int dtype, const void* Q, const void* K, const void* V, voi
   if (num_splits < 0 || num_splits > 1024) return FMHA_ERR_UNSUPPORTED;
   return fmha_common(dtype == 1, Q, K, V, O, mask, batch, heads, seq_q, seq_kv, head_dim, scale,
                      reinterpret_cast<cudaStream_t>(stream), num_splits, workspace, workspace_bytes);
+}
+
+int fmha_streamk_plan(int batch, int heads, int seq_q, int seq_kv, int mask_kind, int sm_count, int* tail_items) {
+  if (tail_items) *tail_items = 0;
+  if (batch <= 0 || heads <= 0 || seq_q <= 0 || seq_kv <= 0 || sm_count <= 0) return 1;
+  if (mask_kind == FMHA_MASK_KEY_BIAS || mask_kind == FMHA_MASK_ATTN_BIAS) return 1;
+  int pair_mode = 0;
+  const long long units = static_cast<long long>(batch) * heads;
+  const int nq = (seq_q + 127) / 128;
+  const long long items = dense_items(units, nq, mask_kind, &pair_mode);
+  long long rest = 0;
+  const int s = streamk_plan(items, (seq_kv + 127) / 128, sm_count, singles_tail(items, units * nq, pair_mode, sm_count),
+                             &rest);
+  if (tail_items) *tail_items = static_cast<int>(rest);
+  return s;
+}
+
+size_t fmha_streamk_workspace_bytes(int head_dim, int sm_count) {
+  if (head_dim != 64 && head_dim != 128) return 0;
+  if (sm_count <= 0 && check_device(&sm_count) != FMHA_OK) return 0;
+  return streamk_ws_bytes(head_dim, sm_count);
+}
+
+int fmha_fwd_streamk(int dtype, const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask,
+                     int batch, int heads, int seq_q, int seq_kv, int head_dim, float scale, void* workspace,
+                     size_t workspace_bytes, fmha_stream_t stream) {
+  if (dtype != 0 && dtype != 1) return FMHA_ERR_UNSUPPORTED;
+  return fmha_common(dtype == 1, Q, K, V, O, mask, batch, heads, seq_q, seq_kv, head_dim, scale,
+                     reinterpret_cast<cudaStream_t>(stream), 1, workspace, workspace_bytes, nullptr, true);
 }
 
 int mlp_fused_fwd(const void* X, const void* W, const void* bias, void* Y, int M, int width, int layers, int act,

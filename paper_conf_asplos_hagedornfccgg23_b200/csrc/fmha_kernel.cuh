@@ -78,6 +78,14 @@ __device__ unsigned int g_fmha_trace_n = 0;
 #endif
 // FMHA_ELECT: the per-row hand-offs (S_FREE, P_FULL, L_FULL, L_EMPTY, O_EMPTY) arrive once per warp
 // (elect.sync, barrier count 4) instead of once per thread (count 128): 32x fewer mbarrier updates.
+// FMHA_SK_ABL (timing only, wrong results): bit 0 skips the stream-K count + merge, bit 1 the pieces'
+// workspace stores
+#ifndef FMHA_SK_ABL
+#define FMHA_SK_ABL 0
+#endif
+#ifndef FMHA_SUMCHECK
+#define FMHA_SUMCHECK 0
+#endif
 #ifndef FMHA_ELECT
 #define FMHA_ELECT 0
 #endif
@@ -195,7 +203,18 @@ struct FmhaParams {
   const uint16_t* attn_bias;
   long long ab_sb, ab_sh, ab_sq;
   int bias_cols8;
+  // Stream-K tail (MODE_DENSE_TAIL / MODE_PAIRX_TAIL, fmha_fwd_streamk): items
+  // idx >= tail_from are pieces of the last, partial round's items: piece idx - tail_from is split
+  // s = (idx - tail_from) % tail_splits of tail item r = (idx - tail_from) / tail_splits (= the
+  // item tail_from + r of the plain numbering) and visits its KV tiles [s * tail_tiles, (s + 1) *
+  // tail_tiles).  Every piece writes its online-softmax state (unnormalised O, mc, l) to ws_tail and
+  // counts itself in tail_cnt[r]; the piece that counts last merges the splits and stores O.
+  int tail_from, tail_splits, tail_tiles;
+  FastDiv div_tail;
+  unsigned int* tail_cnt;  // [tail items]; zero before the launch, zero again after it
+  float* ws_tail;          // [tail item][split][tile] x {O [D/4][128 rows] float4, mc [128], l [128]} (fp32)
 };
+constexpr int MAX_TAIL_SPLITS = 4;
 
 template <int D>
 struct FmhaCfg {
@@ -224,7 +243,8 @@ struct FmhaCfg {
   static constexpr int OFF_ONES = OFF_STG + NSTG * TILE;  // LSUM_MMA: 128 x 64 ones (16 KB)
   static constexpr int OFF_LSUM = OFF_ONES + (LSUM_MMA ? CHUNK : 0);  // float l[2 tiles][128 rows]
   static constexpr int OFF_MC = OFF_LSUM + 2 * 128 * 4;    // float mc[2 tiles][128 rows] (turn fence)
-  static constexpr int OFF_BAR = OFF_MC + 2 * 128 * 4;
+  static constexpr int OFF_MREF = OFF_MC + 2 * 128 * 4;  // float mc[2 tiles][128 rows] at item end (tail pieces)
+  static constexpr int OFF_BAR = OFF_MREF + 2 * 128 * 4;
   // barrier slots
   enum : int {
     B_S_FULL = 0, B_P_FULL = 2, B_O_FULL = 4, B_PV_DONE = 6, B_O_EMPTY = 8, B_L_FULL = 12,
@@ -234,7 +254,8 @@ struct FmhaCfg {
   // be two P hand-offs ahead of the MMA warp (S_FULL_g only implies PV_{g-2} was issued), which one
   // barrier's phase parity cannot tell apart; two barriers by step parity can.
   static constexpr int B_P_FULL2 = B_KV + 2 * NS;
-  static constexpr int NUM_BARS = B_P_FULL2 + 2;
+  static constexpr int B_MERGE = B_P_FULL2 + 2;  // stream-K merge: bulk loads of the pieces' states
+  static constexpr int NUM_BARS = B_MERGE + 1;
   static constexpr int OFF_TMEMPTR = OFF_BAR + NUM_BARS * 8;
   static constexpr int OFF_SCHED = OFF_TMEMPTR + 16;  // SchedTable (sched mode 1 only)
   static constexpr int SMEM_ALLOC = OFF_SCHED + 4 * (3 * (SCHED_MAX_LEVELS + 2) + SCHED_MAX_SEQS);
@@ -404,6 +425,7 @@ struct WorkItem {
   int bat0, bat1;   // dense: b of unit bh0 / bh1
   int jb;          // split-KV: first KV tile of this item's range (0 otherwise)
   int split;       // split-KV: split index
+  int tail;        // stream-K tail piece: its tail item r (-1: a whole item)
   // 4-D TMA coordinates (c1, c2, c3) of the block starting at row r of tile t (c0 = d):
   // dense maps are {D, rows, heads, batch}, varlen maps {D, heads, tokens, 1}
   __device__ __forceinline__ int c1(bool varlen, int t, int r) const { return varlen ? (t ? head1 : head) : r; }
@@ -424,12 +446,22 @@ struct WorkItem {
   }
 };
 
-template <bool PAIRX, bool VL, bool SPLIT = false>
+template <bool PAIRX, bool VL, bool SPLIT = false, bool TAIL = false>
 __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
   WorkItem w;
   int qt0;
   w.jb = 0;
   w.split = 0;
+  w.tail = -1;
+  if constexpr (TAIL) {
+    if (idx >= p.tail_from) {  // piece (tail item r, split) of item tail_from + r
+      const int piece = idx - p.tail_from;
+      const int r = p.div_tail.div(piece);
+      w.split = piece - r * p.tail_splits;
+      w.tail = r;
+      idx = p.tail_from + r;
+    }
+  }
   if constexpr (SPLIT) {
     const int rest = p.div_splits.div(idx);
     w.split = idx - rest * p.num_splits;
@@ -502,6 +534,13 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
     w.jb = w.split * p.split_tiles;
     w.n0 = min(max(w.n0 - w.jb, 0), p.split_tiles);
     w.n1 = min(max(w.n1 - w.jb, 0), p.split_tiles);
+  }
+  if constexpr (TAIL) {  // a tail piece: its split's KV tiles [jb, jb + tail_tiles)
+    if (w.tail >= 0) {
+      w.jb = w.split * p.tail_tiles;
+      w.n0 = min(max(w.n0 - w.jb, 0), p.tail_tiles);
+      w.n1 = min(max(w.n1 - w.jb, 0), p.tail_tiles);
+    }
   }
   return w;
 }
@@ -596,6 +635,7 @@ __device__ __forceinline__ WorkItem sched_item(const FmhaParams& p, const SchedT
   WorkItem w;
   w.jb = 0;
   w.split = 0;
+  w.tail = -1;
   w.has0 = true;
   int si0, h0, si1, h1;
   if (r < full) {  // q-tiles 2 pr, 2 pr + 1 of one unit
@@ -638,12 +678,12 @@ __device__ __forceinline__ WorkItem sched_item(const FmhaParams& p, const SchedT
 }
 
 // decode_item, or sched_item in sched mode
-template <bool PAIRX, bool VL, bool SPLIT, bool SCHED>
+template <bool PAIRX, bool VL, bool SPLIT, bool SCHED, bool TAIL = false>
 __device__ __forceinline__ WorkItem get_item(const FmhaParams& p, const SchedTable* tb, int idx) {
   if constexpr (SCHED) {
     return sched_item(p, tb, idx);
   } else {
-    return decode_item<PAIRX, VL, SPLIT>(p, idx);
+    return decode_item<PAIRX, VL, SPLIT, TAIL>(p, idx);
   }
 }
 
@@ -651,16 +691,21 @@ __device__ __forceinline__ WorkItem get_item(const FmhaParams& p, const SchedTab
 // FmhaParams::pair_mode); varlen packed; varlen packed with the cost-sorted schedule.  Separate
 // instances keep the varlen and scheduling code out of the dense kernels entirely.
 enum : int { MODE_DENSE = 0, MODE_PAIRX = 1, MODE_VARLEN = 2, MODE_VARLEN_SCHED = 3, MODE_SPLIT = 4, MODE_BIAS = 5,
-             MODE_BIAS2D = 6 };
+             MODE_BIAS2D = 6, MODE_DENSE_TAIL = 7, MODE_PAIRX_TAIL = 8 };
 
 template <int D, bool BF16, int MODE>
 __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
   using C = FmhaCfg<D>;
-  using XS = ExpShape<D, MODE == MODE_PAIRX, MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
+  using XS = ExpShape<D, MODE == MODE_PAIRX || MODE == MODE_PAIRX_TAIL, MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
                       MODE == MODE_BIAS || MODE == MODE_BIAS2D>;
-  constexpr bool PAIRX = MODE == MODE_PAIRX, VL = MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
+  constexpr bool TAIL = MODE == MODE_DENSE_TAIL || MODE == MODE_PAIRX_TAIL;
+  constexpr bool PAIRX = MODE == MODE_PAIRX || MODE == MODE_PAIRX_TAIL, VL = MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
                  SCHED = MODE == MODE_VARLEN_SCHED, SPLIT = MODE == MODE_SPLIT, BIAS = MODE == MODE_BIAS,
                  BIAS2D = MODE == MODE_BIAS2D;
+  // FMHA_SUMCHECK: the row max is taken over the polynomial columns only once a row has a reference,
+  // and the step's sum of p guards the rest (softmax loop, redo_step)
+  constexpr bool SUMCHK = FMHA_SUMCHECK && C::SEP_P && !C::ROT && !C::PREFETCH_S && !C::SPLIT_LD && !C::LSUM_MMA &&
+                          !BIAS && !BIAS2D && !SPLIT && FMHA_ABL == 0 && C::DEFER_ST == 0;
   // Dynamic shared memory starts at the (1024-byte aligned) base of the CTA's shared window; the
   // SWIZZLE_128B tiles need that alignment.  Using the base directly keeps smem addresses uniform.
   extern __shared__ __align__(1024) uint8_t smem[];
@@ -695,6 +740,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         mbar_init(Q_EMPTY(t, q), 1);
       }
     }
+    mbar_init(BAR(C::B_MERGE), 1);
     for (int s = 0; s < C::NS; ++s) {
       mbar_init(KV_FULL(s), 1);
       mbar_init(KV_EMPTY(s), 2);  // released by both MMA warps
@@ -756,7 +802,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         }
       };
       for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
-        const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED>(p, sched, idx);
+        const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED, TAIL>(p, sched, idx);
         const int N = max(w.n0, w.n1);
 #pragma unroll
         for (int t = 0; t < 2; ++t) {
@@ -823,7 +869,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       auto seek = [&](Cursor& cu, int k, uint32_t base) {
         cu.valid = false;
         for (int idx; (idx = item_at<SCHED>(p, sched, k)) >= 0; ++k) {
-          const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED>(p, sched, idx);
+          const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED, TAIL>(p, sched, idx);
           const int N = max(w.n0, w.n1);
           if (N == 0) continue;
           cu.w.n0 = w.n0;
@@ -988,7 +1034,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     uint32_t g = 0, lc = 0;
     PROF_DECL
     for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
-      const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED>(p, sched, idx);
+      const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED, TAIL>(p, sched, idx);
       const int n = w.n(t);
       const int N = C::TURNS ? max(w.n0, w.n1) : n;
       TRACE_EV(EV_ITEM, 1);
@@ -1156,6 +1202,24 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           for (int k = 0; k < 128; ++k)
             if (k >= rem) s[k] = __float_as_uint(-INFINITY);
         }
+        // SUMCHK: once the row has a reference, only the scores of the polynomial-exp2 columns are
+        // max-reduced (the polynomial needs x <= 8); the MUFU columns are checked after the fact by
+        // the step's sum of p (a p > 2^15 makes the sum exceed 2^15, an overflow makes it inf), and a
+        // step that fails the check is redone from the full max (redo_step below).
+        bool full_max = true;
+        if constexpr (SUMCHK) {
+          if (m_ref != -INFINITY) {
+            float pa = -INFINITY, pb = -INFINITY;
+#pragma unroll
+            for (int q = 0; q < 64; q += 2) {
+              if (XS::poly_pair(q)) pa = fmax3(pa, __uint_as_float(s[2 * q]), __uint_as_float(s[2 * q + 1]));
+              if (XS::poly_pair(q + 1)) pb = fmax3(pb, __uint_as_float(s[2 * q + 2]), __uint_as_float(s[2 * q + 3]));
+            }
+            full_max = (fmaxf(pa, pb) - m_ref) * c > 8.f;
+          }
+        }
+        float m_new = m_ref;
+        if (full_max) {
         // (SPLIT_LD: the first 64 columns' max is mxh when none of them is masked, else recomputed)
         const int k_max0 = (C::SPLIT_LD && mxh != -INFINITY) ? 64 : 0;
         float mx0 = fmaxf(m_ref, mxh), mx1 = -INFINITY, mx2 = -INFINITY, mx3 = -INFINITY;
@@ -1167,7 +1231,8 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           mx2 = fmax3(mx2, __uint_as_float(s[k + 4]), __uint_as_float(s[k + 5]));
           mx3 = fmax3(mx3, __uint_as_float(s[k + 6]), __uint_as_float(s[k + 7]));
         }
-        const float m_new = (FMHA_ABL & 2) ? 1.f : fmaxf(fmaxf(mx0, mx1), fmaxf(mx2, mx3));
+        m_new = (FMHA_ABL & 2) ? 1.f : fmaxf(fmaxf(mx0, mx1), fmaxf(mx2, mx3));
+        }
         PROF_MARK(3);  // masks, bias, row max
         TRACE_EV(EV_MAX_DONE, j);
         // Lazy rescale: keep the old reference while the max grows by < 8 in the log2 domain (the
@@ -1177,7 +1242,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           alpha = (m_ref == -INFINITY) ? 0.f : ex2((m_ref - m_new) * c);
           m_ref = m_new;
         }
-        const float mc = (m_ref == -INFINITY) ? 0.f : m_ref * c;
+        float mc = (m_ref == -INFINITY) ? 0.f : m_ref * c;
         TRACE_EV(EV_COR_ST, j);
         // PV_{t,j-1} must be done before P_t is overwritten (separate P) and before O_t is rescaled.
         // (With P over S, S_{t,j} was computed after PV_{t,j-1}: S_FULL already implies it.)
@@ -1196,8 +1261,9 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         float mcv = mc;
         // two instances: no chunk test at all on unmasked steps (the common case), so ptxas can
         // interleave the chunks freely; per-chunk skipping on steps with masked columns
-        auto exp_phase = [&](auto skip_tag) {
+        auto exp_phase = [&](auto skip_tag, auto turn_tag) {
           constexpr bool SKIP = decltype(skip_tag)::value;
+          constexpr bool TURN = decltype(turn_tag)::value;  // false: a SUMCHK redo, already inside the turn
           // DEFER_ST: the tcgen05.st of a post-turn chunk's P is issued after the next chunk's math
           // (1: all at the end of the phase; 2: one chunk later) -- ptxas does not move MUFU work of
           // a later chunk above a tcgen05.st, so storing each chunk right away left a burst of
@@ -1205,7 +1271,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           uint32_t pk_all[4][16];
 #pragma unroll
         for (int hh = 0; hh < 4; ++hh) {
-          if (hh == XS::PRE_CHUNKS) {
+          if (TURN && hh == XS::PRE_CHUNKS) {
             // The exponentials are register-only work that ptxas would hoist above the barrier:
             // round-trip their input through shared memory, which bar.sync does order.
             const uint32_t slot = sbase + C::OFF_MC + (t * 128 + row) * 4;
@@ -1272,9 +1338,34 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         if (FMHA_ABL & 16) {  // (timing ablation: no exponential phase, only its turn)
           if (C::TURNS) named_bar_sync(my_turn, 64);
         } else if (rem_w >= 128)
-          exp_phase(std::false_type{});
+          exp_phase(std::false_type{}, std::true_type{});
         else
-          exp_phase(std::true_type{});
+          exp_phase(std::true_type{}, std::true_type{});
+        if constexpr (SUMCHK) {  // redo_step: some p of this row exceeded 2^15 (rare; inside the turn)
+          const bool bad = !(((acc0.x + acc0.y) + (acc1.x + acc1.y)) <= 32768.f);
+          if (__any_sync(0xffffffffu, bad)) {
+            if (bad) {  // full max, lazy-rescale factor, new reference (alpha was 1: no full max ran)
+              float mx0 = m_ref, mx1 = -INFINITY;
+#pragma unroll
+              for (int k = 0; k < 128; k += 4) {
+                mx0 = fmax3(mx0, __uint_as_float(s[k]), __uint_as_float(s[k + 1]));
+                mx1 = fmax3(mx1, __uint_as_float(s[k + 2]), __uint_as_float(s[k + 3]));
+              }
+              const float mn = fmaxf(mx0, mx1);
+              alpha = ex2((m_ref - mn) * c);
+              m_ref = mn;
+              mc = m_ref * c;
+            }
+            mcv = mc;  // (rows that passed recompute bit-identical p)
+            acc0 = make_float2(0.f, 0.f);
+            acc1 = make_float2(0.f, 0.f);
+            tmem_wait_st();  // the first pass's P stores have landed before they are overwritten
+            if (rem_w >= 128)
+              exp_phase(std::false_type{}, std::false_type{});
+            else
+              exp_phase(std::true_type{}, std::false_type{});
+          }
+        }
         if (C::TURNS) named_bar_arrive(other_turn, 64);
         PROF_MARK(7);  // exponentials inside the turn
         TRACE_EV(EV_EXP_DONE, j);
@@ -1339,6 +1430,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       TRACE_EV(EV_ITEM, 3);
       ++lc;
       s_lsum[t * 128 + row] = l;
+      if constexpr (TAIL) reinterpret_cast<float*>(smem + C::OFF_MREF)[t * 128 + row] = (m_ref == -INFINITY) ? -INFINITY : m_ref * c;
       if constexpr (SPLIT) {  // this split's row statistics (rows inside the sequence only)
         if (qi < p.seq_q) {
           const size_t o = (static_cast<size_t>(w.split) * p.num_units + w.bh(t)) * p.seq_q + qi;
@@ -1368,7 +1460,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     // (which lived in local memory)
     uint32_t ofbits = 0, lbits = 0;
     for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
-      const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED>(p, sched, idx);
+      const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED, TAIL>(p, sched, idx);
       // ------------------------------------------------------------ epilogue per tile (a9)
 #pragma unroll 1
       for (int t = 0; t < 2; ++t) {
@@ -1377,6 +1469,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         TRACE_EV(EV_EPI, 100 + t);
         lbits ^= 1u << t;
         float l = s_lsum[t * 128 + row];
+        const float mref = TAIL ? reinterpret_cast<const float*>(smem + C::OFF_MREF)[t * 128 + row] : 0.f;
         __syncwarp();
         FMHA_ROW_ARRIVE(BAR(C::B_L_EMPTY + t));
         const int n = w.n(t);
@@ -1385,6 +1478,36 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           TRACE_EV(EV_EPI, 110 + t);
           ofbits ^= 1u << t;
           tc_fence_after();
+        }
+        if constexpr (TAIL) {
+          if (w.tail >= 0 && !(FMHA_SK_ABL & 2)) {  // stream-K piece: this split's state to the workspace, O
+                              // as float4 columns [D/4][128 rows] (a warp's store instruction writes 512
+                              // contiguous bytes; the merge reads it back the same way, conflict-free)
+            float* dst = p.ws_tail + static_cast<size_t>((w.tail * p.tail_splits + w.split) * 2 + t) * (128 * (D + 2));
+            const uint32_t tO = tmem + lane_off + C::col_o(t);
+#pragma unroll 1
+            for (int q = 0; q < D / 32; ++q) {
+              uint32_t o[32];
+              if (n > 0) {
+                tmem_ld_32x32b_x32(tO + 32 * q, o);
+                tmem_wait_ld();
+                reg_fence(o);
+              } else {
+#pragma unroll
+                for (int k = 0; k < 32; ++k) o[k] = 0u;
+              }
+#pragma unroll
+              for (int c4 = 0; c4 < 8; ++c4)
+                st_global_v4(dst + ((8 * q + c4) * 128 + row) * 4, o[4 * c4], o[4 * c4 + 1], o[4 * c4 + 2], o[4 * c4 + 3]);
+            }
+            dst[D * 128 + row] = mref;
+            dst[(D + 1) * 128 + row] = l;
+            if (n > 0) {
+              tc_fence_before();
+              FMHA_ROW_ARRIVE(BAR(C::B_O_EMPTY + t));
+            }
+            continue;
+          }
         }
         if constexpr (C::LSUM_MMA) {  // l = O_t[row, D] (the ones column of the PV MMA)
           l = 0.f;
@@ -1462,6 +1585,122 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           }
         }
         TRACE_EV(EV_EPI, 120 + t);
+      }
+      if constexpr (TAIL && !(FMHA_SK_ABL & 1)) {
+        if (w.tail >= 0) {
+          // count this piece (after its stores are visible GPU-wide); the piece that counts last merges
+          //   M = max_s mc_s,  O = sum_s 2^(mc_s - M) O_s / sum_s 2^(mc_s - M) l_s
+          // (as fmha_splitkv_combine_kernel) and stores O through the usual staging buffer + TMA
+          __threadfence();
+          named_bar_sync(1, 128);
+          volatile uint32_t* last_flag = reinterpret_cast<volatile uint32_t*>(smem + C::OFF_TMEMPTR + 4);
+          if (row == 0) {
+            const unsigned prev = atomicAdd(p.tail_cnt + w.tail, 1u);
+            const bool last = prev == static_cast<unsigned>(p.tail_splits - 1);
+            if (last) atomicExch(p.tail_cnt + w.tail, 0u);  // every piece has counted: reset for the next launch
+            *last_flag = last ? 1u : 0u;
+          }
+          named_bar_sync(1, 128);
+          if (*last_flag) {
+            // The merging piece is its CTA's last item (the pieces fill the final round), so the Q + K/V
+            // ring region [0, OFF_STG) is idle: the splits' states land there by bulk copies, 64 columns
+            // of every split at a time (S x 32 KB) plus their row statistics (S x 1 KB), then each
+            // thread merges its own row out of shared memory.
+            const int S = p.tail_splits;
+            constexpr int TS = 128 * (D + 2);       // floats per (piece, tile)
+            constexpr uint32_t HALF = 128 * 64 * 4; // bytes of 64 columns of one split
+            constexpr uint32_t STAT = MAX_TAIL_SPLITS * HALF;  // landing offset of the statistics
+            static_assert(STAT + MAX_TAIL_SPLITS * 1024 <= C::OFF_STG, "merge landing zone");
+            const uint32_t mbar = BAR(C::B_MERGE);
+            uint32_t mph = 0;
+            if (row == 0) {
+              __threadfence();
+              fence_proxy_async_all();  // the other pieces' generic stores, then async-proxy reads
+            }
+#pragma unroll 1
+            for (int t = 0; t < 2; ++t) {
+              if (!w.has(t)) continue;
+              const float* src = p.ws_tail + static_cast<size_t>(w.tail * S * 2 + t) * TS;  // split s at + 2 s TS
+              float wt[MAX_TAIL_SPLITS];
+              float inv = 0.f;
+              const uint32_t stg = sbase + C::OFF_STG + (t % C::NSTG) * C::TILE;
+              if (row == 0) tma_store_wait_read0();
+#pragma unroll 1
+              for (int hf = 0; hf < D / 64; ++hf) {
+                if (row == 0) {
+                  fence_proxy_async_smem();  // earlier generic reads of the landing zone, then async writes
+                  mbar_arrive_expect_tx(mbar, S * HALF + (hf == 0 ? S * 1024u : 0u));
+                  for (int sp = 0; sp < S; ++sp) {
+                    bulk_load(sbase + sp * HALF, src + sp * 2 * TS + hf * (HALF / 4), HALF, mbar);
+                    if (hf == 0) bulk_load(sbase + STAT + sp * 1024, src + sp * 2 * TS + D * 128, 1024, mbar);
+                  }
+                }
+                mbar_wait(mbar, mph);
+                mph ^= 1;
+                if (hf == 0) {  // M = max_s mc_s, weights 2^(mc_s - M), L = sum_s w_s l_s
+                  const float* st = reinterpret_cast<const float*>(smem + STAT);
+                  float M = -INFINITY, L = 0.f;
+#pragma unroll
+                  for (int sp = 0; sp < MAX_TAIL_SPLITS; ++sp)
+                    if (sp < S) M = fmaxf(M, st[sp * 256 + row]);
+#pragma unroll
+                  for (int sp = 0; sp < MAX_TAIL_SPLITS; ++sp) {
+                    wt[sp] = 0.f;
+                    if (sp < S) {
+                      const float m = st[sp * 256 + row];
+                      if (m != -INFINITY) {  // (a split with no visible key for this row has l = 0, O = 0)
+                        wt[sp] = ex2(m - M);
+                        L += wt[sp] * st[sp * 256 + 128 + row];
+                      }
+                    }
+                  }
+                  inv = (L > 0.f) ? 1.f / L : 0.f;  // fully masked row -> 0 (R4)
+#pragma unroll
+                  for (int sp = 0; sp < MAX_TAIL_SPLITS; ++sp) wt[sp] *= inv;
+                  named_bar_sync(1, 128);  // (the staging buffer's previous store has been read)
+                }
+#pragma unroll 1
+                for (int q = 0; q < 2; ++q) {  // 32-column chunks of this half
+                  float v[32];
+#pragma unroll
+                  for (int k = 0; k < 32; ++k) v[k] = 0.f;
+#pragma unroll
+                  for (int sp = 0; sp < MAX_TAIL_SPLITS; ++sp) {
+                    if (sp < S) {
+#pragma unroll
+                      for (int c4 = 0; c4 < 8; ++c4) {
+                        const float4 x = ld_shared_f4(sbase + sp * HALF + ((8 * q + c4) * 128 + row) * 16);
+                        v[4 * c4] += wt[sp] * x.x;
+                        v[4 * c4 + 1] += wt[sp] * x.y;
+                        v[4 * c4 + 2] += wt[sp] * x.z;
+                        v[4 * c4 + 3] += wt[sp] * x.w;
+                      }
+                    }
+                  }
+                  const int col0 = 64 * hf + 32 * q;
+                  const uint32_t box = stg + (col0 / 64) * C::CHUNK + row * 128;
+#pragma unroll
+                  for (int u = 0; u < 4; ++u) {
+                    const int unit = ((col0 % 64) / 8) + u;
+                    st_shared_v4(box + ((unit ^ (row & 7)) << 4), pack2<BF16>(v[8 * u], v[8 * u + 1]),
+                                 pack2<BF16>(v[8 * u + 2], v[8 * u + 3]), pack2<BF16>(v[8 * u + 4], v[8 * u + 5]),
+                                 pack2<BF16>(v[8 * u + 6], v[8 * u + 7]));
+                  }
+                }
+                named_bar_sync(1, 128);  // every thread has read this half's landing zone
+              }
+              fence_proxy_async_smem();
+              named_bar_sync(1, 128);
+              if (row == 0) {
+#pragma unroll
+                for (int c2 = 0; c2 < D / 64; ++c2)
+                  tma_store_4d(&p.tmO, stg + c2 * C::CHUNK, c2 * 64, w.c1(false, t, w.row0(t)), w.c2(false, t, w.row0(t)),
+                               w.c3(false, t));
+                tma_store_commit();
+              }
+            }
+          }
+        }
       }
     }
     if (row == 0) tma_store_wait0();
