@@ -134,6 +134,14 @@ bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) ==
 // dense, cross-unit pair and varlen modes, selected with B200_FMHA_KS=1.  Off by default: measured
 // against the two-tile kernel on the same boxes it is level on BERT-large-512 (640 vs 657 TFLOP/s),
 // slower on BERT-large-384 and BERT-base and +3% on the packed varlen batch.
+bool snake_enabled() {  // B200_FMHA_SNAKE=0 turns the causal snake order off (A/B only)
+  static const bool on = [] {
+    const char* v = std::getenv("B200_FMHA_SNAKE");
+    return !(v && v[0] == '0');
+  }();
+  return on;
+}
+
 bool ks_enabled() {
   static const bool on = [] {
     const char* v = std::getenv("B200_FMHA_KS");
@@ -411,6 +419,9 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   }
   if (items > 2147483647LL || units * prm.num_q_tiles > 2147483647LL) return FMHA_ERR_UNSUPPORTED;
   prm.num_items = static_cast<int>(items);
+  // causal items come longest first with decreasing cost: deal them in snake order (gpt_causal: the
+  // busiest SM 132 -> 126 KV steps for a 124.5 mean); equal-cost items need no snake
+  prm.snake = (kind == FMHA_MASK_CAUSAL && snake_enabled()) ? 1 : 0;
   prm.div_units.init(static_cast<uint32_t>(std::max(prm.num_units, 1)));
   prm.div_pairs.init(static_cast<uint32_t>(std::max((prm.num_q_tiles + 1) / 2, 1)));
   prm.div_qtiles.init(static_cast<uint32_t>(std::max(prm.num_q_tiles, 1)));

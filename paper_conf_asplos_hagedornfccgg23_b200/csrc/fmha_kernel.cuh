@@ -168,6 +168,8 @@ struct FmhaParams {
   uint8_t* o_ptr;             // O base (varlen partial-tile stores)
   int o_row_elems;            // elements between consecutive tokens of O (H * D)
   int sched;                  // 0: item idx = blockIdx.x + k * gridDim.x;  1: cost-sorted (above)
+  int snake;                  // sched 0: odd rounds k visit the CTAs in reverse (idx = (k + 1) G - 1 - c), so
+                              // longest-first items of decreasing cost (causal) balance like LPT
   int num_seqs;               // varlen
   int max_level;              // ceil(max_seqlen / 128) (sched 1: <= SCHED_MAX_LEVELS)
   int seq_q;
@@ -615,7 +617,7 @@ template <bool SCHED>
 __device__ __forceinline__ int item_at(const FmhaParams& p, const SchedTable* tb, int k) {
   const int G = gridDim.x, c = blockIdx.x;
   if constexpr (!SCHED) {
-    const long long idx = c + static_cast<long long>(k) * G;
+    const long long idx = ((k & 1) && p.snake ? G - 1 - c : c) + static_cast<long long>(k) * G;
     return idx < p.num_items ? static_cast<int>(idx) : -1;
   } else {
     const long long pos = static_cast<long long>(k) * G + ((k & 1) ? G - 1 - c : c);
