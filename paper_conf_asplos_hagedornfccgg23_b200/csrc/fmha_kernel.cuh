@@ -706,8 +706,10 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
                  BIAS2D = MODE == MODE_BIAS2D;
   // FMHA_SUMCHECK: the row max is taken over the polynomial columns only once a row has a reference,
   // and the step's sum of p guards the rest (softmax loop, redo_step)
-  constexpr bool SUMCHK = FMHA_SUMCHECK && C::SEP_P && !C::ROT && !C::PREFETCH_S && !C::SPLIT_LD && !C::LSUM_MMA &&
-                          !BIAS && !BIAS2D && !SPLIT && FMHA_ABL == 0 && C::DEFER_ST == 0;
+  // (bit 0: the D = 64 instances, bit 1: D = 128, where P overwrites S in TMEM -- s[] stays in registers)
+  constexpr bool SUMCHK = ((D == 64 && (FMHA_SUMCHECK & 1)) || (D == 128 && (FMHA_SUMCHECK & 2))) && !C::ROT &&
+                          !C::PREFETCH_S && !C::SPLIT_LD && !C::LSUM_MMA && !BIAS && !BIAS2D && !SPLIT && FMHA_ABL == 0 &&
+                          C::DEFER_ST == 0;
   // Dynamic shared memory starts at the (1024-byte aligned) base of the CTA's shared window; the
   // SWIZZLE_128B tiles need that alignment.  Using the base directly keeps smem addresses uniform.
   extern __shared__ __align__(1024) uint8_t smem[];

@@ -35,7 +35,8 @@ sys.path.insert(0, ".")
 import paper_conf_asplos_hagedornfccgg23_b200 as fm  # noqa: E402
 
 for (b, h, s, d, dt, causal) in [(32, 16, 512, 64, torch.float16, False), (32, 16, 384, 64, torch.float16, False),
-                                 (8, 32, 2048, 128, torch.bfloat16, True)]:
+                                 (8, 32, 2048, 128, torch.bfloat16, True), (8, 32, 2048, 128, torch.bfloat16, False),
+                                 (4, 32, 4096, 128, torch.bfloat16, True), (8, 32, 2048, 64, torch.float16, True)]:
     q = torch.randn(b, h, s, d, device=dev, dtype=dt)
     k = torch.randn(b, h, s, d, device=dev, dtype=dt)
     v = torch.randn(b, h, s, d, device=dev, dtype=dt)

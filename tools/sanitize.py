@@ -10,7 +10,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import paper_conf_asplos_hagedornfccgg23_b200 as fm  # noqa: E402
 
 dev = torch.device("cuda:0")
-PART = os.environ.get("SAN_PART", "all")  # all | base | strided | bias2d | rest
+PART = os.environ.get("SAN_PART", "all")  # all | base | strided | bias2d | streamk | rest
 want = lambda part: PART in ("all", part)
 g = torch.Generator(device="cpu").manual_seed(0)
 r = lambda *s, dt=torch.float16: torch.randn(*s, generator=g).to(dt).to(dev)
@@ -38,6 +38,16 @@ for d in (64, 128):
         ab = torch.randn(1, 1, 200, 304, generator=g).to(dt).to(dev)[..., :300]
         if want("bias2d"):
             fm.fmha_fwd(q, k, v, attn_bias=ab)
+        # round 2: the stream-K tail (MODE_DENSE_TAIL / MODE_PAIRX_TAIL): every item of these small
+        # problems is split along the keys, counted with atomics and merged by the last piece through
+        # bulk copies into the idle Q/K/V region; run twice so the counters' reset is exercised
+        if want("streamk"):
+            kl = r(1, 2, 1000, d, dt=dt)
+            for _ in range(2):
+                fm.fmha_fwd_streamk(q, kl, kl)                 # dense pairs (2 q-tiles), 8 KV tiles -> 4 pieces
+                fm.fmha_fwd_streamk(r(1, 3, 384, d, dt=dt), kl.expand(1, 3, 1000, d).contiguous(),
+                                    kl.expand(1, 3, 1000, d).contiguous())  # cross-unit pairs
+                fm.fmha_fwd_streamk(q, kl, kl, causal=True)
 qkv = r(300, 3, 4, 64)
 cu = torch.tensor([0, 100, 100, 300], dtype=torch.int32, device=dev)
 a, w, b = r(300, 136), r(264, 136) * 0.1, r(264)
