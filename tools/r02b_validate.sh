@@ -12,6 +12,7 @@ timeout 300 python bench.py --steps 20 --warmup 5 > gpurun_out/r02b_bench_defaul
 ncu --metrics gpu__time_duration.sum --clock-control none -c 40 --csv --log-file gpurun_out/r02b_bl5_launches.csv python bench.py --steps 5 --warmup 3 --no-cpu-baseline --no-e2e --sustained 0 > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:fmha_fwd_sm100 -s 2 -c 1 -o gpurun_out/r02b_bl5_full python tools/fmha_prof.py bert_large_512 4 > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:fmha_fwd_sm100 -s 2 -c 1 -o gpurun_out/r02b_streamk_full python tools/streamk_prof.py > /dev/null 2>&1
+# (compute-sanitizer is closed on this pool in round 2b; the loop below reports nothing there)
 : > gpurun_out/r02b_sanitizer.txt
 for tool in memcheck racecheck synccheck; do
   for ks in 0 1; do
