@@ -86,6 +86,14 @@ __device__ unsigned int g_fmha_trace_n = 0;
 #ifndef FMHA_SUMCHECK
 #define FMHA_SUMCHECK 0
 #endif
+// FMHA_WARP_STORES: (dense maps) each epilogue warp stores its own 32 rows of O_t with its own TMA store,
+// so the epilogue warps never wait for one another (as GEMM2_WARP_STORES in gemm_kernel.cuh).  Correct
+// (GPU suite passes) but measured -1% on BERT-large-512 / -0.8% on 384, level elsewhere: the epilogue is
+// not on the FMHA's critical path, four stores per tile cost more than the barrier (off;
+// profiles/r02b_ab_fmha_warp_stores.txt)
+#ifndef FMHA_WARP_STORES
+#define FMHA_WARP_STORES 0
+#endif
 #ifndef FMHA_ELECT
 #define FMHA_ELECT 0
 #endif
@@ -159,6 +167,7 @@ struct FmhaParams {
   CUtensorMap tmV;
   CUtensorMap tmO;  // same geometry as Q
   CUtensorMap tmO32;  // O with a 32-row box (key-split kernel: one store per (tile, lane quarter))
+  CUtensorMap tmO32w;  // O with a {64, 32}-element box, SWIZZLE_128B: one epilogue warp's 32 rows (WARP_ST)
   const int32_t* kv_len;
   // Variable-length packed mode (fmha_fwd_varlen): sequence b of the batch is
   // tokens [cu_seqlens[b], cu_seqlens[b+1]) of QKV [T, 3, H, D] / O [T, H, D]; the tensor maps are
@@ -701,6 +710,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
   using XS = ExpShape<D, MODE == MODE_PAIRX || MODE == MODE_PAIRX_TAIL, MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
                       MODE == MODE_BIAS || MODE == MODE_BIAS2D>;
   constexpr bool TAIL = MODE == MODE_DENSE_TAIL || MODE == MODE_PAIRX_TAIL;
+  constexpr bool WARP_ST = FMHA_WARP_STORES && MODE != MODE_VARLEN && MODE != MODE_VARLEN_SCHED;
   constexpr bool PAIRX = MODE == MODE_PAIRX || MODE == MODE_PAIRX_TAIL, VL = MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
                  SCHED = MODE == MODE_VARLEN_SCHED, SPLIT = MODE == MODE_SPLIT, BIAS = MODE == MODE_BIAS,
                  BIAS2D = MODE == MODE_BIAS2D;
@@ -1531,8 +1541,13 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         // sequence's rows, so each thread stores its own row (if inside the sequence) instead
         const bool rowwise = VL && w.row0(t) + 128 > w.len(t);
         const uint32_t stg = sbase + C::OFF_STG + (t % C::NSTG) * C::TILE;
-        if (row == 0) tma_store_wait_read0();  // previous store out of this staging buffer done
-        named_bar_sync(1, 128);
+        if constexpr (WARP_ST) {  // this warp's previous stores have read its rows of the staging buffer
+          if (lane == 0) tma_store_wait_read0();
+          __syncwarp();
+        } else {
+          if (row == 0) tma_store_wait_read0();  // previous store out of this staging buffer done
+          named_bar_sync(1, 128);
+        }
         const uint32_t tO = tmem + lane_off + C::col_o(t);
 #pragma unroll 1
         for (int q = 0; q < D / 32; ++q) {
@@ -1576,7 +1591,17 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           tc_fence_before();
           FMHA_ROW_ARRIVE(BAR(C::B_O_EMPTY + t));
         }
-        if (!rowwise && !SPLIT) {
+        if (WARP_ST && !SPLIT) {
+          fence_proxy_async_smem();
+          __syncwarp();
+          if (lane == 0) {
+#pragma unroll
+            for (int c2 = 0; c2 < D / 64; ++c2)
+              tma_store_4d(&p.tmO32w, stg + c2 * C::CHUNK + quad * 32 * 128, c2 * 64, w.c1(false, t, w.row0(t) + 32 * quad),
+                           w.c2(false, t, w.row0(t)), w.c3(false, t));
+            tma_store_commit();
+          }
+        } else if (!rowwise && !SPLIT) {
           fence_proxy_async_smem();
           named_bar_sync(1, 128);
           if (row == 0) {
@@ -1628,7 +1653,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
               float wt[MAX_TAIL_SPLITS];
               float inv = 0.f;
               const uint32_t stg = sbase + C::OFF_STG + (t % C::NSTG) * C::TILE;
-              if (row == 0) tma_store_wait_read0();
+              if (WARP_ST ? lane == 0 : row == 0) tma_store_wait_read0();  // (every warp's own earlier stores)
 #pragma unroll 1
               for (int hf = 0; hf < D / 64; ++hf) {
                 if (row == 0) {
@@ -1707,7 +1732,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         }
       }
     }
-    if (row == 0) tma_store_wait0();
+    if (WARP_ST ? lane == 0 : row == 0) tma_store_wait0();
   }
 
   tc_fence_before();
