@@ -361,7 +361,6 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   if ((st = map4(&prm.tmV, V, cs.v, seq_kv, 128, 64)) != FMHA_OK) return st;
   if ((st = map4(&prm.tmO, O, cs.o, seq_q, 128, 64)) != FMHA_OK) return st;
   if ((st = map4(&prm.tmO32, O, cs.o, seq_q, 32, 32)) != FMHA_OK) return st;
-  if ((st = map4(&prm.tmO32w, O, cs.o, seq_q, 32, 64)) != FMHA_OK) return st;
   prm.kv_len = (kind == FMHA_MASK_KEY_PADDING) ? mask->kv_len : nullptr;
   prm.cu_seqlens = nullptr;
   prm.seq_q = seq_q;

@@ -86,14 +86,6 @@ __device__ unsigned int g_fmha_trace_n = 0;
 #ifndef FMHA_SUMCHECK
 #define FMHA_SUMCHECK 0
 #endif
-// FMHA_WARP_STORES: (dense maps) each epilogue warp stores its own 32 rows of O_t with its own TMA store,
-// so the epilogue warps never wait for one another (as GEMM2_WARP_STORES in gemm_kernel.cuh).  Correct
-// (GPU suite passes) but measured -1% on BERT-large-512 / -0.8% on 384, level elsewhere: the epilogue is
-// not on the FMHA's critical path, four stores per tile cost more than the barrier (off;
-// profiles/r02b_ab_fmha_warp_stores.txt)
-#ifndef FMHA_WARP_STORES
-#define FMHA_WARP_STORES 0
-#endif
 #ifndef FMHA_ELECT
 #define FMHA_ELECT 0
 #endif
@@ -167,7 +159,6 @@ struct FmhaParams {
   CUtensorMap tmV;
   CUtensorMap tmO;  // same geometry as Q
   CUtensorMap tmO32;  // O with a 32-row box (key-split kernel: one store per (tile, lane quarter))
-  CUtensorMap tmO32w;  // O with a {64, 32}-element box, SWIZZLE_128B: one epilogue warp's 32 rows (WARP_ST)
   const int32_t* kv_len;
   // Variable-length packed mode (fmha_fwd_varlen): sequence b of the batch is
   // tokens [cu_seqlens[b], cu_seqlens[b+1]) of QKV [T, 3, H, D] / O [T, H, D]; the tensor maps are
@@ -236,7 +227,13 @@ struct FmhaCfg {
 #ifndef FMHA_NS64
 #define FMHA_NS64 6
 #endif
-  static constexpr int NS = (D == 64) ? FMHA_NS64 : 3;  // K/V ring slots (K_j, V_j alternate)
+  // D128_RING4: at D = 128 a fourth K/V ring slot (the MMA warp waited ~300 cycles per step for K_{j+1}
+  // with three), paid for by a half-size O staging buffer (one 64-column chunk, stored before the next)
+#ifndef FMHA_D128_RING4
+#define FMHA_D128_RING4 0
+#endif
+  static constexpr bool D128_RING4 = FMHA_D128_RING4 && D == 128;
+  static constexpr int NS = (D == 64) ? FMHA_NS64 : (D128_RING4 ? 4 : 3);  // K/V ring slots (K_j, V_j alternate)
   static constexpr int QS = (D == 64) ? 2 : 1;  // Q stages per tile: the next item's Q loads early
   static constexpr int NSTG = (D == 64) ? 2 : 1;  // O staging buffers (D=128: both tiles share one)
   static constexpr int OFF_Q = 0;               // Q[stage][tile]
@@ -251,7 +248,8 @@ struct FmhaCfg {
 #endif
   static constexpr bool LSUM_MMA = FMHA_LSUM_MMA && D == 64;
   static constexpr int OW = LSUM_MMA ? D + 16 : D;  // O_t columns in TMEM (and PV MMA N)
-  static constexpr int OFF_ONES = OFF_STG + NSTG * TILE;  // LSUM_MMA: 128 x 64 ones (16 KB)
+  static constexpr int STG_CHUNKS = D128_RING4 ? 1 : D / 64;  // 64-column chunks one staging buffer holds
+  static constexpr int OFF_ONES = OFF_STG + NSTG * STG_CHUNKS * CHUNK;  // LSUM_MMA: 128 x 64 ones (16 KB)
   static constexpr int OFF_LSUM = OFF_ONES + (LSUM_MMA ? CHUNK : 0);  // float l[2 tiles][128 rows]
   static constexpr int OFF_MC = OFF_LSUM + 2 * 128 * 4;    // float mc[2 tiles][128 rows] (turn fence)
   static constexpr int OFF_MREF = OFF_MC + 2 * 128 * 4;  // float mc[2 tiles][128 rows] at item end (tail pieces)
@@ -710,7 +708,6 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
   using XS = ExpShape<D, MODE == MODE_PAIRX || MODE == MODE_PAIRX_TAIL, MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
                       MODE == MODE_BIAS || MODE == MODE_BIAS2D>;
   constexpr bool TAIL = MODE == MODE_DENSE_TAIL || MODE == MODE_PAIRX_TAIL;
-  constexpr bool WARP_ST = FMHA_WARP_STORES && MODE != MODE_VARLEN && MODE != MODE_VARLEN_SCHED;
   constexpr bool PAIRX = MODE == MODE_PAIRX || MODE == MODE_PAIRX_TAIL, VL = MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
                  SCHED = MODE == MODE_VARLEN_SCHED, SPLIT = MODE == MODE_SPLIT, BIAS = MODE == MODE_BIAS,
                  BIAS2D = MODE == MODE_BIAS2D;
@@ -1540,14 +1537,9 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         // varlen tile that crosses its sequence's end: a TMA store would overwrite the next
         // sequence's rows, so each thread stores its own row (if inside the sequence) instead
         const bool rowwise = VL && w.row0(t) + 128 > w.len(t);
-        const uint32_t stg = sbase + C::OFF_STG + (t % C::NSTG) * C::TILE;
-        if constexpr (WARP_ST) {  // this warp's previous stores have read its rows of the staging buffer
-          if (lane == 0) tma_store_wait_read0();
-          __syncwarp();
-        } else {
-          if (row == 0) tma_store_wait_read0();  // previous store out of this staging buffer done
-          named_bar_sync(1, 128);
-        }
+        const uint32_t stg = sbase + C::OFF_STG + (t % C::NSTG) * C::STG_CHUNKS * C::CHUNK;
+        if (row == 0) tma_store_wait_read0();  // previous store out of this staging buffer done
+        named_bar_sync(1, 128);
         const uint32_t tO = tmem + lane_off + C::col_o(t);
 #pragma unroll 1
         for (int q = 0; q < D / 32; ++q) {
@@ -1571,7 +1563,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
             }
             continue;
           }
-          const uint32_t box = stg + (col0 / 64) * C::CHUNK + row * 128;
+          const uint32_t box = stg + ((col0 / 64) % C::STG_CHUNKS) * C::CHUNK + row * 128;
 #pragma unroll
           for (int u = 0; u < 4; ++u) {
             const int unit = ((col0 % 64) / 8) + u;
@@ -1586,30 +1578,33 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
               st_global_v4(p.o_ptr + 2 * (tokn * p.o_row_elems + (t ? w.head1 : w.head) * D + col0 + 8 * u), v0, v1, v2, v3);
             }
           }
+          if constexpr (C::STG_CHUNKS < D / 64) {  // half staging: store this 64-column chunk before the next
+            if (!rowwise && (q & 1) && q + 1 < D / 32) {
+              fence_proxy_async_smem();
+              named_bar_sync(1, 128);
+              if (row == 0) {
+                constexpr bool vl = VL;
+                tma_store_4d(&p.tmO, stg, (q / 2) * 64, w.c1(vl, t, w.row0(t)), w.c2(vl, t, w.row0(t)), w.c3(vl, t));
+                tma_store_commit();
+                tma_store_wait_read0();
+              }
+              named_bar_sync(1, 128);
+            }
+          }
         }
         if (n > 0) {  // O_t read: the next item's first PV may overwrite it
           tc_fence_before();
           FMHA_ROW_ARRIVE(BAR(C::B_O_EMPTY + t));
         }
-        if (WARP_ST && !SPLIT) {
-          fence_proxy_async_smem();
-          __syncwarp();
-          if (lane == 0) {
-#pragma unroll
-            for (int c2 = 0; c2 < D / 64; ++c2)
-              tma_store_4d(&p.tmO32w, stg + c2 * C::CHUNK + quad * 32 * 128, c2 * 64, w.c1(false, t, w.row0(t) + 32 * quad),
-                           w.c2(false, t, w.row0(t)), w.c3(false, t));
-            tma_store_commit();
-          }
-        } else if (!rowwise && !SPLIT) {
+        if (!rowwise && !SPLIT) {
           fence_proxy_async_smem();
           named_bar_sync(1, 128);
           if (row == 0) {
             constexpr bool vl = VL;
 #pragma unroll
-            for (int c2 = 0; c2 < D / 64; ++c2)
-              tma_store_4d(&p.tmO, stg + c2 * C::CHUNK, c2 * 64, w.c1(vl, t, w.row0(t)), w.c2(vl, t, w.row0(t)),
-                           w.c3(vl, t));
+            for (int c2 = D / 64 - C::STG_CHUNKS; c2 < D / 64; ++c2)  // (half staging: the last chunk)
+              tma_store_4d(&p.tmO, stg + (c2 % C::STG_CHUNKS) * C::CHUNK, c2 * 64, w.c1(vl, t, w.row0(t)),
+                           w.c2(vl, t, w.row0(t)), w.c3(vl, t));
             tma_store_commit();
           }
         }
@@ -1652,8 +1647,8 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
               const float* src = p.ws_tail + static_cast<size_t>(w.tail * S * 2 + t) * TS;  // split s at + 2 s TS
               float wt[MAX_TAIL_SPLITS];
               float inv = 0.f;
-              const uint32_t stg = sbase + C::OFF_STG + (t % C::NSTG) * C::TILE;
-              if (WARP_ST ? lane == 0 : row == 0) tma_store_wait_read0();  // (every warp's own earlier stores)
+              const uint32_t stg = sbase + C::OFF_STG + (t % C::NSTG) * C::STG_CHUNKS * C::CHUNK;
+              if (row == 0) tma_store_wait_read0();
 #pragma unroll 1
               for (int hf = 0; hf < D / 64; ++hf) {
                 if (row == 0) {
@@ -1707,7 +1702,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
                     }
                   }
                   const int col0 = 64 * hf + 32 * q;
-                  const uint32_t box = stg + (col0 / 64) * C::CHUNK + row * 128;
+                  const uint32_t box = stg + ((col0 / 64) % C::STG_CHUNKS) * C::CHUNK + row * 128;
 #pragma unroll
                   for (int u = 0; u < 4; ++u) {
                     const int unit = ((col0 % 64) / 8) + u;
@@ -1716,23 +1711,34 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
                                  pack2<BF16>(v[8 * u + 6], v[8 * u + 7]));
                   }
                 }
+                if constexpr (C::STG_CHUNKS < D / 64) {  // half staging: store this chunk now
+                  fence_proxy_async_smem();
+                  named_bar_sync(1, 128);  // (also: every thread has read this half's landing zone)
+                  if (row == 0) {
+                    tma_store_4d(&p.tmO, stg, hf * 64, w.c1(false, t, w.row0(t)), w.c2(false, t, w.row0(t)), w.c3(false, t));
+                    tma_store_commit();
+                    tma_store_wait_read0();
+                  }
+                }
                 named_bar_sync(1, 128);  // every thread has read this half's landing zone
               }
-              fence_proxy_async_smem();
-              named_bar_sync(1, 128);
-              if (row == 0) {
+              if constexpr (C::STG_CHUNKS == D / 64) {
+                fence_proxy_async_smem();
+                named_bar_sync(1, 128);
+                if (row == 0) {
 #pragma unroll
-                for (int c2 = 0; c2 < D / 64; ++c2)
-                  tma_store_4d(&p.tmO, stg + c2 * C::CHUNK, c2 * 64, w.c1(false, t, w.row0(t)), w.c2(false, t, w.row0(t)),
-                               w.c3(false, t));
-                tma_store_commit();
+                  for (int c2 = 0; c2 < D / 64; ++c2)
+                    tma_store_4d(&p.tmO, stg + c2 * C::CHUNK, c2 * 64, w.c1(false, t, w.row0(t)), w.c2(false, t, w.row0(t)),
+                                 w.c3(false, t));
+                  tma_store_commit();
+                }
               }
             }
           }
         }
       }
     }
-    if (WARP_ST ? lane == 0 : row == 0) tma_store_wait0();
+    if (row == 0) tma_store_wait0();
   }
 
   tc_fence_before();
