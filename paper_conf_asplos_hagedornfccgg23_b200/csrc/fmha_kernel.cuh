@@ -86,6 +86,16 @@ __device__ unsigned int g_fmha_trace_n = 0;
 #ifndef FMHA_SUMCHECK
 #define FMHA_SUMCHECK 0
 #endif
+// FMHA_PREFETCH_FIRST (default on): the first item's Q and FMHA_PREFETCH_STEPS K/V steps into L2 before
+// griddepcontrol.wait (below).  Measured in one session (profiles/r02c_ab_prefetch_first.txt): BERT-base
+// padded 98.0 -> 105.3 TFLOP/s, BERT-large-384 +2.5%, BERT-large-512 +1.3%, gpt_causal level; the 8-way
+// strong-scaling shard of BERT-large-512 11.75 -> 10.96 us per launch.  1, 2 or 4 steps: level.
+#ifndef FMHA_PREFETCH_FIRST
+#define FMHA_PREFETCH_FIRST 1
+#endif
+#ifndef FMHA_PREFETCH_STEPS
+#define FMHA_PREFETCH_STEPS 2
+#endif
 #ifndef FMHA_ELECT
 #define FMHA_ELECT 0
 #endif
@@ -455,7 +465,7 @@ struct WorkItem {
   }
 };
 
-template <bool PAIRX, bool VL, bool SPLIT = false, bool TAIL = false>
+template <bool PAIRX, bool VL, bool SPLIT = false, bool TAIL = false, bool NOLOAD = false>
 __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
   WorkItem w;
   int qt0;
@@ -526,7 +536,7 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
     w.has0 = w.r0 < w.len0;
     w.has1 = w.has1 && w.r1 < w.len0;
   }
-  if (p.mask_kind == MASK_KEY_PADDING) {
+  if (!NOLOAD && p.mask_kind == MASK_KEY_PADDING) {  // (NOLOAD: no global reads -- before pdl_wait)
     w.kv0 = min(max(__ldg(p.kv_len + w.bat0), 0), p.seq_kv);
     w.kv1 = w.shared ? w.kv0
                      : min(max(__ldg(p.kv_len + p.div_heads.div(min(w.bh1, p.num_units - 1))), 0), p.seq_kv);
@@ -776,6 +786,33 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     tmem_relinquish();
   }
   // PDL: the setup above overlaps the previous kernel's tail; global memory only from here on
+  // FMHA_PREFETCH_FIRST: while the previous kernel on the stream drains (PDL), the TMA warp prefetches its
+  // CTA's first item's Q and first two K/V steps into L2.  A prefetch reads no data into the CTA and
+  // writes nothing, so it is safe before griddepcontrol.wait; the item is decoded without the kv_len
+  // read (which may be the previous kernel's output).
+  if constexpr (FMHA_PREFETCH_FIRST && !VL) {
+    if (warp == C::W_TMA) {
+      const int idx0 = blockIdx.x;
+      if (idx0 < p.num_items) {
+        const WorkItem w = decode_item<PAIRX, false, SPLIT, TAIL, true>(p, idx0);
+#pragma unroll
+        for (int t = 0; t < 2; ++t) {
+          if (w.n(t) == 0) continue;
+#pragma unroll
+          for (int c = 0; c < D / 64; ++c)
+            tma_prefetch_l2_4d_elect(&p.tmQ, c * 64, w.c1(false, t, w.row0(t)), w.c2(false, t, w.row0(t)), w.c3(false, t));
+          if (t == 1 && w.shared) continue;
+          for (int j = 0; j < min(w.n(t), FMHA_PREFETCH_STEPS); ++j)
+#pragma unroll
+            for (int c = 0; c < D / 64; ++c) {
+              const int r = (w.jb + j) * 128;
+              tma_prefetch_l2_4d_elect(&p.tmK, c * 64, w.c1(false, t, r), w.c2(false, t, r), w.c3(false, t));
+              tma_prefetch_l2_4d_elect(&p.tmV, c * 64, w.c1(false, t, r), w.c2(false, t, r), w.c3(false, t));
+            }
+        }
+      }
+    }
+  }
   pdl_wait();
   pdl_trigger();
   const SchedTable* sched = reinterpret_cast<const SchedTable*>(smem + C::OFF_SCHED);

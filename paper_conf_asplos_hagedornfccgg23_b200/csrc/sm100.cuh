@@ -299,6 +299,17 @@ __device__ __forceinline__ void tma_load_4d_hint_elect(uint32_t dst, const CUten
       : "memory");
 }
 
+// L2 prefetch of one 4-D tensor tile (no shared memory, no barrier), issued by one elected lane.
+__device__ __forceinline__ void tma_prefetch_l2_4d_elect(const CUtensorMap* m, int c0, int c1, int c2, int c3) {
+  asm volatile(
+      "{\n\t.reg .pred e;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "@e cp.async.bulk.prefetch.tensor.4d.L2.global.tile [%0, {%1, %2, %3, %4}];\n\t}" ::"l"(
+          reinterpret_cast<uint64_t>(m)),
+      "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+      : "memory");
+}
+
 // ------------------------------------------------------------------ CTA pair (cta_group::2)
 __device__ __forceinline__ uint32_t cluster_ctarank() {
   uint32_t r;
