@@ -343,6 +343,13 @@ __global__ void __launch_bounds__(384, 1) gemm_bias_act_kernel(const __grid_cons
 //   EMPTY[s]     both CTAs, count 1: the leader's MMA commit is multicast to both
 //   ACC_FULL[b]  both CTAs, count 1: multicast commit after a tile's last MMA
 //   ACC_EMPTY[b] leader only, count 16: one arrival per epilogue warp of either CTA (remote for r = 1)
+// GEMM2_PREFETCH_FIRST: the FMHA's first-item L2 prefetch applied to the CTA-pair GEMM (first tile's first
+// STAGES K blocks of A and W before griddepcontrol.wait): measured level to -0.5% on the MLP block, BERT
+// layer and LSTM cell (profiles/r02c_ab_gemm_prefetch_first.txt; ~100 us launches have little fill to
+// hide), so off
+#ifndef GEMM2_PREFETCH_FIRST
+#define GEMM2_PREFETCH_FIRST 0
+#endif
 // GEMM2_WARP_STORES: each epilogue warp writes its 32 rows to the staging buffer and stores them with
 // its own TMA store (box 64 x 32), so the four warps of a column group never wait for one another
 // (the group's two named barriers per tile were the top stall of the GELU GEMM, 2.3 warps per issue
@@ -406,6 +413,16 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1) gemm_bias_ac
     tma_prefetch_desc(&p.tmC);
   }
   if (warp == 1) tmem_alloc_2sm(smem_u32(tmem_holder), 512);
+  // GEMM2_PREFETCH_FIRST: this CTA's first tile's first STAGES K blocks of A and W into L2 while the previous
+  // kernel drains (a prefetch writes nothing, so it is safe before griddepcontrol.wait; as the FMHA)
+  if (GEMM2_PREFETCH_FIRST && warp == 0 && lane == 0 && cid < num_tiles) {
+    const GemmUnit gu = gemm_unit2(p, cid);
+    const bool half = gu.width == 128;
+    for (int kb = 0; kb < min(nk1, C::STAGES); ++kb) {
+      tma_prefetch_l2_3d(&p.tmA[0], kb * C::BK, gu.m0 + 128 * static_cast<int>(rank), 0);
+      tma_prefetch_l2_3d(&p.tmW[0][half ? 2 : 1], kb * C::BK, gu.n0 + (half ? 64 : 128) * static_cast<int>(rank), 0);
+    }
+  }
   tc_fence_before();
   cluster_sync_all();  // both CTAs' barriers initialised and TMEM allocated before any signal crosses
   tc_fence_after();
