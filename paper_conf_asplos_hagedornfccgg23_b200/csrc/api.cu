@@ -190,7 +190,12 @@ int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) 
   // persistent: one CTA per SM (or fewer when there is less work)
   dim3 grid(static_cast<unsigned>(std::min(prm.num_items, sm_count)), 1, 1);
   // PDL measured: +0.5% (BERT-large-512) to +4.5% (BERT-base, padded); -5% on the varlen schedule
-  const bool pdl = mode != b200::MODE_VARLEN && mode != b200::MODE_VARLEN_SCHED;
+  // (B200_VARLEN_PDL=1 turns it on for varlen too, A/B only)
+  static const bool varlen_pdl = [] {
+    const char* v = std::getenv("B200_VARLEN_PDL");
+    return v && v[0] == '1';
+  }();
+  const bool pdl = varlen_pdl || (mode != b200::MODE_VARLEN && mode != b200::MODE_VARLEN_SCHED);
   cudaError_t e = b200::launch_pdl(pdl, kern, grid, dim3(C::THREADS), C::SMEM_ALLOC, stream, prm);
   if (e != cudaSuccess) return cuda_fail(e, "fmha_fwd_kernel launch");
   if (mode == b200::MODE_SPLIT) {  // merge the splits into O (same stream, so after the kernel)
