@@ -45,8 +45,8 @@ for d in (64, 128):
             kl = r(1, 2, 1000, d, dt=dt)
             for _ in range(2):
                 fm.fmha_fwd_streamk(q, kl, kl)                 # dense pairs (2 q-tiles), 8 KV tiles -> 4 pieces
-                fm.fmha_fwd_streamk(r(1, 3, 384, d, dt=dt), kl.expand(1, 3, 1000, d).contiguous(),
-                                    kl.expand(1, 3, 1000, d).contiguous())  # cross-unit pairs
+                k3 = torch.cat([kl, kl[:, :1]], dim=1)      # 3 heads
+                fm.fmha_fwd_streamk(r(1, 3, 384, d, dt=dt), k3, k3)  # cross-unit pairs
                 fm.fmha_fwd_streamk(q, kl, kl, causal=True)
 qkv = r(300, 3, 4, 64)
 cu = torch.tensor([0, 100, 100, 300], dtype=torch.int32, device=dev)
