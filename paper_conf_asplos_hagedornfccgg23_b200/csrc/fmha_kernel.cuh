@@ -322,7 +322,12 @@ struct FmhaCfg {
 #ifndef FMHA_TURNS
 #define FMHA_TURNS 1
 #endif
-  static constexpr bool TURNS = FMHA_TURNS;
+// (FMHA_TURNS128=0, D = 128 without turns: gpt_causal 871 -> 837 TFLOP/s, 8x32x2048 non-causal 1047 -> 890;
+// profiles/r02c_ab_d128_noturns.txt)
+#ifndef FMHA_TURNS128
+#define FMHA_TURNS128 FMHA_TURNS
+#endif
+  static constexpr bool TURNS = (D == 128) ? FMHA_TURNS128 : FMHA_TURNS;
   // Split S load: max of the first 64 columns overlaps the TMEM load of the last 64 (A/B knob)
 #ifndef FMHA_SPLIT_LD
 #define FMHA_SPLIT_LD 0
