@@ -190,11 +190,14 @@ _STREAMK_WS: dict = {}
 
 
 def streamk_workspace(device: torch.device, head_dim: int) -> torch.Tensor:
-    """The zero-filled workspace of fmha_fwd_streamk for `device` (cached: every launch leaves it
-    zero-filled again, so one buffer per device serves all launches on one stream)."""
+    """The zero-filled workspace of fmha_fwd_streamk for `device` and its current stream (cached per
+    (device, head_dim, stream): every launch leaves it zero-filled again, so one buffer serves all
+    launches on one stream; launches on different streams get different buffers, since two concurrent
+    launches must not share the per-item counters)."""
     lib = _lib.load()
     device = torch.device(device)
-    key = (device.index if device.index is not None else torch.cuda.current_device(), head_dim)
+    dev_index = device.index if device.index is not None else torch.cuda.current_device()
+    key = (dev_index, head_dim, torch.cuda.current_stream(dev_index).cuda_stream)
     ws = _STREAMK_WS.get(key)
     if ws is None:
         with torch.cuda.device(device):
