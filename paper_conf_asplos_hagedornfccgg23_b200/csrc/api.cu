@@ -238,13 +238,22 @@ int splitkv_default(long long units, int seq_q, int seq_kv, int sms) {
 }
 
 // Work items of the dense schedule and its pairing mode: (unit, q-tile pair) items, or (pair_mode 1)
-// pairs of the flattened (unit, q-tile) list when a unit has an odd number (>= 3) of q-tiles and the
-// mask is not causal / a bias (BERT-large-384: no half-empty items, +8%).  With a single q-tile per
-// unit (short sequences) every item is one latency-bound step and pairing across units measured
-// slower, so those keep pair_mode 0.
-long long dense_items(long long units, int num_q_tiles, int kind, int* pair_mode) {
-  *pair_mode = (kind != FMHA_MASK_CAUSAL && kind != FMHA_MASK_KEY_BIAS && kind != FMHA_MASK_ATTN_BIAS &&
-                (num_q_tiles & 1) && num_q_tiles >= 3) ? 1 : 0;
+// pairs of the flattened (unit, q-tile) list when a unit has an odd number of q-tiles (>= 3, or 1 with
+// more units than SMs) and the mask is not causal / a bias (BERT-large-384: no half-empty items, +8%).
+long long dense_items(long long units, int num_q_tiles, int kind, int sms, int* pair_mode, long long decide_units = -1) {
+  // Single-q-tile units (seq_q <= 128) are paired too once they fill more than one round unpaired (one
+  // round of pair steps is shorter than two of single-tile steps); with fewer units than SMs pairing
+  // would halve the busy SMs.  Measured on BERT-base padded (384 units): 105 -> 117 TFLOP/s
+  // (profiles/r02c_ab_pair1.txt).  B200_FMHA_PAIR1=0 restores round 1's rule (A/B only).
+  static const bool pair1 = [] {
+    const char* v = std::getenv("B200_FMHA_PAIR1");
+    return !(v && v[0] == '0');
+  }();
+  // (decide_units: the whole problem's units when this launch is one batch chunk of it, so every chunk of
+  // fmha_fwd_from_host takes the same decision and the results stay bitwise those of fmha_fwd)
+  const long long du = decide_units >= 0 ? decide_units : units;
+  const bool odd = (num_q_tiles & 1) && (num_q_tiles >= 3 || (pair1 && num_q_tiles == 1 && du > sms));
+  *pair_mode = (kind != FMHA_MASK_CAUSAL && kind != FMHA_MASK_KEY_BIAS && kind != FMHA_MASK_ATTN_BIAS && odd) ? 1 : 0;
   return *pair_mode ? (units * num_q_tiles + 1) / 2 : units * ((num_q_tiles + 1) / 2);
 }
 
@@ -326,7 +335,7 @@ int validate_shape(int batch, int heads, int seq_q, int seq_kv, int head_dim, fl
 int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O, const fmha_mask_t* mask,
                 int batch, int heads, int seq_q, int seq_kv, int head_dim, float scale, cudaStream_t stream,
                 int splits = 1, void* workspace = nullptr, size_t workspace_bytes = 0,
-                const fmha_strides_t* strides = nullptr, bool streamk = false) {
+                const fmha_strides_t* strides = nullptr, bool streamk = false, long long decide_units = -1) {
   g_last_cuda_error[0] = 0;
   bool empty = false;
   if (int vs = validate_shape(batch, heads, seq_q, seq_kv, head_dim, scale, mask, splits, &empty); vs != FMHA_OK || empty)
@@ -378,7 +387,7 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
   // scores (-inf) still map to exp2(-inf) = 0 instead of -inf * 0 = NaN.  1e-30 perturbs visible
   // scores by < 1e-25 in the exponent.
   prm.scale_log2 = std::max(scale * 1.4426950408889634f, 1e-30f);
-  long long items = dense_items(units, prm.num_q_tiles, kind, &prm.pair_mode);
+  long long items = dense_items(units, prm.num_q_tiles, kind, sm_count, &prm.pair_mode, decide_units);
   if (kind == FMHA_MASK_KEY_BIAS) {
     prm.key_bias = mask->key_bias;
     prm.key_bias_stride = mask->key_bias_stride;
@@ -726,7 +735,7 @@ int fmha_fwd_from_host(int dtype, const void* hQ, const void* hK, const void* hV
     fmha_mask_t cm = dmask;
     if (cm.kv_len) cm.kv_len = dL + b0;
     st = fmha_common(dtype == 1, dQ + oq, dK + okv, dV + okv, dO + oq, &cm, nb, heads, seq_q, seq_kv, head_dim, scale,
-                     sc);
+                     sc, 1, nullptr, 0, nullptr, false, static_cast<long long>(batch) * heads);
     if (st != FMHA_OK) break;
     if ((e = cudaEventRecord(ev_c[c], sc)) != cudaSuccess || (e = cudaStreamWaitEvent(sd, ev_c[c], 0)) != cudaSuccess ||
         (e = cudaMemcpyAsync(static_cast<uint8_t*>(hO) + oq, dO + oq, nb * qb1, cudaMemcpyDeviceToHost, sd)) !=
@@ -804,7 +813,7 @@ int fmha_streamk_plan(int batch, int heads, int seq_q, int seq_kv, int mask_kind
   int pair_mode = 0;
   const long long units = static_cast<long long>(batch) * heads;
   const int nq = (seq_q + 127) / 128;
-  const long long items = dense_items(units, nq, mask_kind, &pair_mode);
+  const long long items = dense_items(units, nq, mask_kind, sm_count, &pair_mode);
   long long rest = 0;
   const int s = streamk_plan(items, (seq_kv + 127) / 128, sm_count, singles_tail(items, units * nq, pair_mode, sm_count),
                              &rest);

@@ -15,18 +15,23 @@ from paper_conf_asplos_hagedornfccgg23_b200 import _lib
 MASK_NONE, MASK_KEY_PADDING, MASK_CAUSAL, MASK_KEY_BIAS, MASK_ATTN_BIAS = 0, 1, 2, 3, 4
 
 
+def pairs_across_units(b, h, nq, mask, sms):
+    """fmha_fwd's pair_mode 1: odd q-tile counts >= 3, or 1 with more units than SMs."""
+    return mask != MASK_CAUSAL and nq % 2 == 1 and (nq >= 3 or (nq == 1 and b * h > sms))
+
+
 def singles(b, h, sq, items, mask, sms):
     nq = math.ceil(sq / 128)
-    pair = mask != MASK_CAUSAL and nq % 2 == 1 and nq >= 3
+    pair = pairs_across_units(b, h, nq, mask, sms)
     full = items // sms * sms
     rest_tiles = b * h * nq - 2 * full
     return pair and full > 0 and 0 < rest_tiles <= sms
 
 
-def items_of(b, h, sq, mask):
-    """fmha_fwd's two-tile items: cross-unit pairs for odd q-tile counts >= 3 (non-causal)."""
+def items_of(b, h, sq, mask, sms):
+    """fmha_fwd's two-tile items: cross-unit pairs in pair_mode 1, else per-unit pairs."""
     nq = math.ceil(sq / 128)
-    if mask != MASK_CAUSAL and nq % 2 == 1 and nq >= 3:
+    if pairs_across_units(b, h, nq, mask, sms):
         return (b * h * nq + 1) // 2
     return b * h * ((nq + 1) // 2)
 
@@ -66,7 +71,7 @@ def test_plan_invariants(seed):
         mask = int(rng.choice([MASK_NONE, MASK_KEY_PADDING, MASK_CAUSAL]))
         sms = int(rng.choice([8, 132, 148]))
         s, tail = fm.streamk_plan(b, h, sq, skv, sms, mask)
-        items = items_of(b, h, sq, mask)
+        items = items_of(b, h, sq, mask, sms)
         nkv = math.ceil(skv / 128)
         if s == 1:
             assert tail == 0
