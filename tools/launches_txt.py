@@ -19,5 +19,9 @@ for r in rows[1:]:
         if k in r[iname]:
             ours[k] += t
     print(f"{r[ik]:>3} {t:10.3f} us  grid {r[ig]:>14} block {r[ib]:>14}  {r[iname][:110]}")
+spin = sum(float(r[iv].replace(",", "")) * {"ns": 1e-3, "nsecond": 1e-3, "us": 1.0, "usecond": 1.0, "ms": 1e3,
+                                             "msecond": 1e3}[r[iu]] for r in rows[1:] if "spin_kernel" in r[iname])
 for k in keys:
-    print(f"# {k} share of listed device time: {100 * ours[k] / tot:.1f}%")
+    print(f"# {k} share of listed device time: {100 * ours[k] / tot:.1f}%"
+          + (f"; {100 * ours[k] / (tot - spin):.1f}% without bench.lead_in's spin_kernel (run before each timed"
+             f" region, outside it)" if spin > 0 else ""))
