@@ -134,6 +134,14 @@ bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) ==
 // dense, cross-unit pair and varlen modes, selected with B200_FMHA_KS=1.  Off by default: measured
 // against the two-tile kernel on the same boxes it is level on BERT-large-512 (640 vs 657 TFLOP/s),
 // slower on BERT-large-384 and BERT-base and +3% on the packed varlen batch.
+bool split_pair_enabled() {  // B200_SPLIT_PAIR=0 turns split pairing off (A/B only)
+  static const bool on = [] {
+    const char* v = std::getenv("B200_SPLIT_PAIR");
+    return !(v && v[0] == '0');
+  }();
+  return on;
+}
+
 bool snake_enabled() {  // B200_FMHA_SNAKE=0 turns the causal snake order off (A/B only)
   static const bool on = [] {
     const char* v = std::getenv("B200_FMHA_SNAKE");
@@ -169,7 +177,7 @@ int launch_fmha_ks(const b200::FmhaParams& prm, int mode, int sm_count, cudaStre
 template <int D, bool BF16>
 int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) {
   using C = b200::FmhaCfg<D>;
-  const int mode = prm.num_splits > 1 ? b200::MODE_SPLIT
+  const int mode = prm.num_splits > 1 ? (prm.split_pair ? b200::MODE_SPLIT_PAIR : b200::MODE_SPLIT)
                    : prm.tail_splits > 1 ? (prm.pair_mode ? b200::MODE_PAIRX_TAIL : b200::MODE_DENSE_TAIL)
                    : prm.attn_bias  ? b200::MODE_BIAS2D
                    : prm.key_bias   ? b200::MODE_BIAS
@@ -179,6 +187,7 @@ int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) 
                                    : mode == b200::MODE_PAIRX  ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_PAIRX>
                                    : mode == b200::MODE_VARLEN ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_VARLEN>
                                    : mode == b200::MODE_SPLIT  ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_SPLIT>
+                                   : mode == b200::MODE_SPLIT_PAIR ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_SPLIT_PAIR>
                                    : mode == b200::MODE_BIAS   ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_BIAS>
                                    : mode == b200::MODE_BIAS2D ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_BIAS2D>
                                    : mode == b200::MODE_DENSE_TAIL ? b200::fmha_fwd_sm100<D, BF16, b200::MODE_DENSE_TAIL>
@@ -198,7 +207,7 @@ int launch_fmha(const b200::FmhaParams& prm, int sm_count, cudaStream_t stream) 
   const bool pdl = varlen_pdl || (mode != b200::MODE_VARLEN && mode != b200::MODE_VARLEN_SCHED);
   cudaError_t e = b200::launch_pdl(pdl, kern, grid, dim3(C::THREADS), C::SMEM_ALLOC, stream, prm);
   if (e != cudaSuccess) return cuda_fail(e, "fmha_fwd_kernel launch");
-  if (mode == b200::MODE_SPLIT) {  // merge the splits into O (same stream, so after the kernel)
+  if (mode == b200::MODE_SPLIT || mode == b200::MODE_SPLIT_PAIR) {  // merge the splits into O (same stream, after the kernel)
     const long long rows = static_cast<long long>(prm.num_units) * prm.seq_q;
     const long long blocks = (rows * 32 + 255) / 256;
     b200::fmha_splitkv_combine_kernel<D, BF16><<<static_cast<unsigned>(blocks), 256, 0, stream>>>(
@@ -220,6 +229,7 @@ size_t splitkv_ws_bytes(long long units, int seq_q, int head_dim, int splits) {
 // already fills the SMs.
 int splitkv_default(long long units, int seq_q, int seq_kv, int sms) {
   const long long items = units * (((seq_q + 127) / 128 + 1) / 2);  // (unit, q-tile pair) items
+  const bool pair = (seq_q + 127) / 128 == 1 && split_pair_enabled();  // two splits per item (split_pair)
   const int nkv = (seq_kv + 127) / 128;
   if (items <= 0 || items >= sms || nkv <= 1) return 1;
   int best_s = 1;
@@ -227,7 +237,7 @@ int splitkv_default(long long units, int seq_q, int seq_kv, int sms) {
   for (int s = 1; s <= std::min(nkv, 64); ++s) {
     const int per = (nkv + s - 1) / s;
     if ((nkv + per - 1) / per != s) continue;  // s not reachable with whole tiles per split
-    const long long rounds = (items * s + sms - 1) / sms;
+    const long long rounds = ((pair ? items * ((s + 1) / 2) : items * s) + sms - 1) / sms;
     const long long cost = rounds * (per + 2);
     if (best < 0 || cost < best) {
       best = cost;
@@ -453,10 +463,14 @@ int fmha_common(bool bf16, const void* Q, const void* K, const void* V, void* O,
     prm.num_splits = splits;
     prm.split_tiles = (nkv + splits - 1) / splits;
     prm.pair_mode = 0;  // (pairs of one unit's q-tiles; the split index is the fastest item digit)
-    const long long items = units * ((prm.num_q_tiles + 1) / 2) * splits;
+    // one q-tile per unit: pair consecutive splits of the unit in one item (tile 1 = the same rows, the
+    // next key range), so the second softmax warpgroup is not idle (decode_splitkv: 4 -> 8 splits)
+    prm.split_pair = (prm.num_q_tiles == 1 && split_pair_enabled()) ? 1 : 0;
+    const int per_item = prm.split_pair ? (splits + 1) / 2 : splits;
+    const long long items = units * ((prm.num_q_tiles + 1) / 2) * per_item;
     if (items > 2147483647LL) return FMHA_ERR_UNSUPPORTED;
     prm.num_items = static_cast<int>(items);
-    prm.div_splits.init(static_cast<uint32_t>(splits));
+    prm.div_splits.init(static_cast<uint32_t>(per_item));
     float* ws = static_cast<float*>(workspace);
     const size_t rows = static_cast<size_t>(units) * seq_q;
     prm.ws_o = ws;

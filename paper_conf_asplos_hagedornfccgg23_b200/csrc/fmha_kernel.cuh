@@ -200,7 +200,11 @@ struct FmhaParams {
   // its unnormalised partial O (fp32), its exp2 reference mc = scale*log2e*m and its row sum l to
   // the workspace; fmha_splitkv_combine_kernel merges the splits.
   int num_splits, split_tiles;
-  FastDiv div_splits;
+  FastDiv div_splits;  // ceil(num_splits / 2) with split_pair, else num_splits
+  // split_pair (units with one q-tile; the MODE_SPLIT_PAIR instance): an item's tile 1 is the same q-tile
+  // as tile 0 with the NEXT split's key range (its own K/V stream), so both softmax warpgroups work and the
+  // items halve
+  int split_pair;
   float* ws_o;   // [num_splits][num_units][seq_q][D]
   float* ws_m;   // [num_splits][num_units][seq_q]
   float* ws_l;   // [num_splits][num_units][seq_q]
@@ -449,6 +453,9 @@ struct WorkItem {
   int bat0, bat1;   // dense: b of unit bh0 / bh1
   int jb;          // split-KV: first KV tile of this item's range (0 otherwise)
   int split;       // split-KV: split index
+  int jb1, split1; // the same for tile 1 (differ from tile 0's only with split pairing, FmhaParams::split_pair)
+  __device__ __forceinline__ int jbt(int t) const { return t ? jb1 : jb; }
+  __device__ __forceinline__ int splt(int t) const { return t ? split1 : split; }
   int tail;        // stream-K tail piece: its tail item r (-1: a whole item)
   // 4-D TMA coordinates (c1, c2, c3) of the block starting at row r of tile t (c0 = d):
   // dense maps are {D, rows, heads, batch}, varlen maps {D, heads, tokens, 1}
@@ -470,12 +477,13 @@ struct WorkItem {
   }
 };
 
-template <bool PAIRX, bool VL, bool SPLIT = false, bool TAIL = false, bool NOLOAD = false>
+// SPLIT: 0 none, 1 split-KV, 2 split-KV with split pairing (MODE_SPLIT_PAIR)
+template <bool PAIRX, bool VL, int SPLIT = 0, bool TAIL = false, bool NOLOAD = false>
 __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
   WorkItem w;
   int qt0;
-  w.jb = 0;
-  w.split = 0;
+  w.jb = w.jb1 = 0;
+  w.split = w.split1 = 0;
   w.tail = -1;
   if constexpr (TAIL) {
     if (idx >= p.tail_from) {  // piece (tail item r, split) of item tail_from + r
@@ -486,9 +494,11 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
       idx = p.tail_from + r;
     }
   }
-  if constexpr (SPLIT) {
+  if constexpr (SPLIT != 0) {
+    const int ns = SPLIT == 2 ? (p.num_splits + 1) >> 1 : p.num_splits;  // items per (unit, q-tile pair)
     const int rest = p.div_splits.div(idx);
-    w.split = idx - rest * p.num_splits;
+    const int sp = idx - rest * ns;
+    w.split = SPLIT == 2 ? 2 * sp : sp;
     idx = rest;
   }
   if (!PAIRX) {
@@ -523,6 +533,14 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
     w.r0 = qt0 * 128;
     w.r1 = qt1 * 128;
   }
+  if constexpr (SPLIT == 2) {
+    {  // tile 1: the same q-tile (one per unit), the next split's key range
+      w.has1 = w.split + 1 < p.num_splits;
+      w.bh1 = w.bh0;
+      w.r1 = w.r0;
+      w.shared = false;
+    }
+  }
   w.has0 = true;
   w.kv0 = w.kv1 = p.seq_kv;
   w.tok0 = w.tok1 = 0;
@@ -554,14 +572,17 @@ __device__ __forceinline__ WorkItem decode_item(const FmhaParams& p, int idx) {
   }
   w.n0 = w.has0 ? (kv_end0 + 127) / 128 : 0;
   w.n1 = w.has1 ? (kv_end1 + 127) / 128 : 0;
-  if constexpr (SPLIT) {  // this split's KV tiles [jb, jb + split_tiles) of each tile's range
+  if constexpr (SPLIT != 0) {  // this split's KV tiles [jb, jb + split_tiles) of each tile's range
     w.jb = w.split * p.split_tiles;
+    w.split1 = SPLIT == 2 ? w.split + 1 : w.split;
+    w.jb1 = SPLIT == 2 ? w.split1 * p.split_tiles : w.jb;
     w.n0 = min(max(w.n0 - w.jb, 0), p.split_tiles);
-    w.n1 = min(max(w.n1 - w.jb, 0), p.split_tiles);
+    w.n1 = min(max(w.n1 - w.jb1, 0), p.split_tiles);
   }
   if constexpr (TAIL) {  // a tail piece: its split's KV tiles [jb, jb + tail_tiles)
     if (w.tail >= 0) {
-      w.jb = w.split * p.tail_tiles;
+      w.jb = w.jb1 = w.split * p.tail_tiles;
+      w.split1 = w.split;
       w.n0 = min(max(w.n0 - w.jb, 0), p.tail_tiles);
       w.n1 = min(max(w.n1 - w.jb, 0), p.tail_tiles);
     }
@@ -657,8 +678,8 @@ __device__ __forceinline__ WorkItem sched_item(const FmhaParams& p, const SchedT
   const int r = pos - tb->items_end[l + 1];
   const int H = p.heads, nl = tb->seq_count[l] * H, full = nl * (l >> 1);
   WorkItem w;
-  w.jb = 0;
-  w.split = 0;
+  w.jb = w.jb1 = 0;
+  w.split = w.split1 = 0;
   w.tail = -1;
   w.has0 = true;
   int si0, h0, si1, h1;
@@ -702,7 +723,7 @@ __device__ __forceinline__ WorkItem sched_item(const FmhaParams& p, const SchedT
 }
 
 // decode_item, or sched_item in sched mode
-template <bool PAIRX, bool VL, bool SPLIT, bool SCHED, bool TAIL = false>
+template <bool PAIRX, bool VL, int SPLIT, bool SCHED, bool TAIL = false>
 __device__ __forceinline__ WorkItem get_item(const FmhaParams& p, const SchedTable* tb, int idx) {
   if constexpr (SCHED) {
     return sched_item(p, tb, idx);
@@ -715,7 +736,7 @@ __device__ __forceinline__ WorkItem get_item(const FmhaParams& p, const SchedTab
 // FmhaParams::pair_mode); varlen packed; varlen packed with the cost-sorted schedule.  Separate
 // instances keep the varlen and scheduling code out of the dense kernels entirely.
 enum : int { MODE_DENSE = 0, MODE_PAIRX = 1, MODE_VARLEN = 2, MODE_VARLEN_SCHED = 3, MODE_SPLIT = 4, MODE_BIAS = 5,
-             MODE_BIAS2D = 6, MODE_DENSE_TAIL = 7, MODE_PAIRX_TAIL = 8 };
+             MODE_BIAS2D = 6, MODE_DENSE_TAIL = 7, MODE_PAIRX_TAIL = 8, MODE_SPLIT_PAIR = 9 };
 
 template <int D, bool BF16, int MODE>
 __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__ FmhaParams p) {
@@ -723,8 +744,9 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
   using XS = ExpShape<D, MODE == MODE_PAIRX || MODE == MODE_PAIRX_TAIL, MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
                       MODE == MODE_BIAS || MODE == MODE_BIAS2D>;
   constexpr bool TAIL = MODE == MODE_DENSE_TAIL || MODE == MODE_PAIRX_TAIL;
+  constexpr int SPLIT_KIND = MODE == MODE_SPLIT_PAIR ? 2 : MODE == MODE_SPLIT ? 1 : 0;
   constexpr bool PAIRX = MODE == MODE_PAIRX || MODE == MODE_PAIRX_TAIL, VL = MODE == MODE_VARLEN || MODE == MODE_VARLEN_SCHED,
-                 SCHED = MODE == MODE_VARLEN_SCHED, SPLIT = MODE == MODE_SPLIT, BIAS = MODE == MODE_BIAS,
+                 SCHED = MODE == MODE_VARLEN_SCHED, SPLIT = MODE == MODE_SPLIT || MODE == MODE_SPLIT_PAIR, BIAS = MODE == MODE_BIAS,
                  BIAS2D = MODE == MODE_BIAS2D;
   // FMHA_SUMCHECK: the row max is taken over the polynomial columns only once a row has a reference,
   // and the step's sum of p guards the rest (softmax loop, redo_step)
@@ -799,7 +821,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     if (warp == C::W_TMA) {
       const int idx0 = blockIdx.x;
       if (idx0 < p.num_items) {
-        const WorkItem w = decode_item<PAIRX, false, SPLIT, TAIL, true>(p, idx0);
+        const WorkItem w = decode_item<PAIRX, false, SPLIT_KIND, TAIL, true>(p, idx0);
 #pragma unroll
         for (int t = 0; t < 2; ++t) {
           if (w.n(t) == 0) continue;
@@ -810,7 +832,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           for (int j = 0; j < min(w.n(t), FMHA_PREFETCH_STEPS); ++j)
 #pragma unroll
             for (int c = 0; c < D / 64; ++c) {
-              const int r = (w.jb + j) * 128;
+              const int r = (w.jbt(t) + j) * 128;
               tma_prefetch_l2_4d_elect(&p.tmK, c * 64, w.c1(false, t, r), w.c2(false, t, r), w.c3(false, t));
               tma_prefetch_l2_4d_elect(&p.tmV, c * 64, w.c1(false, t, r), w.c2(false, t, r), w.c3(false, t));
             }
@@ -851,11 +873,11 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
                                      keep);
             else
               tma_load_4d_hint_elect(sbase + C::OFF_RING + s * C::TILE + c * C::CHUNK, map, KV_FULL(s), c * 64,
-                                     w.c1(vl, t, (w.jb + j) * 128), w.c2(vl, t, (w.jb + j) * 128), w.c3(vl, t), keep);
+                                     w.c1(vl, t, (w.jbt(t) + j) * 128), w.c2(vl, t, (w.jbt(t) + j) * 128), w.c3(vl, t), keep);
         }
       };
       for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
-        const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED, TAIL>(p, sched, idx);
+        const WorkItem w = get_item<PAIRX, VL, SPLIT_KIND, SCHED, TAIL>(p, sched, idx);
         const int N = max(w.n0, w.n1);
 #pragma unroll
         for (int t = 0; t < 2; ++t) {
@@ -922,7 +944,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       auto seek = [&](Cursor& cu, int k, uint32_t base) {
         cu.valid = false;
         for (int idx; (idx = item_at<SCHED>(p, sched, k)) >= 0; ++k) {
-          const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED, TAIL>(p, sched, idx);
+          const WorkItem w = get_item<PAIRX, VL, SPLIT_KIND, SCHED, TAIL>(p, sched, idx);
           const int N = max(w.n0, w.n1);
           if (N == 0) continue;
           cu.w.n0 = w.n0;
@@ -1087,7 +1109,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     uint32_t g = 0, lc = 0;
     PROF_DECL
     for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
-      const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED, TAIL>(p, sched, idx);
+      const WorkItem w = get_item<PAIRX, VL, SPLIT_KIND, SCHED, TAIL>(p, sched, idx);
       const int n = w.n(t);
       const int N = C::TURNS ? max(w.n0, w.n1) : n;
       TRACE_EV(EV_ITEM, 1);
@@ -1111,7 +1133,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
         if constexpr (BIAS && C::BIAS_PF4) {  // lanes 0-3: this step's four bias lines, 4-7: the next step's
           if (lane < 8) {
             const float* brow = p.key_bias + static_cast<size_t>(p.div_heads.div(w.bh(t))) * p.key_bias_stride;
-            const int pf = (w.jb + j) * 128 + 32 * lane;
+            const int pf = (w.jbt(t) + j) * 128 + 32 * lane;
             if (pf < p.seq_kv) asm volatile("prefetch.global.L1 [%0];" ::"l"(brow + pf));
           }
         }
@@ -1145,7 +1167,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           reg_fence(*reinterpret_cast<uint32_t(*)[64]>(&s[0]));
           tmem_ld_32x32b_x32(tS + 64, *reinterpret_cast<uint32_t(*)[32]>(&s[64]));
           tmem_ld_32x32b_x32(tS + 96, *reinterpret_cast<uint32_t(*)[32]>(&s[96]));
-          const int rem0 = lim - (w.jb + j) * 128;
+          const int rem0 = lim - (w.jbt(t) + j) * 128;
           if (!BIAS && rem0 >= 64) {
             float a0 = -INFINITY, a1 = -INFINITY, a2 = -INFINITY, a3 = -INFINITY;
 #pragma unroll
@@ -1175,14 +1197,14 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           tc_fence_before();
           FMHA_ROW_ARRIVE(S_FREE);
         }
-        const int rem = lim - (w.jb + j) * 128;
+        const int rem = lim - (w.jbt(t) + j) * 128;
         // 32-key chunks no row of this warp can see are skipped: their P is stored as zeros
-        const int rem_w = lim_w - (w.jb + j) * 128;
+        const int rem_w = lim_w - (w.jbt(t) + j) * 128;
         if constexpr (BIAS) {  // s' = s + bias / scale (R20), 32 keys at a time; L1-resident, the
                                // next step's keys prefetched (every softmax warp reads the same row)
           const int b = p.div_heads.div(w.bh(t));
           const float* brow = p.key_bias + static_cast<size_t>(b) * p.key_bias_stride;
-          const int key0 = (w.jb + j) * 128;
+          const int key0 = (w.jbt(t) + j) * 128;
           // a step's 128 keys are 512 B = four 128-B lines (BIAS_PF4 prefetches all of this and the
           // next step's; otherwise only the next step's first line, and the other three miss L1)
           if constexpr (C::BIAS_PF4) {
@@ -1224,7 +1246,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           const int bb = t ? w.bat1 : w.bat0, hh = t ? w.head1 : w.head;
           const uint4* brow = reinterpret_cast<const uint4*>(
               p.attn_bias + bb * p.ab_sb + hh * p.ab_sh + static_cast<long long>(min(qi, p.seq_q - 1)) * p.ab_sq);
-          const int c80 = (w.jb + j) * 16;  // first 8-key group of this step
+          const int c80 = (w.jbt(t) + j) * 16;  // first 8-key group of this step
           const float2 is2 = make_float2(p.inv_scale, p.inv_scale);
 #pragma unroll
           for (int q = 0; q < 4; ++q) {
@@ -1486,7 +1508,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
       if constexpr (TAIL) reinterpret_cast<float*>(smem + C::OFF_MREF)[t * 128 + row] = (m_ref == -INFINITY) ? -INFINITY : m_ref * c;
       if constexpr (SPLIT) {  // this split's row statistics (rows inside the sequence only)
         if (qi < p.seq_q) {
-          const size_t o = (static_cast<size_t>(w.split) * p.num_units + w.bh(t)) * p.seq_q + qi;
+          const size_t o = (static_cast<size_t>(w.splt(t)) * p.num_units + w.bh(t)) * p.seq_q + qi;
           p.ws_m[o] = (m_ref == -INFINITY) ? -INFINITY : m_ref * c;
           if constexpr (!C::LSUM_MMA) p.ws_l[o] = l;  // (LSUM_MMA: the epilogue reads l from TMEM)
         }
@@ -1513,7 +1535,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
     // (which lived in local memory)
     uint32_t ofbits = 0, lbits = 0;
     for (int kk = 0, idx; (idx = item_at<SCHED>(p, sched, kk)) >= 0; ++kk) {
-      const WorkItem w = get_item<PAIRX, VL, SPLIT, SCHED, TAIL>(p, sched, idx);
+      const WorkItem w = get_item<PAIRX, VL, SPLIT_KIND, SCHED, TAIL>(p, sched, idx);
       // ------------------------------------------------------------ epilogue per tile (a9)
 #pragma unroll 1
       for (int t = 0; t < 2; ++t) {
@@ -1572,7 +1594,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           }
           if constexpr (SPLIT) {
             const int qi = w.row0(t) + row;
-            if (qi < p.seq_q) p.ws_l[(static_cast<size_t>(w.split) * p.num_units + w.bh(t)) * p.seq_q + qi] = l;
+            if (qi < p.seq_q) p.ws_l[(static_cast<size_t>(w.splt(t)) * p.num_units + w.bh(t)) * p.seq_q + qi] = l;
           }
         }
         const float inv_l = (l > 0.f) ? 1.f / l : 0.f;  // fully masked row -> 0 (R4)
@@ -1598,7 +1620,7 @@ __global__ void __launch_bounds__(512, 1) fmha_fwd_sm100(const __grid_constant__
           if constexpr (SPLIT) {  // unnormalised fp32 partial O of this split, rows inside the sequence
             const int qi = w.row0(t) + row;
             if (qi < p.seq_q) {
-              float* dst = p.ws_o + ((static_cast<size_t>(w.split) * p.num_units + w.bh(t)) * p.seq_q + qi) * D + col0;
+              float* dst = p.ws_o + ((static_cast<size_t>(w.splt(t)) * p.num_units + w.bh(t)) * p.seq_q + qi) * D + col0;
 #pragma unroll
               for (int u = 0; u < 8; ++u)
                 st_global_v4(dst + 4 * u, o[4 * u], o[4 * u + 1], o[4 * u + 2], o[4 * u + 3]);
