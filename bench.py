@@ -276,6 +276,8 @@ def main():
             dist.barrier()
         torch.cuda.synchronize()
         lead_in(stream)
+        for _ in range(int(os.environ.get("B200_BENCH_WARM_REPLAYS", "0"))):  # (A/B of device warm-up)
+            graph.replay()
         ev0.record(stream)
         graph.replay()
         ev1.record(stream)
