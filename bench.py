@@ -266,11 +266,13 @@ def main():
     with torch.cuda.graph(graph):
         for i in range(args.steps):
             step(i)
-    graph.replay()
-    torch.cuda.synchronize()
-
+    # (the NVML sampler is initialised before the upload replay, so the device is not left idle for the
+    # NVML start-up between that replay and the timed one: an idle gap costs the first launches after it
+    # a few % -- DESIGN.md §7)
     sampler = ClockSampler(local)
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    graph.replay()
+    torch.cuda.synchronize()
     with sampler:
         if dist:
             dist.barrier()
@@ -437,10 +439,10 @@ def run_mlp(args, world, rank, local):
     with torch.cuda.graph(graph):
         for _ in range(args.steps):
             step()
+    stream = torch.cuda.current_stream(dev)
+    sampler = ClockSampler(local)  # (before the upload replay: no idle NVML start-up gap before timing)
     graph.replay()
     torch.cuda.synchronize()
-    stream = torch.cuda.current_stream(dev)
-    sampler = ClockSampler(local)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with sampler:
         torch.cuda.synchronize()
@@ -500,10 +502,10 @@ def run_varlen(args, world, rank, local):
     with torch.cuda.graph(graph):
         for i in range(args.steps):
             step(i)
+    stream = torch.cuda.current_stream(dev)
+    sampler = ClockSampler(local)  # (before the upload replay: no idle NVML start-up gap before timing)
     graph.replay()
     torch.cuda.synchronize()
-    stream = torch.cuda.current_stream(dev)
-    sampler = ClockSampler(local)
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with sampler:
         if dist:
@@ -674,9 +676,9 @@ def run_layer(args, world, rank, local):
     with torch.cuda.graph(graph):
         for _ in range(args.steps):
             step()
+    sampler = ClockSampler(local)  # (before the upload replay: no idle NVML start-up gap before timing)
     graph.replay()
     torch.cuda.synchronize()
-    sampler = ClockSampler(local)
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with sampler:
         if dist:
