@@ -700,11 +700,18 @@ int fmha_fwd_from_host(int dtype, const void* hQ, const void* hK, const void* hV
   // created once per thread and device and reused (thread-local, so concurrent callers on other
   // threads never share them).
   cudaError_t e;
-  const int chunks = std::min(batch, 4);
+  // B200_E2E_CHUNKS: A/B of the pipelining depth (BERT-large-512 e2e: 4 chunks 15.5 TFLOP/s, 8 15.0-15.1,
+  // 16 13.3-13.6 -- smaller copies lose more PCIe efficiency than the shorter tail gains)
+  static const int max_chunks = [] {
+    const char* v = std::getenv("B200_E2E_CHUNKS");
+    const int c = v ? std::atoi(v) : 4;
+    return (c >= 1 && c <= 16) ? c : 4;
+  }();
+  const int chunks = std::min(batch, max_chunks);
   const size_t qb1 = qb / batch, kvb1 = kvb / batch;  // bytes per batch element
   struct HostPipe {
     cudaStream_t sh = nullptr, sc = nullptr, sd = nullptr;
-    cudaEvent_t start = nullptr, d = nullptr, h[4] = {}, c[4] = {};
+    cudaEvent_t start = nullptr, d = nullptr, h[16] = {}, c[16] = {};
     bool ok = false;
   };
   thread_local HostPipe pipes[64];
@@ -717,7 +724,7 @@ int fmha_fwd_from_host(int dtype, const void* hQ, const void* hK, const void* hV
               cudaStreamCreateWithFlags(&hp.sd, cudaStreamNonBlocking) == cudaSuccess &&
               cudaEventCreateWithFlags(&hp.start, cudaEventDisableTiming) == cudaSuccess &&
               cudaEventCreateWithFlags(&hp.d, cudaEventDisableTiming) == cudaSuccess;
-    for (int c = 0; ok && c < 4; ++c)
+    for (int c = 0; ok && c < 16; ++c)
       ok = cudaEventCreateWithFlags(&hp.h[c], cudaEventDisableTiming) == cudaSuccess &&
            cudaEventCreateWithFlags(&hp.c[c], cudaEventDisableTiming) == cudaSuccess;
     if (!ok) return cuda_fail(cudaGetLastError(), "fmha_fwd_from_host streams/events");
